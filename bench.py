@@ -1,0 +1,378 @@
+#!/usr/bin/env python
+"""Headline benchmark: SpMV GFLOP/s and effective HBM GB/s (% of roofline) of
+BRO formats vs the in-repo uncompressed ELL/HYB kernels (BASELINE.json).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C5]
+                  [--impl ours|reference] [--dtype f64|f32]
+
+A step is one pass of the hot path: one bro_spmv (BRO-ELL: one kernel; BRO-HYB:
+ELL kernel + COO kernel + fix-up) over the resident matrix; for N > 1 also the
+NCCL allgather of the y blocks (row-block iteration of a CG loop).  Default
+workload: C5 (3D 27-point stencil on 200^3, 8M rows, 213.8M nnz, fp64,
+BRO-ELL) — the largest config, the one BASELINE.json runs at 1/2/4/8 GPUs.
+Its 2.0 GB working set exceeds the 126 MB L2, so no flush is needed between
+steps.  Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "SpMV GFLOP/s and effective HBM GB/s (% of roofline) vs uncompressed ELL/HYB"
+WORKLOADS = {
+    "C1": (1, "ell"), "C2": (2, "ell"), "C3": (3, "hyb"), "C4": (4, "hyb"), "C5": (5, "ell"),
+}
+L2_BYTES = 126 * 2**20
+FALLBACK_HBM = 6650.0
+
+# SMI throttle-reason bits (nvml clocks_event_reasons)
+REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+           0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+           0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+           0x100: "display_clock_setting"}
+
+
+def parse_args():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=2000)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--workload", default="C5", choices=sorted(WORKLOADS))
+    ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--vec-words", type=int, default=4)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--flush-l2", action="store_true", help="write a 2xL2 buffer between steps")
+    return ap.parse_args()
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    return FALLBACK_HBM, "fallback"
+
+
+def load_workload(name, dtype, lib=None):
+    """Generate the config (seeded) and apply BAR (method 0) for C4."""
+    from gen import make_config, permute_rows
+    cfg, fmt = WORKLOADS[name]
+    A = make_config(cfg, dtype)
+    if cfg == 4 and lib is not None:
+        perm = lib.bro_reorder_bar(A.m, A.n, A.row_ptr, A.col, dtype=dtype, method=0)
+        A = permute_rows(A, perm)
+    return A, fmt
+
+
+class ClockSampler:
+    """nvidia-smi sampling during the timed region (median SM clock + reasons)."""
+
+    def __init__(self, index=0):
+        self.index = index
+        self.proc = None
+        self.path = None
+
+    def start(self):
+        import tempfile
+        self.path = tempfile.mktemp(suffix=".csv")
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active")
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                 "-lms", "50"], stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+            time.sleep(0.4)
+        except (OSError, FileNotFoundError):
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        time.sleep(0.1)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        rows = []
+        with open(self.path) as f:
+            for line in f:
+                parts = [p.strip() for p in line.split(",")]
+                if len(parts) < 4:
+                    continue
+                try:
+                    rows.append((float(parts[0]), float(parts[1]), float(parts[2]), int(parts[3], 16)))
+                except ValueError:
+                    continue
+        os.unlink(self.path)
+        if not rows:
+            return None
+        loaded = [r for r in rows if not (r[3] & 0x1)] or rows
+        sm = sorted(r[0] for r in loaded)
+        mask = 0
+        for r in loaded:
+            mask |= r[3]
+        return {"sm_mhz": sm[len(sm) // 2], "sm_max_mhz": max(r[1] for r in rows),
+                "power_w_max": max(r[2] for r in loaded), "samples": len(loaded),
+                "reasons": [v for k, v in REASONS.items() if mask & k and k != 0x1]}
+
+
+def cpu_oracle_baseline(A, x, target_s=12.0, max_rows=None):
+    """The oracle's csr_spmv (as it stands, single core) on a bounded row
+    sample of the same workload; GFLOP/s over the sample."""
+    from oracle import spmv as ospmv
+    m = A.m if max_rows is None else min(A.m, max_rows)
+    rows = m
+    # size the sample so one call is ~target_s/3
+    probe = min(m, 200_000)
+    t0 = time.perf_counter()
+    ospmv.csr_spmv(A.row_ptr[:probe + 1], A.col[:A.row_ptr[probe]], A.vals[:A.row_ptr[probe]], x)
+    dt = max(time.perf_counter() - t0, 1e-6)
+    rows = int(min(m, probe * (target_s / 3) / dt))
+    nnz = int(A.row_ptr[rows])
+    times = []
+    for _ in range(3):
+        t0 = time.perf_counter()
+        ospmv.csr_spmv(A.row_ptr[:rows + 1], A.col[:nnz], A.vals[:nnz], x)
+        times.append(time.perf_counter() - t0)
+    t = float(np.median(times))
+    return {"value": 2.0 * nnz / t / 1e9, "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+            "sample": f"rows [0,{rows}) of the workload ({nnz} nnz), median of 3 calls, "
+                      f"np.longdouble accumulation, of {os.cpu_count()} host cores"}
+
+
+def time_steps(fn, steps, warmup, stream, flush=None):
+    """Per-step CUDA-event durations on `stream` (ms)."""
+    import torch
+    for _ in range(warmup):
+        fn()
+    torch.cuda.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    for s, e in ev:
+        if flush is not None:
+            flush()
+        s.record(stream)
+        fn()
+        e.record(stream)
+    torch.cuda.synchronize()
+    return np.array([s.elapsed_time(e) for s, e in ev])
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle (the only reference this paper-only
+    tier has), as it stands, on the host cores; rank 0 only."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    dtype = np.float64 if args.dtype == "f64" else np.float32
+    A, fmt = load_workload(args.workload, dtype)
+    from gen import make_x
+    x = make_x(A.n, WORKLOADS[args.workload][0], dtype)
+    from oracle import spmv as ospmv
+    # each step: a bounded row sample (~1 s of oracle work)
+    probe = min(A.m, 100_000)
+    t0 = time.perf_counter()
+    ospmv.csr_spmv(A.row_ptr[:probe + 1], A.col[:A.row_ptr[probe]], A.vals[:A.row_ptr[probe]], x)
+    dt = max(time.perf_counter() - t0, 1e-6)
+    rows = int(min(A.m, probe * 1.0 / dt))
+    nnz = int(A.row_ptr[rows])
+    for _ in range(args.warmup):
+        ospmv.csr_spmv(A.row_ptr[:rows + 1], A.col[:nnz], A.vals[:nnz], x)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        ospmv.csr_spmv(A.row_ptr[:rows + 1], A.col[:nnz], A.vals[:nnz], x)
+    t = time.perf_counter() - t0
+    val = 2.0 * nnz * args.steps / t / 1e9
+    sample = f"rows [0,{rows}) of {args.workload} ({nnz} nnz) per step"
+    out = {"impl": "reference", "metric": METRIC, "value": val, "unit": "GFLOP/s", "n_gpus": args.gpus,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t / args.steps,
+           "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": args.dtype,
+           "data": "synthetic", "config": {"workload": args.workload, "format": "CSR (oracle)"},
+           "cpu_baseline": {"value": val, "unit": "GFLOP/s", "cores": 1, "kind": "oracle", "sample": sample},
+           "e2e": {"value": val, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    args = parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+    import torch
+    import torch.distributed as dist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus and world > 1:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    import paper_conf_sc_tangtrwckgtw13_b200 as P
+    from paper_conf_sc_tangtrwckgtw13_b200.dist import RowBlockSpmv, choose_partition
+    from gen import make_x
+
+    dtype = np.float64 if args.dtype == "f64" else np.float32
+    tdt = torch.float64 if dtype == np.float64 else torch.float32
+    cfg, fmt = WORKLOADS[args.workload]
+    A, fmt = load_workload(args.workload, dtype, P)
+    x_host = make_x(A.n, cfg, dtype)
+    bounds = choose_partition(A.row_ptr, world)
+    stream = torch.cuda.current_stream(dev)
+    x = torch.from_numpy(x_host).to(dev)
+
+    blk = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=1, dtype=dtype, bounds=bounds,
+                       vec_words=args.vec_words)
+    base = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=0, dtype=dtype, bounds=bounds)
+    info, binfo = blk.mat.info, base.mat.info
+    launches = 1 if info["nnz_coo"] == 0 else 3  # ELL kernel (+ COO kernel + fix-up)
+    flush_buf = torch.empty(2 * L2_BYTES // 4, dtype=torch.int32, device=dev) if args.flush_l2 else None
+    flush = (lambda: flush_buf.fill_(1)) if args.flush_l2 else None
+
+    if world > 1:
+        def step():
+            blk.step(x, stream)
+
+        def step_base():
+            base.step(x, stream)
+    else:
+        def step():
+            blk.spmv(x, stream)
+
+        def step_base():
+            base.spmv(x, stream)
+
+    # --- timed region (ours) with clock sampling
+    clocks = ClockSampler(local) if rank == 0 else None
+    if clocks:
+        clocks.start()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    per_step = time_steps(step, args.steps, args.warmup, stream, flush)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ck = clocks.stop() if clocks else None
+    total_ms = float(per_step.sum())
+    # kernel-only duration (SpMV launch without the allgather) for the roofline
+    kern = time_steps(lambda: blk.spmv(x, stream), min(args.steps, 500), 3, stream, flush)
+    kern_ms = float(np.mean(kern))
+    base_ms = float(np.mean(time_steps(step_base, min(args.steps, 500), args.warmup, stream, flush)))
+    base_kern_ms = float(np.mean(time_steps(lambda: base.spmv(x, stream), min(args.steps, 500), 3,
+                                            stream, flush)))
+    if world > 1:
+        t = torch.tensor([total_ms, base_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms, base_ms = float(t[0]), float(t[1])
+
+    # --- end to end through the C ABI with pinned host buffers (rank 0 / N=1 path)
+    e2e = None
+    if not args.no_e2e:
+        xh = torch.from_numpy(x_host).pin_memory()
+        yh = torch.empty(blk.mat.m, dtype=tdt).pin_memory()
+        xh_np, yh_np = xh.numpy(), yh.numpy()
+        P.bro_spmv_host(blk.mat.h, xh_np, yh_np, stream.cuda_stream)  # warm
+        e2e_steps = max(3, min(args.steps, 30))
+        if world > 1:
+            dist.barrier()
+        t0e, t1e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        t0e.record(stream)
+        for _ in range(e2e_steps):
+            P.bro_spmv_host(blk.mat.h, xh_np, yh_np, stream.cuda_stream)
+        t1e.record(stream)
+        torch.cuda.synchronize()
+        e2e_ms = t0e.elapsed_time(t1e) / e2e_steps
+        if world > 1:
+            t = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e2e_ms = float(t[0])
+        isz = np.dtype(dtype).itemsize
+        e2e = {"value": 2.0 * A.nnz / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s",
+               "h2d_bytes_per_step": int(A.n * isz), "d2h_bytes_per_step": int(blk.mat.m * isz),
+               "ms_per_step": e2e_ms,
+               "path": "bro_spmv_host: pinned x H2D + bro_spmv + y D2H + stream sync, per rank"}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    peak, peak_kind = measured_peaks()
+    alg_bytes = info["algorithmic_bytes"]
+    achieved = alg_bytes / (kern_ms * 1e-3) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        with open(tp) as f:
+            tr = json.load(f).get(f"{args.workload}:{args.dtype}:bro:{world}")
+        if tr:
+            traffic = tr
+    value = 2.0 * A.nnz / (total_ms / args.steps * 1e-3) / 1e9
+    base_value = 2.0 * A.nnz / (base_ms * 1e-3) / 1e9
+    cpu = None
+    if not args.no_cpu_baseline and world == 1:
+        cpu = cpu_oracle_baseline(A, x_host)
+    bro_name = {"ell": "BRO-ELL", "hyb": "BRO-HYB", "coo": "BRO-COO"}[fmt]
+    out = {
+        "metric": METRIC,
+        "value": value,
+        "unit": "GFLOP/s",
+        "n_gpus": world,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": total_ms / args.steps,
+        "higher_is_better": True,
+        "scaling": "strong",
+        "vs_baseline": None,
+        "dtype": args.dtype,
+        "data": "synthetic",
+        "config": {
+            "workload": f"{args.workload}: " + {1: "2D 5-point Laplacian 64x64", 2: "FEM banded 62,424 rows",
+                                                3: "webbase-like 1,000,005 rows", 4: "random-block 2M rows, BAR-reordered",
+                                                5: "3D 27-point stencil 200^3"}[cfg],
+            "format": bro_name, "m": A.m, "n": A.n, "nnz": A.nnz,
+            "vec_words": args.vec_words,
+            "l2": ("flushed (2x L2 write) before every step" if args.flush_l2 else
+                   ("inputs larger than L2" if alg_bytes > 2 * L2_BYTES else "L2-resident (warm)")),
+            "parallelism": f"row-block x{world}" + (" + NCCL allgather of y per step" if world > 1 else ""),
+            "eta_stream": info["eta_stream"], "eta_total": info["eta_total"],
+        },
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic,
+                     "peak_kind": peak_kind,
+                     "kernel": f"bro_ell_spmv<{'double' if dtype == np.float64 else 'float'},V={args.vec_words}>"
+                     if fmt == "ell" else "bro_ell_spmv + coo_spmv + coo_fixup",
+                     "algorithmic_bytes_per_launch": alg_bytes, "kernel_ms": kern_ms,
+                     "frac_of_8TBps_spec": achieved / 8000.0},
+        "uncompressed": {"format": {"ell": "ELLPACK", "hyb": "HYB", "coo": "COO"}[fmt], "value": base_value,
+                         "unit": "GFLOP/s", "kernel_ms": base_kern_ms,
+                         "algorithmic_bytes": binfo["algorithmic_bytes"],
+                         "achieved_GBps": binfo["algorithmic_bytes"] / (base_kern_ms * 1e-3) / 1e9,
+                         "speedup_bro": value / base_value},
+        "gpu_launches": int(launches * args.steps),
+        "clocks": ck,
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gflops_kernel_only": 2.0 * A.nnz / world / (kern_ms * 1e-3) / 1e9 if world == 1 else None,
+    }
+    print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

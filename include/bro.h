@@ -1,0 +1,211 @@
+/*
+ * bro.h — C ABI of the B200-native BRO SpMV library (libbro.so).
+ *
+ * Implements the data-parallel hot path of Tang et al., "Accelerating Sparse
+ * Matrix-Vector Multiplication on GPUs using Bit-Representation-Optimized
+ * Schemes", SC'13:  y = A.x  over BRO-ELL (Alg. 1
+ * P:L128-138), BRO-COO and BRO-HYB, plus the
+ * uncompressed ELLPACK / COO / HYB baselines the paper compares against
+ * (P:L51-81).
+ *
+ * Problem statement followed by the boundary:
+ *   - A is fixed across the iterations of an iterative solver, so compression
+ *     runs ONCE, offline, on the host, inside bro_create_*;
+ *   - decompression runs online on the GPU, inside every bro_spmv;
+ *   - host<->device transfers are not part of bro_spmv (bro_spmv_host is the
+ *     end-to-end variant that includes them).
+ *
+ * Conventions
+ *   - All functions are extern "C", never throw, and return bro_status_t.
+ *     On error a thread-local message is available from bro_last_error().
+ *   - Matrices are given as canonical CSR: row_ptr int64[m+1] with
+ *     row_ptr[0] = 0 and non-decreasing; col_idx int32[nnz] 0-based, in
+ *     [0, n) and STRICTLY increasing within each row (a repeated column would
+ *     encode a zero delta, which BRO-ELL reserves for "invalid");
+ *     vals float or double [nnz] (dtype).  m, n < 2^31.
+ *   - Host input arrays are borrowed only for the duration of the call (they
+ *     are validated, encoded and copied; the caller keeps ownership).
+ *   - A handle owns all of its device memory until bro_destroy.
+ *   - Device vectors passed to bro_spmv are caller-owned, of the handle's
+ *     dtype, resident on the handle's device: x has n elements, y has m.
+ *   - bro_stream_t is a cudaStream_t (struct CUstream_st*); NULL means the
+ *     legacy default stream.  PyTorch passes
+ *     torch.cuda.current_stream().cuda_stream.
+ *
+ * Encoded layout (bit-exact):
+ *   BRO-ELL, slice height h = 32 rows (one warp per slice), sym_len = 32:
+ *     colptr[t]  = sum_{t'<t} l_t'       (l_t = num_col of slice t)
+ *     symptr[t]  = sum_{t'<t} S_t'       (S_t = 32-bit symbols per row stream)
+ *     bit_alloc[colptr[t] + j] = b_{t,j} (b_p implied by S_t)
+ *     symbol q of row r of slice t at words[32*symptr[t] + place(r,q,S_t,V)]
+ *     value of slot (r,j) of slice t at vals[32*colptr[t] + place(r,j,l_t,Vv)]
+ *     place(r,q,S,V) = 32*V*(q/V) + r*V + q%V          if q/V < S/V
+ *                    = 32*V*F + r*(S-V*F) + (q-V*F)    otherwise (F = S/V)
+ *     V = opts.vec_words (1 = the paper's comp_str_i[q*h+tid]), Vv = 16/sizeof(val).
+ *     Row streams are concatenated b-bit deltas, most significant bit first,
+ *     delta_0 = col_0 + 1, delta_j = col_j - col_{j-1}, 0 = padding.
+ *   BRO-COO, intervals of 32*T entries (T = opts.coo_T = 32): entry
+ *     i*32*T + 32*t + lane is element (t, lane); each lane's rows are delta
+ *     coded down t from base_row[i] with one width width[i]; lane
+ *     word q at coo_words[32*coo_symptr[i] + place(lane,q,S_i,V)].
+ *
+ * Thread safety: distinct handles may be used concurrently; one handle must
+ * not be used by two threads at once.
+ */
+#ifndef BRO_H_
+#define BRO_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define BRO_VERSION 1
+/* device id that builds a host-only handle: encoded on the host, exportable,
+ * never uploaded; bro_spmv on it returns BRO_ERR_UNSUPPORTED (no CPU path). */
+#define BRO_DEVICE_HOST_ONLY (-1)
+
+typedef struct bro_matrix_s* bro_matrix_t;
+typedef struct CUstream_st* bro_stream_t;
+
+typedef enum { BRO_FP32 = 0, BRO_FP64 = 1 } bro_dtype_t;
+
+typedef enum {
+  BRO_OK = 0,
+  BRO_ERR_ARG = 1,         /* null pointer, bad option, aliasing x == y, buffer too small */
+  BRO_ERR_INDEX = 2,       /* column out of range, unsorted or repeated column, bad row_ptr */
+  BRO_ERR_SHAPE = 3,       /* m or n out of range (>= 2^31 or negative) */
+  BRO_ERR_OOM = 4,         /* host or device allocation failed */
+  BRO_ERR_CUDA = 5,        /* a CUDA runtime call or kernel launch failed */
+  BRO_ERR_UNSUPPORTED = 6  /* option or operation not supported by this handle */
+} bro_status_t;
+
+typedef struct {
+  int32_t slice_h;   /* BRO-ELL slice height h. Must be 32 (one warp per slice). */
+  int32_t sym_bits;  /* sym_len. Must be 32. */
+  int32_t vec_words; /* V: 1, 2 or 4 symbols per lane chunk (4 = 16-byte loads). Default 4. */
+  int32_t coo_T;     /* BRO-COO steps per interval (interval = 32*T entries). Must be 32. */
+  int64_t hyb_K;     /* HYB dividing column; -1 = the "less than a third" rule. */
+  int32_t codec;     /* 1 = BRO compressed formats; 0 = uncompressed ELL/COO/HYB baseline. */
+  int32_t reserved;  /* must be 0 */
+} bro_opts_t;
+
+typedef struct {
+  int64_t m, n, nnz;
+  int32_t dtype;              /* bro_dtype_t */
+  int32_t codec;              /* 1 BRO, 0 uncompressed */
+  int32_t format;             /* 0 ELL, 1 COO, 2 HYB */
+  int32_t vec_words;
+  int64_t K;                  /* ELL width bound: HYB K, or max row length for ELL */
+  int64_t nnz_ell, nnz_coo;   /* entries in the ELL part and in the COO part */
+  int64_t n_slices;           /* BRO-ELL slices s = ceil(m/32) (0 without an ELL part) */
+  int64_t ell_slots;          /* value slots of the ELL part: 32*colptr[s] (BRO) or K*pitch (plain) */
+  int64_t ell_pitch;          /* plain ELL column pitch (m rounded up to 32) */
+  int64_t n_intervals;        /* COO intervals ceil(nnz_coo / (32*T)) */
+  int64_t ell_stream_bytes;   /* BRO-ELL compressed words (C of P:L246 for the ELL part) */
+  int64_t coo_stream_bytes;   /* BRO-COO compressed row words */
+  int64_t meta_bytes;         /* colptr, symptr, bit_alloc, COO headers */
+  int64_t index_bytes;        /* all stored index data: streams + raw col/row arrays + metadata */
+  int64_t value_bytes;        /* stored values including ELL padding */
+  int64_t device_bytes;       /* device memory held by the handle */
+  int64_t algorithmic_bytes;  /* bytes one bro_spmv must move: stored arrays + n*sizeof(x) + m*sizeof(y) */
+  int64_t orig_index_bytes;   /* O of P:L246: 4*m*K (+ 8*nnz_coo for HYB/COO) */
+  double eta_stream;          /* 1 - C/O, C = compressed streams (+ raw COO col for HYB) */
+  double eta_total;           /* 1 - index_bytes/O (metadata included) */
+  double encode_seconds;      /* host time spent validating + encoding */
+} bro_info_t;
+
+/* Parts of the encoded representation, for bro_export_encoded. */
+typedef enum {
+  BRO_PART_ELL_WORDS = 0,     /* uint32[32*symptr[s]]  BRO-ELL multiplexed stream */
+  BRO_PART_ELL_BIT_ALLOC = 1, /* uint8[colptr[s]]      per-slice per-column widths */
+  BRO_PART_ELL_COLPTR = 2,    /* uint64[s+1] */
+  BRO_PART_ELL_SYMPTR = 3,    /* uint64[s+1] */
+  BRO_PART_ELL_VALS = 4,      /* value[32*colptr[s]]   sliced, interleaved, padding 0 */
+  BRO_PART_COO_WORDS = 5,     /* uint32[32*coo_symptr[nI]] */
+  BRO_PART_COO_BASE_ROW = 6,  /* uint32[nI] */
+  BRO_PART_COO_WIDTH = 7,     /* uint8[nI] */
+  BRO_PART_COO_SYMPTR = 8,    /* uint64[nI+1] */
+  BRO_PART_COO_COL = 9,       /* int32[nnz_coo] (COO order) */
+  BRO_PART_COO_VALS = 10,     /* value[nnz_coo] */
+  BRO_PART_COO_ROW = 11,      /* int32[nnz_coo]  plain COO rows (codec 0) */
+  BRO_PART_PELL_COL = 12,     /* int32[K*pitch]  plain ELL, column-major, -1 = padding (codec 0) */
+  BRO_PART_PELL_VALS = 13     /* value[K*pitch]  plain ELL values (codec 0) */
+} bro_part_t;
+
+/* Fill *opts with the defaults: h 32, sym 32, V 4, T 32, K auto, codec 1. */
+void bro_opts_default(bro_opts_t* opts);
+
+/* Build an ELL-only matrix (BRO-ELL if opts->codec == 1, else ELLPACK with
+ * K = max row length).  device = CUDA ordinal or BRO_DEVICE_HOST_ONLY.
+ * opts may be NULL (defaults).  On success *out owns the encoded matrix. */
+bro_status_t bro_create_ell(int device, bro_dtype_t dtype, int64_t m, int64_t n,
+                            const int64_t* row_ptr, const int32_t* col_idx,
+                            const void* vals, const bro_opts_t* opts, bro_matrix_t* out);
+
+/* Build a COO-only matrix (BRO-COO / plain COO).  Entries must be sorted by
+ * (row, col) with strictly increasing columns within a row. */
+bro_status_t bro_create_coo(int device, bro_dtype_t dtype, int64_t m, int64_t n, int64_t nnz,
+                            const int32_t* row_idx, const int32_t* col_idx,
+                            const void* vals, const bro_opts_t* opts, bro_matrix_t* out);
+
+/* Build a HYB matrix: the first K entries of every row in (BRO-)ELL, the rest
+ * in (BRO-)COO, K from opts->hyb_K or the rule of P:L81 (see bro_hyb_K). */
+bro_status_t bro_create_hyb(int device, bro_dtype_t dtype, int64_t m, int64_t n,
+                            const int64_t* row_ptr, const int32_t* col_idx,
+                            const void* vals, const bro_opts_t* opts, bro_matrix_t* out);
+
+/* y = A.x on `stream` (asynchronous).  y is overwritten (never accumulated);
+ * rows without entries get 0 (Alg. 1 line 22).  x and y must not alias.
+ * Launch errors are returned; device faults surface at the next sync. */
+bro_status_t bro_spmv(bro_matrix_t A, const void* x_dev, void* y_dev, bro_stream_t stream);
+
+/* End-to-end y = A.x with HOST vectors: copies x (n values) host->device,
+ * runs bro_spmv, copies y (m values) device->host and synchronizes `stream`.
+ * Pinned host memory gives full PCIe bandwidth; pageable memory works. */
+bro_status_t bro_spmv_host(bro_matrix_t A, const void* x_host, void* y_host, bro_stream_t stream);
+
+/* Release the handle and all of its memory.  NULL is accepted. */
+bro_status_t bro_destroy(bro_matrix_t A);
+
+/* Sizes, byte counts and space savings of the encoded matrix. */
+bro_status_t bro_get_info(bro_matrix_t A, bro_info_t* info);
+
+/* Copy one encoded part to host memory.  If host_buf is NULL, *nbytes
+ * receives the size; otherwise *nbytes must be >= the size and receives it.
+ * Parts absent from this handle have size 0. */
+bro_status_t bro_export_encoded(bro_matrix_t A, int32_t part, void* host_buf, size_t* nbytes);
+
+/* GPU decode of the index streams (debug/parity surface): d_ell_cols
+ * (int32[info.ell_slots], may be NULL) receives the decoded column of every
+ * ELL slot in V = 1 slot order — slot 32*colptr[t] + 32*j + r for BRO-ELL,
+ * j*pitch + r for plain ELL — or -1 for padding; d_coo_rows (int32[nnz_coo],
+ * may be NULL) receives every COO entry's row.  Asynchronous on `stream`. */
+bro_status_t bro_decode_indices(bro_matrix_t A, int32_t* d_ell_cols, int32_t* d_coo_rows,
+                                bro_stream_t stream);
+
+/* The HYB dividing column K = min{k >= 0 : 3*|{i : len_i > k}| < m}
+ * ("less than a third", pinned by the split of P:L79).  Host only. */
+bro_status_t bro_hyb_K(int64_t m, const int64_t* row_ptr, int64_t* K_out);
+
+/* BRO-aware row reordering (Sec. 3.4), host only.  Writes a
+ * permutation perm[m] (row i of A' = row perm[i] of A, A' = P.A).
+ * method 0 = signature clustering (stable sort by
+ * row length then by the bit-width signature of the row's deltas, O(nnz log m));
+ * method 1 = Algorithm 2 greedy on Eqn. (1) with h = w = 32, alpha = sym_len = 32 and
+ * Omega(c) = 128-byte line of x[c] for the dtype (O(m^2 k / h); m <= 65536,
+ * else BRO_ERR_UNSUPPORTED).  Partitions hold 32 rows except the last. */
+bro_status_t bro_reorder_bar(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                             bro_dtype_t dtype, int32_t method, int64_t* perm_out);
+
+const char* bro_status_str(bro_status_t s);
+/* Message of the last failed call on this thread ("" if none). */
+const char* bro_last_error(void);
+int bro_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BRO_H_ */

@@ -1,0 +1,594 @@
+// C ABI of libbro.so (include/bro.h): validation, host encode, upload, launch.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "../../include/bro.h"
+#include "encode.hpp"
+#include "kernels.cuh"
+
+namespace {
+
+thread_local std::string g_err;
+
+bro_status_t fail(bro_status_t s, const std::string& msg) {
+  g_err = msg;
+  return s;
+}
+
+constexpr int kEllThreads = 256;
+constexpr int kCooThreads = 256;
+constexpr int kPlainThreads = 256;
+
+struct DeviceGuard {
+  int prev = -1, want = -1;
+  explicit DeviceGuard(int d) : want(d) {
+    cudaGetDevice(&prev);
+    if (prev != d) cudaSetDevice(d);
+  }
+  ~DeviceGuard() {
+    if (prev >= 0 && prev != want) cudaSetDevice(prev);
+  }
+};
+
+enum Format { FMT_ELL = 0, FMT_COO = 1, FMT_HYB = 2 };
+
+}  // namespace
+
+struct bro_matrix_s {
+  int device = -1;
+  bool host_only = false;
+  bro_dtype_t dtype = BRO_FP64;
+  int vsize = 8;
+  bro_opts_t opts{};
+  int format = FMT_ELL;
+  int64_t m = 0, n = 0, nnz = 0, K = 0, nnz_ell = 0, nnz_coo = 0;
+  bool has_ell = false, has_coo = false;
+  // host encodings (kept only by host-only handles after create)
+  bro::EllCode ell;
+  bro::PlainEll pell;
+  bro::CooCode coo;
+  int64_t s = 0, ell_words = 0, ell_slots = 0, pitch = 0, nI = 0, coo_words = 0;
+  // device buffers
+  uint32_t* d_words = nullptr;
+  uint8_t* d_bit_alloc = nullptr;
+  uint64_t* d_colptr = nullptr;
+  uint64_t* d_symptr = nullptr;
+  void* d_ell_vals = nullptr;
+  int32_t* d_pell_col = nullptr;
+  uint32_t* d_coo_words = nullptr;
+  uint32_t* d_coo_base = nullptr;
+  uint8_t* d_coo_width = nullptr;
+  uint64_t* d_coo_symptr = nullptr;
+  int32_t* d_coo_row = nullptr;
+  int32_t* d_coo_col = nullptr;
+  void* d_coo_vals = nullptr;
+  void* d_cf = nullptr;
+  void* d_cl = nullptr;
+  int32_t* d_last_row = nullptr;
+  void* d_xs = nullptr;
+  void* d_ys = nullptr;
+  int64_t device_bytes = 0;
+  bro_info_t info{};
+};
+
+namespace {
+
+template <typename P>
+bro_status_t dev_upload(bro_matrix_s* A, P** dst, const void* src, size_t bytes) {
+  *dst = nullptr;
+  if (bytes == 0) return BRO_OK;
+  void* p = nullptr;
+  cudaError_t e = cudaMalloc(&p, bytes);
+  if (e != cudaSuccess) return fail(BRO_ERR_OOM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
+  A->device_bytes += (int64_t)bytes;
+  *dst = static_cast<P*>(p);
+  if (src) {
+    e = cudaMemcpy(p, src, bytes, cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("cudaMemcpy H2D: ") + cudaGetErrorString(e));
+  }
+  return BRO_OK;
+}
+
+void free_device(bro_matrix_s* A) {
+  if (A->host_only || A->device < 0) return;
+  DeviceGuard g(A->device);
+  void* ps[] = {A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr, A->d_ell_vals, A->d_pell_col,
+                A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr, A->d_coo_row,
+                A->d_coo_col, A->d_coo_vals, A->d_cf, A->d_cl, A->d_last_row, A->d_xs, A->d_ys};
+  for (void* p : ps)
+    if (p) cudaFree(p);
+}
+
+bro_status_t check_opts(const bro_opts_t& o) {
+  if (o.slice_h != 32) return fail(BRO_ERR_UNSUPPORTED, "slice_h must be 32 (one warp per slice)");
+  if (o.sym_bits != 32) return fail(BRO_ERR_UNSUPPORTED, "sym_bits must be 32");
+  if (o.vec_words != 1 && o.vec_words != 2 && o.vec_words != 4)
+    return fail(BRO_ERR_ARG, "vec_words must be 1, 2 or 4");
+  if (o.coo_T != 32) return fail(BRO_ERR_UNSUPPORTED, "coo_T must be 32");
+  if (o.codec != 0 && o.codec != 1) return fail(BRO_ERR_ARG, "codec must be 0 or 1");
+  if (o.hyb_K < -1) return fail(BRO_ERR_ARG, "hyb_K must be >= -1");
+  if (o.reserved != 0) return fail(BRO_ERR_ARG, "reserved must be 0");
+  return BRO_OK;
+}
+
+void fill_info(bro_matrix_s* A, double secs) {
+  bro_info_t& I = A->info;
+  std::memset(&I, 0, sizeof(I));
+  const int64_t vs = A->vsize;
+  I.m = A->m; I.n = A->n; I.nnz = A->nnz;
+  I.dtype = A->dtype; I.codec = A->opts.codec; I.format = A->format; I.vec_words = A->opts.vec_words;
+  I.K = A->K; I.nnz_ell = A->nnz_ell; I.nnz_coo = A->nnz_coo;
+  I.n_slices = A->s; I.ell_pitch = A->pitch; I.n_intervals = A->nI;
+  I.encode_seconds = secs;
+  int64_t meta = 0, stream = 0, raw_index = 0, values = 0;
+  if (A->has_ell) {
+    if (A->opts.codec) {
+      I.ell_slots = A->ell_slots;
+      I.ell_stream_bytes = 4 * A->ell_words;
+      meta += 16 * (A->s + 1) + (A->s ? int64_t(A->ell_slots / 32) : 0);  // colptr, symptr, bit_alloc
+      stream += I.ell_stream_bytes;
+      values += A->ell_slots * vs;
+    } else {
+      I.ell_slots = A->K * A->pitch;
+      raw_index += 4 * A->K * A->pitch;
+      values += A->K * A->pitch * vs;
+    }
+  }
+  if (A->has_coo) {
+    if (A->opts.codec) {
+      I.coo_stream_bytes = 4 * A->coo_words;
+      stream += I.coo_stream_bytes;
+      meta += A->nI * (4 + 1) + 8 * (A->nI + 1);  // base_row, width, symptr
+      raw_index += 4 * A->nnz_coo;                // col
+    } else {
+      raw_index += 8 * A->nnz_coo;                // row + col
+      meta += 4 * A->nI;                          // interval first rows
+    }
+    values += A->nnz_coo * vs;
+  }
+  I.meta_bytes = meta;
+  I.index_bytes = stream + raw_index + meta;
+  I.value_bytes = values;
+  I.device_bytes = A->device_bytes;
+  I.algorithmic_bytes = I.index_bytes + values + (A->n + A->m) * vs;
+  const int64_t O = (A->has_ell ? 4 * A->m * A->K : 0) + 8 * A->nnz_coo;
+  I.orig_index_bytes = O;
+  const int64_t C = stream + (A->opts.codec ? 4 * A->nnz_coo : raw_index);
+  I.eta_stream = O > 0 ? 1.0 - double(C) / double(O) : 0.0;
+  I.eta_total = O > 0 ? 1.0 - double(I.index_bytes) / double(O) : 0.0;
+}
+
+// Build the handle from validated CSR + a split point K (ELL part = first
+// min(len, K) entries of each row; COO part = the rest).
+bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const int64_t* row_ptr,
+                   const int32_t* col, const void* vals, const bro_opts_t& o, int format,
+                   int64_t K, bro_matrix_t* out) {
+  auto t0 = std::chrono::steady_clock::now();
+  bro_matrix_s* A = new (std::nothrow) bro_matrix_s();
+  if (!A) return fail(BRO_ERR_OOM, "host allocation failed");
+  A->device = device;
+  A->host_only = device == BRO_DEVICE_HOST_ONLY;
+  A->dtype = dtype;
+  A->vsize = dtype == BRO_FP64 ? 8 : 4;
+  A->opts = o;
+  A->format = format;
+  A->m = m; A->n = n; A->nnz = row_ptr[m];
+  A->K = K;
+  const uint8_t* v8 = static_cast<const uint8_t*>(vals);
+  try {
+    // ELL part
+    if (format != FMT_COO) {
+      A->has_ell = true;
+      bro::RowsView rv;
+      rv.m = m; rv.row_ptr = row_ptr; rv.col = col; rv.vals = v8; rv.vsize = A->vsize; rv.cap = K;
+      int64_t ne = 0;
+      for (int64_t i = 0; i < m; ++i) ne += rv.len(i);
+      A->nnz_ell = ne;
+      if (o.codec) {
+        bro::encode_bro_ell(rv, o.vec_words, 16 / A->vsize, A->ell);
+        A->s = A->ell.s;
+        A->ell_words = (int64_t)A->ell.words.size();
+        A->ell_slots = (int64_t)(A->ell.vals.size() / A->vsize);
+      } else {
+        bro::build_plain_ell(rv, K, A->pell);
+        A->pitch = A->pell.pitch;
+      }
+    }
+    // COO part
+    A->nnz_coo = A->nnz - A->nnz_ell;
+    if (format != FMT_ELL && A->nnz_coo > 0) {
+      A->has_coo = true;
+      std::vector<int32_t> cr, cc;
+      std::vector<uint8_t> cv;
+      cr.reserve(A->nnz_coo); cc.reserve(A->nnz_coo); cv.reserve(size_t(A->nnz_coo) * A->vsize);
+      const int64_t cap = format == FMT_COO ? 0 : K;
+      for (int64_t i = 0; i < m; ++i) {
+        for (int64_t p = row_ptr[i] + cap; p < row_ptr[i + 1]; ++p) {
+          cr.push_back((int32_t)i);
+          cc.push_back(col[p]);
+          cv.insert(cv.end(), v8 + size_t(p) * A->vsize, v8 + size_t(p + 1) * A->vsize);
+        }
+      }
+      if (o.codec)
+        bro::encode_bro_coo(A->nnz_coo, cr.data(), cc.data(), cv.data(), A->vsize, o.coo_T, o.vec_words, A->coo);
+      else
+        bro::build_plain_coo(A->nnz_coo, cr.data(), cc.data(), cv.data(), A->vsize, o.coo_T, A->coo);
+      A->nI = A->coo.nI;
+      A->coo_words = (int64_t)A->coo.words.size();
+    }
+  } catch (const std::bad_alloc&) {
+    delete A;
+    return fail(BRO_ERR_OOM, "host allocation failed during encode");
+  }
+  double secs = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+  if (!A->host_only) {
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
+      delete A;
+      return fail(BRO_ERR_CUDA, "no such CUDA device: " + std::to_string(device));
+    }
+    DeviceGuard g(device);
+    bro_status_t st = BRO_OK;
+#define UP(dst, vec) \
+  if (st == BRO_OK) st = dev_upload(A, &(dst), (vec).data(), (vec).size() * sizeof(*(vec).data()))
+    if (A->has_ell && o.codec) {
+      UP(A->d_words, A->ell.words);
+      UP(A->d_bit_alloc, A->ell.bit_alloc);
+      UP(A->d_colptr, A->ell.colptr);
+      UP(A->d_symptr, A->ell.symptr);
+      if (st == BRO_OK) st = dev_upload(A, &A->d_ell_vals, A->ell.vals.data(), A->ell.vals.size());
+    }
+    if (A->has_ell && !o.codec) {
+      UP(A->d_pell_col, A->pell.col);
+      if (st == BRO_OK) st = dev_upload(A, &A->d_ell_vals, A->pell.vals.data(), A->pell.vals.size());
+    }
+    if (A->has_coo) {
+      UP(A->d_coo_base, A->coo.base_row);
+      UP(A->d_coo_col, A->coo.col);
+      if (st == BRO_OK) st = dev_upload(A, &A->d_coo_vals, A->coo.vals.data(), A->coo.vals.size());
+      if (o.codec) {
+        UP(A->d_coo_words, A->coo.words);
+        UP(A->d_coo_width, A->coo.width);
+        UP(A->d_coo_symptr, A->coo.symptr);
+      } else {
+        UP(A->d_coo_row, A->coo.row);
+      }
+      if (st == BRO_OK) st = dev_upload(A, &A->d_cf, nullptr, size_t(A->nI) * A->vsize);
+      if (st == BRO_OK) st = dev_upload(A, &A->d_cl, nullptr, size_t(A->nI) * A->vsize);
+      if (st == BRO_OK) st = dev_upload(A, &A->d_last_row, nullptr, size_t(A->nI) * 4);
+    }
+#undef UP
+    if (st != BRO_OK) {
+      std::string msg = g_err;
+      free_device(A);
+      delete A;
+      return fail(st, msg);
+    }
+    // host copies are not needed any more (export reads the device copy)
+    fill_info(A, secs);
+    A->ell = bro::EllCode();
+    A->pell = bro::PlainEll();
+    A->coo = bro::CooCode();
+  } else {
+    fill_info(A, secs);
+  }
+  *out = A;
+  return BRO_OK;
+}
+
+bro_status_t common_checks(bro_dtype_t dtype, const bro_opts_t* opts, bro_opts_t* o, bro_matrix_t* out) {
+  if (!out) return fail(BRO_ERR_ARG, "out is NULL");
+  *out = nullptr;
+  if (dtype != BRO_FP32 && dtype != BRO_FP64) return fail(BRO_ERR_ARG, "dtype must be BRO_FP32 or BRO_FP64");
+  if (opts) *o = *opts; else bro_opts_default(o);
+  return check_opts(*o);
+}
+
+template <typename T>
+bro_status_t launch_spmv(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+  using namespace bro::dev;
+  const int V = A->opts.vec_words;
+  if (A->has_ell) {
+    if (A->opts.codec) {
+      if (A->s > 0) {
+        const int warps = kEllThreads / 32;
+        dim3 grid((unsigned)((A->s + warps - 1) / warps));
+        if (V == 4)
+          bro_ell_spmv<T, 4, kEllThreads><<<grid, kEllThreads, 0, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc,
+              A->d_colptr, A->d_symptr, (const T*)A->d_ell_vals, x, y);
+        else if (V == 2)
+          bro_ell_spmv<T, 2, kEllThreads><<<grid, kEllThreads, 0, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc,
+              A->d_colptr, A->d_symptr, (const T*)A->d_ell_vals, x, y);
+        else
+          bro_ell_spmv<T, 1, kEllThreads><<<grid, kEllThreads, 0, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc,
+              A->d_colptr, A->d_symptr, (const T*)A->d_ell_vals, x, y);
+      }
+    } else if (A->m > 0) {
+      dim3 grid((unsigned)((A->m + kPlainThreads - 1) / kPlainThreads));
+      ell_spmv<T, kPlainThreads><<<grid, kPlainThreads, 0, st>>>(A->m, A->K, A->pitch, A->d_pell_col,
+                                                                  (const T*)A->d_ell_vals, x, y);
+    }
+  } else if (A->m > 0) {
+    cudaMemsetAsync(y, 0, size_t(A->m) * sizeof(T), st);
+  }
+  if (A->has_coo && A->nI > 0) {
+    const int warps = kCooThreads / 32;
+    dim3 grid((unsigned)((A->nI + warps - 1) / warps));
+    const int T_ = A->opts.coo_T;
+    if (A->opts.codec) {
+      if (V == 4)
+        coo_spmv<T, 4, true, kCooThreads><<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, A->d_coo_words,
+            A->d_coo_base, A->d_coo_width, A->d_coo_symptr, nullptr, A->d_coo_col, (const T*)A->d_coo_vals, x, y,
+            (T*)A->d_cf, (T*)A->d_cl, A->d_last_row);
+      else if (V == 2)
+        coo_spmv<T, 2, true, kCooThreads><<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, A->d_coo_words,
+            A->d_coo_base, A->d_coo_width, A->d_coo_symptr, nullptr, A->d_coo_col, (const T*)A->d_coo_vals, x, y,
+            (T*)A->d_cf, (T*)A->d_cl, A->d_last_row);
+      else
+        coo_spmv<T, 1, true, kCooThreads><<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, A->d_coo_words,
+            A->d_coo_base, A->d_coo_width, A->d_coo_symptr, nullptr, A->d_coo_col, (const T*)A->d_coo_vals, x, y,
+            (T*)A->d_cf, (T*)A->d_cl, A->d_last_row);
+    } else {
+      coo_spmv<T, 4, false, kCooThreads><<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, nullptr,
+          A->d_coo_base, nullptr, nullptr, A->d_coo_row, A->d_coo_col, (const T*)A->d_coo_vals, x, y,
+          (T*)A->d_cf, (T*)A->d_cl, A->d_last_row);
+    }
+    dim3 g2((unsigned)((A->nI + 255) / 256));
+    coo_fixup<T><<<g2, 256, 0, st>>>(A->nI, A->d_coo_base, A->d_last_row, (const T*)A->d_cf,
+                                     (const T*)A->d_cl, y);
+  }
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("kernel launch: ") + cudaGetErrorString(e));
+  return BRO_OK;
+}
+
+struct PartView {
+  const void* host = nullptr;
+  const void* dev = nullptr;
+  size_t bytes = 0;
+};
+
+PartView part_view(bro_matrix_s* A, int32_t part) {
+  PartView v;
+  const bool bro_ell = A->has_ell && A->opts.codec;
+  const bool plain_ell = A->has_ell && !A->opts.codec;
+  const bool coo = A->has_coo;
+  const bool bro_coo = coo && A->opts.codec;
+  const size_t vs = A->vsize;
+  auto set = [&](const void* h, const void* d, size_t b) { v.host = h; v.dev = d; v.bytes = b; };
+  switch (part) {
+    case BRO_PART_ELL_WORDS: if (bro_ell) set(A->ell.words.data(), A->d_words, 4 * size_t(A->ell_words)); break;
+    case BRO_PART_ELL_BIT_ALLOC: if (bro_ell) set(A->ell.bit_alloc.data(), A->d_bit_alloc, size_t(A->ell_slots / 32)); break;
+    case BRO_PART_ELL_COLPTR: if (bro_ell) set(A->ell.colptr.data(), A->d_colptr, 8 * size_t(A->s + 1)); break;
+    case BRO_PART_ELL_SYMPTR: if (bro_ell) set(A->ell.symptr.data(), A->d_symptr, 8 * size_t(A->s + 1)); break;
+    case BRO_PART_ELL_VALS: if (bro_ell) set(A->ell.vals.data(), A->d_ell_vals, vs * size_t(A->ell_slots)); break;
+    case BRO_PART_COO_WORDS: if (bro_coo) set(A->coo.words.data(), A->d_coo_words, 4 * size_t(A->coo_words)); break;
+    case BRO_PART_COO_BASE_ROW: if (bro_coo) set(A->coo.base_row.data(), A->d_coo_base, 4 * size_t(A->nI)); break;
+    case BRO_PART_COO_WIDTH: if (bro_coo) set(A->coo.width.data(), A->d_coo_width, size_t(A->nI)); break;
+    case BRO_PART_COO_SYMPTR: if (bro_coo) set(A->coo.symptr.data(), A->d_coo_symptr, 8 * size_t(A->nI + 1)); break;
+    case BRO_PART_COO_COL: if (coo) set(A->coo.col.data(), A->d_coo_col, 4 * size_t(A->nnz_coo)); break;
+    case BRO_PART_COO_VALS: if (coo) set(A->coo.vals.data(), A->d_coo_vals, vs * size_t(A->nnz_coo)); break;
+    case BRO_PART_COO_ROW: if (coo && !A->opts.codec) set(A->coo.row.data(), A->d_coo_row, 4 * size_t(A->nnz_coo)); break;
+    case BRO_PART_PELL_COL: if (plain_ell) set(A->pell.col.data(), A->d_pell_col, 4 * size_t(A->K * A->pitch)); break;
+    case BRO_PART_PELL_VALS: if (plain_ell) set(A->pell.vals.data(), A->d_ell_vals, vs * size_t(A->K * A->pitch)); break;
+    default: v.bytes = SIZE_MAX;
+  }
+  return v;
+}
+
+}  // namespace
+
+extern "C" {
+
+void bro_opts_default(bro_opts_t* o) {
+  if (!o) return;
+  o->slice_h = 32;
+  o->sym_bits = 32;
+  o->vec_words = 4;
+  o->coo_T = 32;
+  o->hyb_K = -1;
+  o->codec = 1;
+  o->reserved = 0;
+}
+
+bro_status_t bro_create_ell(int device, bro_dtype_t dtype, int64_t m, int64_t n, const int64_t* row_ptr,
+                            const int32_t* col_idx, const void* vals, const bro_opts_t* opts,
+                            bro_matrix_t* out) {
+  g_err.clear();
+  bro_opts_t o;
+  bro_status_t st = common_checks(dtype, opts, &o, out);
+  if (st) return st;
+  std::string msg = bro::check_csr(m, n, row_ptr, col_idx);
+  if (!msg.empty()) return fail(msg.rfind("shape", 0) == 0 ? BRO_ERR_SHAPE : (row_ptr ? BRO_ERR_INDEX : BRO_ERR_ARG), msg);
+  if (row_ptr[m] > 0 && !vals) return fail(BRO_ERR_ARG, "vals is NULL");
+  int64_t K = 0;
+  for (int64_t i = 0; i < m; ++i) K = std::max(K, row_ptr[i + 1] - row_ptr[i]);
+  return build(device, dtype, m, n, row_ptr, col_idx, vals, o, FMT_ELL, K, out);
+}
+
+bro_status_t bro_create_hyb(int device, bro_dtype_t dtype, int64_t m, int64_t n, const int64_t* row_ptr,
+                            const int32_t* col_idx, const void* vals, const bro_opts_t* opts,
+                            bro_matrix_t* out) {
+  g_err.clear();
+  bro_opts_t o;
+  bro_status_t st = common_checks(dtype, opts, &o, out);
+  if (st) return st;
+  std::string msg = bro::check_csr(m, n, row_ptr, col_idx);
+  if (!msg.empty()) return fail(msg.rfind("shape", 0) == 0 ? BRO_ERR_SHAPE : (row_ptr ? BRO_ERR_INDEX : BRO_ERR_ARG), msg);
+  if (row_ptr[m] > 0 && !vals) return fail(BRO_ERR_ARG, "vals is NULL");
+  const int64_t K = o.hyb_K >= 0 ? o.hyb_K : bro::hyb_K(m, row_ptr);
+  return build(device, dtype, m, n, row_ptr, col_idx, vals, o, FMT_HYB, K, out);
+}
+
+bro_status_t bro_create_coo(int device, bro_dtype_t dtype, int64_t m, int64_t n, int64_t nnz,
+                            const int32_t* row_idx, const int32_t* col_idx, const void* vals,
+                            const bro_opts_t* opts, bro_matrix_t* out) {
+  g_err.clear();
+  bro_opts_t o;
+  bro_status_t st = common_checks(dtype, opts, &o, out);
+  if (st) return st;
+  std::string msg = bro::check_coo(m, n, nnz, row_idx, col_idx);
+  if (!msg.empty()) return fail(msg.rfind("shape", 0) == 0 ? BRO_ERR_SHAPE : BRO_ERR_INDEX, msg);
+  if (nnz > 0 && !vals) return fail(BRO_ERR_ARG, "vals is NULL");
+  std::vector<int64_t> rp(m + 1, 0);
+  for (int64_t e = 0; e < nnz; ++e) rp[row_idx[e] + 1]++;
+  for (int64_t i = 0; i < m; ++i) rp[i + 1] += rp[i];
+  return build(device, dtype, m, n, rp.data(), col_idx, vals, o, FMT_COO, 0, out);
+}
+
+bro_status_t bro_spmv(bro_matrix_t A, const void* x, void* y, bro_stream_t stream) {
+  if (!A) return fail(BRO_ERR_ARG, "matrix is NULL");
+  if (A->host_only) return fail(BRO_ERR_UNSUPPORTED, "host-only handle: no device copy (there is no CPU SpMV path)");
+  if ((!x && A->n > 0) || (!y && A->m > 0)) return fail(BRO_ERR_ARG, "x or y is NULL");
+  if (x == y && A->m > 0) return fail(BRO_ERR_ARG, "x and y must not alias");
+  DeviceGuard g(A->device);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  if (A->dtype == BRO_FP64) return launch_spmv<double>(A, (const double*)x, (double*)y, st);
+  return launch_spmv<float>(A, (const float*)x, (float*)y, st);
+}
+
+bro_status_t bro_spmv_host(bro_matrix_t A, const void* x_host, void* y_host, bro_stream_t stream) {
+  if (!A) return fail(BRO_ERR_ARG, "matrix is NULL");
+  if (A->host_only) return fail(BRO_ERR_UNSUPPORTED, "host-only handle: no device copy (there is no CPU SpMV path)");
+  if ((!x_host && A->n > 0) || (!y_host && A->m > 0)) return fail(BRO_ERR_ARG, "x or y is NULL");
+  DeviceGuard g(A->device);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  const size_t xb = size_t(A->n) * A->vsize, yb = size_t(A->m) * A->vsize;
+  bro_status_t s = BRO_OK;
+  if (!A->d_xs && xb) s = dev_upload(A, &A->d_xs, nullptr, xb);
+  if (s == BRO_OK && !A->d_ys && yb) s = dev_upload(A, &A->d_ys, nullptr, yb);
+  if (s != BRO_OK) return s;
+  cudaError_t e = xb ? cudaMemcpyAsync(A->d_xs, x_host, xb, cudaMemcpyHostToDevice, st) : cudaSuccess;
+  if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("H2D x: ") + cudaGetErrorString(e));
+  s = bro_spmv(A, A->d_xs, A->d_ys, stream);
+  if (s != BRO_OK) return s;
+  e = yb ? cudaMemcpyAsync(y_host, A->d_ys, yb, cudaMemcpyDeviceToHost, st) : cudaSuccess;
+  if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("D2H y: ") + cudaGetErrorString(e));
+  e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("sync: ") + cudaGetErrorString(e));
+  return BRO_OK;
+}
+
+bro_status_t bro_destroy(bro_matrix_t A) {
+  if (!A) return BRO_OK;
+  free_device(A);
+  delete A;
+  return BRO_OK;
+}
+
+bro_status_t bro_get_info(bro_matrix_t A, bro_info_t* info) {
+  if (!A || !info) return fail(BRO_ERR_ARG, "NULL argument");
+  A->info.device_bytes = A->device_bytes;
+  *info = A->info;
+  return BRO_OK;
+}
+
+bro_status_t bro_export_encoded(bro_matrix_t A, int32_t part, void* host_buf, size_t* nbytes) {
+  if (!A || !nbytes) return fail(BRO_ERR_ARG, "NULL argument");
+  PartView v = part_view(A, part);
+  if (v.bytes == SIZE_MAX) return fail(BRO_ERR_ARG, "unknown part " + std::to_string(part));
+  if (!host_buf) {
+    *nbytes = v.bytes;
+    return BRO_OK;
+  }
+  if (*nbytes < v.bytes) return fail(BRO_ERR_ARG, "buffer too small for part " + std::to_string(part));
+  *nbytes = v.bytes;
+  if (v.bytes == 0) return BRO_OK;
+  if (A->host_only) {
+    std::memcpy(host_buf, v.host, v.bytes);
+    return BRO_OK;
+  }
+  DeviceGuard g(A->device);
+  cudaError_t e = cudaMemcpy(host_buf, v.dev, v.bytes, cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("D2H export: ") + cudaGetErrorString(e));
+  return BRO_OK;
+}
+
+bro_status_t bro_decode_indices(bro_matrix_t A, int32_t* d_ell_cols, int32_t* d_coo_rows, bro_stream_t stream) {
+  using namespace bro::dev;
+  if (!A) return fail(BRO_ERR_ARG, "matrix is NULL");
+  if (A->host_only) return fail(BRO_ERR_UNSUPPORTED, "host-only handle has no device copy");
+  DeviceGuard g(A->device);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  const int V = A->opts.vec_words;
+  if (d_ell_cols && A->has_ell) {
+    if (A->opts.codec) {
+      if (A->s > 0) {
+        dim3 grid((unsigned)((A->s + 7) / 8));
+        if (V == 4) bro_ell_decode<4><<<grid, 256, 0, st>>>(A->s, A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr, d_ell_cols);
+        else if (V == 2) bro_ell_decode<2><<<grid, 256, 0, st>>>(A->s, A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr, d_ell_cols);
+        else bro_ell_decode<1><<<grid, 256, 0, st>>>(A->s, A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr, d_ell_cols);
+      }
+    } else if (A->K * A->pitch > 0) {
+      dim3 grid((unsigned)((A->K * A->pitch + 255) / 256));
+      ell_decode<<<grid, 256, 0, st>>>(A->m, A->K, A->pitch, A->d_pell_col, d_ell_cols);
+    }
+  }
+  if (d_coo_rows && A->has_coo && A->nI > 0) {
+    if (A->opts.codec) {
+      dim3 grid((unsigned)((A->nI + 7) / 8));
+      if (V == 4) bro_coo_decode<4><<<grid, 256, 0, st>>>(A->nnz_coo, A->nI, A->opts.coo_T, A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr, d_coo_rows);
+      else if (V == 2) bro_coo_decode<2><<<grid, 256, 0, st>>>(A->nnz_coo, A->nI, A->opts.coo_T, A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr, d_coo_rows);
+      else bro_coo_decode<1><<<grid, 256, 0, st>>>(A->nnz_coo, A->nI, A->opts.coo_T, A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr, d_coo_rows);
+    } else {
+      cudaMemcpyAsync(d_coo_rows, A->d_coo_row, 4 * size_t(A->nnz_coo), cudaMemcpyDeviceToDevice, st);
+    }
+  }
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("decode launch: ") + cudaGetErrorString(e));
+  return BRO_OK;
+}
+
+bro_status_t bro_hyb_K(int64_t m, const int64_t* row_ptr, int64_t* K_out) {
+  if (!row_ptr || !K_out || m < 0) return fail(BRO_ERR_ARG, "bad argument");
+  *K_out = bro::hyb_K(m, row_ptr);
+  return BRO_OK;
+}
+
+bro_status_t bro_reorder_bar(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                             bro_dtype_t dtype, int32_t method, int64_t* perm_out) {
+  g_err.clear();
+  if (!perm_out) return fail(BRO_ERR_ARG, "perm_out is NULL");
+  if (dtype != BRO_FP32 && dtype != BRO_FP64) return fail(BRO_ERR_ARG, "bad dtype");
+  std::string msg = bro::check_csr(m, n, row_ptr, col_idx);
+  if (!msg.empty()) return fail(msg.rfind("shape", 0) == 0 ? BRO_ERR_SHAPE : BRO_ERR_INDEX, msg);
+  try {
+    if (method == 0) {
+      bro::bar_signature_order(m, row_ptr, col_idx, perm_out);
+      return BRO_OK;
+    }
+    if (method == 1) {
+      std::string err;
+      if (!bro::bar_greedy_order(m, n, row_ptr, col_idx, dtype == BRO_FP64 ? 8 : 4, perm_out, &err))
+        return fail(BRO_ERR_UNSUPPORTED, err);
+      return BRO_OK;
+    }
+  } catch (const std::bad_alloc&) {
+    return fail(BRO_ERR_OOM, "host allocation failed");
+  }
+  return fail(BRO_ERR_ARG, "method must be 0 or 1");
+}
+
+const char* bro_status_str(bro_status_t s) {
+  switch (s) {
+    case BRO_OK: return "BRO_OK";
+    case BRO_ERR_ARG: return "BRO_ERR_ARG";
+    case BRO_ERR_INDEX: return "BRO_ERR_INDEX";
+    case BRO_ERR_SHAPE: return "BRO_ERR_SHAPE";
+    case BRO_ERR_OOM: return "BRO_ERR_OOM";
+    case BRO_ERR_CUDA: return "BRO_ERR_CUDA";
+    case BRO_ERR_UNSUPPORTED: return "BRO_ERR_UNSUPPORTED";
+  }
+  return "BRO_ERR_UNKNOWN";
+}
+
+const char* bro_last_error(void) { return g_err.c_str(); }
+
+int bro_version(void) { return BRO_VERSION; }
+
+}  // extern "C"

@@ -1,0 +1,420 @@
+// Host-side BRO encoder (offline compression on the host CPU).
+//
+// BRO-ELL: per 32-row slice, per column j the width
+// b_j = max Gamma(delta) over the slice's rows, the row streams padded to a
+// multiple of 32 bits, then multiplexed so lane r reads its own symbols with
+// coalesced 16-byte chunk loads.  BRO-COO: per interval of 32*T
+// entries one width for all row deltas.  Multithreaded over slices /
+// intervals (layouts are independent per slice).
+#include "encode.hpp"
+
+#include <algorithm>
+#include <cstring>
+#include <numeric>
+#include <thread>
+#include <unordered_set>
+
+namespace bro {
+
+int num_threads() {
+  unsigned n = std::thread::hardware_concurrency();
+  if (n == 0) n = 1;
+  return (int)std::min(n, 64u);
+}
+
+template <class F>
+static void parallel_for(int64_t n, F&& fn, int64_t grain = 256) {
+  int nt = num_threads();
+  if (n <= grain || nt == 1) {
+    fn(int64_t(0), n);
+    return;
+  }
+  int64_t chunks = std::min<int64_t>(nt, (n + grain - 1) / grain);
+  std::vector<std::thread> th;
+  th.reserve(chunks);
+  for (int64_t c = 0; c < chunks; ++c) {
+    int64_t lo = n * c / chunks, hi = n * (c + 1) / chunks;
+    th.emplace_back([&fn, lo, hi] { fn(lo, hi); });
+  }
+  for (auto& t : th) t.join();
+}
+
+static void exclusive_scan(const std::vector<uint64_t>& cnt, std::vector<uint64_t>& ptr) {
+  ptr.assign(cnt.size() + 1, 0);
+  for (size_t i = 0; i < cnt.size(); ++i) ptr[i + 1] = ptr[i] + cnt[i];
+}
+
+std::string check_csr(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col) {
+  if (m < 0 || n < 0 || m >= (int64_t(1) << 31) || n >= (int64_t(1) << 31))
+    return "shape: m and n must be in [0, 2^31)";
+  if (!row_ptr) return "row_ptr is NULL";
+  if (row_ptr[0] != 0) return "row_ptr[0] != 0";
+  for (int64_t i = 0; i < m; ++i)
+    if (row_ptr[i + 1] < row_ptr[i]) return "row_ptr is not non-decreasing at row " + std::to_string(i);
+  if (row_ptr[m] > 0 && !col) return "col_idx is NULL";
+  std::vector<int64_t> bad(num_threads(), -1);
+  std::vector<int> kind(num_threads(), 0);
+  int nt = num_threads();
+  std::vector<std::thread> th;
+  for (int c = 0; c < nt; ++c) {
+    th.emplace_back([&, c] {
+      int64_t lo = m * c / nt, hi = m * (c + 1) / nt;
+      for (int64_t i = lo; i < hi && bad[c] < 0; ++i) {
+        for (int64_t p = row_ptr[i]; p < row_ptr[i + 1]; ++p) {
+          int32_t cc = col[p];
+          if (cc < 0 || cc >= n) { bad[c] = i; kind[c] = 1; break; }
+          if (p > row_ptr[i] && cc <= col[p - 1]) { bad[c] = i; kind[c] = 2; break; }
+        }
+      }
+    });
+  }
+  for (auto& t : th) t.join();
+  for (int c = 0; c < nt; ++c) {
+    if (bad[c] >= 0)
+      return (kind[c] == 1 ? "column index out of [0, n) in row " : "columns not strictly increasing in row ") +
+             std::to_string(bad[c]);
+  }
+  return "";
+}
+
+std::string check_coo(int64_t m, int64_t n, int64_t nnz, const int32_t* row, const int32_t* col) {
+  if (m < 0 || n < 0 || m >= (int64_t(1) << 31) || n >= (int64_t(1) << 31))
+    return "shape: m and n must be in [0, 2^31)";
+  if (nnz < 0) return "nnz < 0";
+  if (nnz > 0 && (!row || !col)) return "row_idx/col_idx is NULL";
+  for (int64_t e = 0; e < nnz; ++e) {
+    if (row[e] < 0 || row[e] >= m) return "row index out of [0, m) at entry " + std::to_string(e);
+    if (col[e] < 0 || col[e] >= n) return "column index out of [0, n) at entry " + std::to_string(e);
+    if (e > 0) {
+      if (row[e] < row[e - 1]) return "COO entries not sorted by row at entry " + std::to_string(e);
+      if (row[e] == row[e - 1] && col[e] <= col[e - 1])
+        return "columns not strictly increasing within a row at entry " + std::to_string(e);
+    }
+  }
+  return "";
+}
+
+int64_t hyb_K(int64_t m, const int64_t* row_ptr) {
+  // K = min{k >= 0 : 3 * #{rows with len > k} < m}   (reading R12)
+  if (m <= 0) return 0;
+  int64_t maxlen = 0;
+  for (int64_t i = 0; i < m; ++i) maxlen = std::max(maxlen, row_ptr[i + 1] - row_ptr[i]);
+  std::vector<int64_t> hist(maxlen + 1, 0);
+  for (int64_t i = 0; i < m; ++i) hist[row_ptr[i + 1] - row_ptr[i]]++;
+  int64_t at_most = 0;
+  for (int64_t k = 0; k <= maxlen; ++k) {
+    at_most += hist[k];
+    if (3 * (m - at_most) < m) return k;
+  }
+  return maxlen;
+}
+
+// ---------------------------------------------------------------------------
+// BRO-ELL
+// ---------------------------------------------------------------------------
+
+// MSB-first bit writer that emits 32-bit symbols to words[base + place(lane, q)].
+struct SymbolWriter {
+  uint32_t* words;
+  int64_t lane, S, V;
+  uint64_t acc = 0;
+  int nb = 0;
+  int64_t q = 0;
+  void put(uint32_t v, int b) {
+    if (b == 0) return;
+    acc = (acc << b) | v;
+    nb += b;
+    if (nb >= 32) {
+      nb -= 32;
+      words[place(lane, q++, S, V)] = uint32_t(acc >> nb);
+      acc &= (nb ? ((uint64_t(1) << nb) - 1) : 0);
+    }
+  }
+  void flush() {  // append the padding bits b_p (zeros) of P:L114
+    if (nb > 0) {
+      words[place(lane, q++, S, V)] = uint32_t(acc << (32 - nb));
+      nb = 0;
+      acc = 0;
+    }
+  }
+};
+
+void encode_bro_ell(const RowsView& A, int V, int VV, EllCode& out) {
+  const int64_t m = A.m;
+  const int64_t s = (m + kH - 1) / kH;
+  out.s = s;
+  std::vector<uint64_t> ncol(s, 0), nsym(s, 0);
+  // num_col: l_t = longest row of the slice (R9)
+  parallel_for(s, [&](int64_t lo, int64_t hi) {
+    for (int64_t t = lo; t < hi; ++t) {
+      int64_t l = 0;
+      for (int64_t r = t * kH; r < std::min(m, t * kH + kH); ++r) l = std::max(l, A.len(r));
+      ncol[t] = (uint64_t)l;
+    }
+  });
+  exclusive_scan(ncol, out.colptr);
+  out.max_l = s ? (int64_t)*std::max_element(ncol.begin(), ncol.end()) : 0;
+  out.bit_alloc.assign(out.colptr[s], 0);
+  // bit_alloc: b_j = max over rows of Gamma(delta_j)
+  parallel_for(s, [&](int64_t lo, int64_t hi) {
+    for (int64_t t = lo; t < hi; ++t) {
+      uint8_t* ba = out.bit_alloc.data() + out.colptr[t];
+      for (int64_t r = t * kH; r < std::min(m, t * kH + kH); ++r) {
+        const int32_t* c = A.col + A.row_ptr[r];
+        const int64_t len = A.len(r);
+        uint32_t prev1 = 0;  // 1-based previous column, c_{-1} = 0
+        for (int64_t j = 0; j < len; ++j) {
+          uint32_t c1 = uint32_t(c[j]) + 1u;
+          int g = gamma_bits(c1 - prev1);
+          if (g > ba[j]) ba[j] = (uint8_t)g;
+          prev1 = c1;
+        }
+      }
+      uint64_t L = 0;
+      for (uint64_t j = 0; j < ncol[t]; ++j) L += ba[j];
+      nsym[t] = (L + kSym - 1) / kSym;
+    }
+  });
+  exclusive_scan(nsym, out.symptr);
+  out.words.assign(kH * out.symptr[s], 0u);
+  out.vals.resize(size_t(kH) * out.colptr[s] * A.vsize);
+  // pack + multiplex and place values slot-wise
+  parallel_for(s, [&](int64_t lo, int64_t hi) {
+    for (int64_t t = lo; t < hi; ++t) {
+      const uint8_t* ba = out.bit_alloc.data() + out.colptr[t];
+      const int64_t l = (int64_t)ncol[t], S = (int64_t)nsym[t];
+      uint32_t* wbase = out.words.data() + kH * out.symptr[t];
+      uint8_t* vbase = out.vals.data() + size_t(kH) * out.colptr[t] * A.vsize;
+      for (int64_t lane = 0; lane < kH; ++lane) {
+        const int64_t r = t * kH + lane;
+        const int64_t len = r < m ? A.len(r) : 0;
+        const int32_t* c = r < m ? A.col + A.row_ptr[r] : nullptr;
+        SymbolWriter w{wbase, lane, S, V};
+        uint32_t prev1 = 0;
+        for (int64_t j = 0; j < l; ++j) {
+          uint32_t d = 0;  // 0 = invalid (padding)
+          if (j < len) {
+            uint32_t c1 = uint32_t(c[j]) + 1u;
+            d = c1 - prev1;
+            prev1 = c1;
+          }
+          w.put(d, ba[j]);
+        }
+        w.flush();
+        if (r < m) {
+          const uint8_t* src = A.vals + size_t(A.row_ptr[r]) * A.vsize;
+          for (int64_t j = 0; j < len; ++j)
+            std::memcpy(vbase + size_t(place(lane, j, l, VV)) * A.vsize, src + size_t(j) * A.vsize, A.vsize);
+        }
+      }
+    }
+  });
+}
+
+void build_plain_ell(const RowsView& A, int64_t K, PlainEll& out) {
+  out.K = K;
+  out.pitch = (A.m + kH - 1) / kH * kH;
+  out.col.assign(size_t(K) * out.pitch, -1);
+  out.vals.resize(size_t(K) * out.pitch * A.vsize);
+  parallel_for(A.m, [&](int64_t lo, int64_t hi) {
+    for (int64_t r = lo; r < hi; ++r) {
+      const int64_t len = std::min<int64_t>(A.len(r), K);
+      for (int64_t j = 0; j < len; ++j) {
+        const size_t slot = size_t(j) * out.pitch + r;
+        out.col[slot] = A.col[A.row_ptr[r] + j];
+        std::memcpy(out.vals.data() + slot * A.vsize, A.vals + size_t(A.row_ptr[r] + j) * A.vsize, A.vsize);
+      }
+    }
+  }, 4096);
+}
+
+// ---------------------------------------------------------------------------
+// BRO-COO
+// ---------------------------------------------------------------------------
+
+void encode_bro_coo(int64_t nnz, const int32_t* row, const int32_t* col, const uint8_t* vals,
+                    int vsize, int T, int V, CooCode& out) {
+  const int64_t I = int64_t(kH) * T;
+  const int64_t nI = (nnz + I - 1) / I;
+  out.nnz = nnz;
+  out.nI = nI;
+  out.base_row.assign(nI, 0);
+  out.width.assign(nI, 0);
+  std::vector<uint64_t> nsym(nI, 0);
+  auto at = [&](int64_t e) { return (uint32_t)row[std::min(e, nnz - 1)]; };
+  parallel_for(nI, [&](int64_t lo, int64_t hi) {
+    for (int64_t i = lo; i < hi; ++i) {
+      const uint32_t base = at(i * I);
+      uint32_t dmax = 0;
+      for (int lane = 0; lane < kH; ++lane) {
+        uint32_t prev = base;
+        for (int t = 0; t < T; ++t) {
+          uint32_t r = at(i * I + int64_t(kH) * t + lane);
+          dmax = std::max(dmax, r - prev);
+          prev = r;
+        }
+      }
+      out.base_row[i] = base;
+      out.width[i] = (uint8_t)gamma_bits(dmax);  // one width per interval
+      nsym[i] = (uint64_t(T) * out.width[i] + kSym - 1) / kSym;
+    }
+  });
+  exclusive_scan(nsym, out.symptr);
+  out.words.assign(kH * out.symptr[nI], 0u);
+  parallel_for(nI, [&](int64_t lo, int64_t hi) {
+    for (int64_t i = lo; i < hi; ++i) {
+      const int b = out.width[i];
+      const int64_t S = (int64_t)nsym[i];
+      uint32_t* wbase = out.words.data() + kH * out.symptr[i];
+      for (int lane = 0; lane < kH; ++lane) {
+        SymbolWriter w{wbase, lane, S, V};
+        uint32_t prev = out.base_row[i];
+        for (int t = 0; t < T; ++t) {
+          uint32_t r = at(i * I + int64_t(kH) * t + lane);
+          w.put(r - prev, b);
+          prev = r;
+        }
+        w.flush();
+      }
+    }
+  });
+  out.col.assign(col, col + nnz);
+  out.vals.resize(size_t(nnz) * vsize);
+  if (nnz) std::memcpy(out.vals.data(), vals, size_t(nnz) * vsize);
+}
+
+void build_plain_coo(int64_t nnz, const int32_t* row, const int32_t* col, const uint8_t* vals,
+                     int vsize, int T, CooCode& out) {
+  const int64_t I = int64_t(kH) * T;
+  out.nnz = nnz;
+  out.nI = (nnz + I - 1) / I;
+  out.row.assign(row, row + nnz);
+  out.col.assign(col, col + nnz);
+  out.vals.resize(size_t(nnz) * vsize);
+  if (nnz) std::memcpy(out.vals.data(), vals, size_t(nnz) * vsize);
+  out.base_row.assign(out.nI, 0);
+  for (int64_t i = 0; i < out.nI; ++i) out.base_row[i] = (uint32_t)row[i * I];
+}
+
+// ---------------------------------------------------------------------------
+// BAR: BRO-aware reordering
+// ---------------------------------------------------------------------------
+
+// Method 0 ("signature clustering"): stable order by
+// (row length, jump mask, first column, row id), where bit j >= 1 of the
+// jump mask is set when Gamma(delta_j) > 2.  Rows with equal length and
+// jump positions have equal bit allocation patterns up to the jump widths,
+// which is what Eqn (2)'s d(S, j) rewards; ordering by first column inside a
+// group keeps x cachelines shared (Eqn (3)'s c(S, j)).
+void bar_signature_order(int64_t m, const int64_t* row_ptr, const int32_t* col, int64_t* perm) {
+  std::vector<uint64_t> moff(m + 1, 0);
+  for (int64_t i = 0; i < m; ++i) moff[i + 1] = moff[i] + uint64_t((row_ptr[i + 1] - row_ptr[i] + 63) / 64);
+  std::vector<uint64_t> mask(moff[m], 0);
+  parallel_for(m, [&](int64_t lo, int64_t hi) {
+    for (int64_t i = lo; i < hi; ++i) {
+      uint64_t* mk = mask.data() + moff[i];
+      for (int64_t p = row_ptr[i] + 1; p < row_ptr[i + 1]; ++p) {
+        int64_t j = p - row_ptr[i];
+        uint32_t d = uint32_t(col[p]) - uint32_t(col[p - 1]);
+        if (gamma_bits(d) > 2) mk[j / 64] |= uint64_t(1) << (63 - (j % 64));
+      }
+    }
+  }, 4096);
+  std::vector<int64_t> idx(m);
+  std::iota(idx.begin(), idx.end(), 0);
+  auto less = [&](int64_t a, int64_t b) {
+    const int64_t la = row_ptr[a + 1] - row_ptr[a], lb = row_ptr[b + 1] - row_ptr[b];
+    if (la != lb) return la < lb;
+    for (uint64_t w = 0; w < moff[a + 1] - moff[a]; ++w) {
+      uint64_t x = mask[moff[a] + w], y = mask[moff[b] + w];
+      if (x != y) return x < y;
+    }
+    const int64_t fa = la ? col[row_ptr[a]] : -1, fb = lb ? col[row_ptr[b]] : -1;
+    if (fa != fb) return fa < fb;
+    return a < b;
+  };
+  std::sort(idx.begin(), idx.end(), less);
+  std::copy(idx.begin(), idx.end(), perm);
+}
+
+// Method 1: Algorithm 2 — greedy clustering on Eqn (1):
+//   Phi = sum_i h/w * ( ceil(sum_j d(S_i, j) / alpha) + sum_j c(S_i, j) )
+// with h = w = 32 (factor 1, R21), alpha = sym_len = 32, d(S,j) = max Gamma
+// of the j-th deltas (Eqn 2), c(S,j) = number of distinct 128-byte lines of x
+// touched by the j-th columns (Eqn 3, reading R20).  Adding row r to S_p
+// changes only S_p's term, so argmin_p Phi_p = argmin_p DeltaPhi_p; ties go
+// to the lowest p and full partitions are skipped (R22).
+bool bar_greedy_order(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col, int vsize,
+                      int64_t* perm, std::string* err) {
+  (void)n;
+  const int64_t h = kH;
+  if (m > 65536) {
+    if (err) *err = "Algorithm 2 is O(m^2 k / h); limited to m <= 65536";
+    return false;
+  }
+  if (m == 0) return true;
+  const int64_t v = (m + h - 1) / h;
+  auto cap = [&](int64_t p) { return p < v - 1 ? h : m - (v - 1) * h; };
+  int64_t kmax = 0;
+  for (int64_t i = 0; i < m; ++i) kmax = std::max(kmax, row_ptr[i + 1] - row_ptr[i]);
+  // per-row deltas' Gamma and x lines
+  auto gam = [&](int64_t i, int64_t j) -> int {
+    const int64_t p = row_ptr[i] + j;
+    uint32_t c1 = uint32_t(col[p]) + 1u;
+    uint32_t prev = j ? uint32_t(col[p - 1]) + 1u : 0u;
+    return gamma_bits(c1 - prev);
+  };
+  auto line = [&](int64_t i, int64_t j) -> int64_t { return int64_t(col[row_ptr[i] + j]) * vsize / 128; };
+  std::vector<std::vector<uint8_t>> d(v, std::vector<uint8_t>(kmax, 0));
+  std::vector<int64_t> dsum(v, 0);
+  std::vector<std::vector<std::unordered_set<int64_t>>> lines(v, std::vector<std::unordered_set<int64_t>>(kmax));
+  std::vector<std::vector<int64_t>> S(v);
+  auto insert = [&](int64_t p, int64_t i) {
+    const int64_t len = row_ptr[i + 1] - row_ptr[i];
+    for (int64_t j = 0; j < len; ++j) {
+      int g = gam(i, j);
+      if (g > d[p][j]) { dsum[p] += g - d[p][j]; d[p][j] = (uint8_t)g; }
+      lines[p][j].insert(line(i, j));
+    }
+    S[p].push_back(i);
+  };
+  // line 2: sort rows by row length (ascending, stable)
+  std::vector<int64_t> D(m);
+  std::iota(D.begin(), D.end(), 0);
+  std::stable_sort(D.begin(), D.end(), [&](int64_t a, int64_t b) {
+    return row_ptr[a + 1] - row_ptr[a] < row_ptr[b + 1] - row_ptr[b];
+  });
+  // lines 3-6: seed S_t with r_{(t-1)h+1}
+  std::vector<char> used(m, 0);
+  for (int64_t t = 0; t < v; ++t) {
+    insert(t, D[t * h]);
+    used[t * h] = 1;
+  }
+  // lines 7-13
+  const int64_t alpha = kSym;
+  for (int64_t pos = 0; pos < m; ++pos) {
+    if (used[pos]) continue;
+    const int64_t i = D[pos];
+    const int64_t len = row_ptr[i + 1] - row_ptr[i];
+    int64_t best = -1, bestc = 0;
+    for (int64_t p = 0; p < v; ++p) {
+      if ((int64_t)S[p].size() >= cap(p)) continue;
+      int64_t nd = dsum[p];
+      int64_t dc = 0;
+      for (int64_t j = 0; j < len; ++j) {
+        int g = gam(i, j);
+        if (g > d[p][j]) nd += g - d[p][j];
+        if (!lines[p][j].count(line(i, j))) dc++;
+      }
+      const int64_t delta = (nd + alpha - 1) / alpha - (dsum[p] + alpha - 1) / alpha + dc;
+      if (best < 0 || delta < bestc) { best = p; bestc = delta; }
+    }
+    insert(best, i);
+  }
+  int64_t k = 0;
+  for (int64_t p = 0; p < v; ++p)
+    for (int64_t i : S[p]) perm[k++] = i;
+  return true;
+}
+
+}  // namespace bro

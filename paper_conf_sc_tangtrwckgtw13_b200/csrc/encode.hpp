@@ -1,0 +1,96 @@
+// Host-side BRO encoder and layout builder (offline compression).
+// Shares no code with oracle/; both follow DESIGN.md "Encoded layout".
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+namespace bro {
+
+constexpr int kH = 32;        // slice height = warp size (reading R10)
+constexpr int kSym = 32;      // sym_len in bits
+
+// Bytes of one value type.
+struct Bytes {
+  std::vector<uint8_t> v;
+  void resize(size_t n) { v.assign(n, 0); }
+  uint8_t* data() { return v.data(); }
+  const uint8_t* data() const { return v.data(); }
+  size_t size() const { return v.size(); }
+};
+
+// View of the rows that go into an ELL-type part: row i holds the first
+// min(len_i, cap) entries of CSR row i.
+struct RowsView {
+  int64_t m = 0;
+  const int64_t* row_ptr = nullptr;
+  const int32_t* col = nullptr;
+  const uint8_t* vals = nullptr;  // raw value bytes
+  int vsize = 8;                  // bytes per value
+  int64_t cap = INT64_MAX;        // ELL width bound K
+  int64_t len(int64_t i) const {
+    int64_t l = row_ptr[i + 1] - row_ptr[i];
+    return l < cap ? l : cap;
+  }
+};
+
+struct EllCode {                  // BRO-ELL
+  int64_t s = 0;                  // slices
+  std::vector<uint64_t> colptr;   // s+1
+  std::vector<uint64_t> symptr;   // s+1
+  std::vector<uint8_t> bit_alloc; // colptr[s]
+  std::vector<uint32_t> words;    // 32*symptr[s]
+  Bytes vals;                     // 32*colptr[s] values
+  int64_t max_l = 0;              // max num_col over slices
+};
+
+struct CooCode {                  // BRO-COO or plain COO
+  int64_t nnz = 0, nI = 0;
+  std::vector<uint32_t> base_row; // nI
+  std::vector<uint8_t> width;     // nI
+  std::vector<uint64_t> symptr;   // nI+1
+  std::vector<uint32_t> words;    // 32*symptr[nI]
+  std::vector<int32_t> row;       // plain COO only
+  std::vector<int32_t> col;       // nnz
+  Bytes vals;                     // nnz
+};
+
+struct PlainEll {                 // ELLPACK, column-major
+  int64_t K = 0, pitch = 0;
+  std::vector<int32_t> col;       // K*pitch, -1 = padding
+  Bytes vals;                     // K*pitch
+};
+
+// Position of item q of lane r in a block of 32 lanes x S items grouped in
+// chunks of V (tail chunk S - V*floor(S/V)).
+inline int64_t place(int64_t r, int64_t q, int64_t S, int64_t V) {
+  const int64_t F = S / V;
+  const int64_t c = q / V;
+  if (c < F) return kH * V * c + r * V + (q - c * V);
+  return kH * V * F + r * (S - V * F) + (q - V * F);
+}
+
+inline int gamma_bits(uint32_t u) { return u ? 32 - __builtin_clz(u) : 0; }
+
+// Validation of canonical CSR; returns "" if fine, else a message.
+std::string check_csr(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col);
+std::string check_coo(int64_t m, int64_t n, int64_t nnz, const int32_t* row, const int32_t* col);
+
+int64_t hyb_K(int64_t m, const int64_t* row_ptr);
+
+void encode_bro_ell(const RowsView& A, int V, int value_chunk, EllCode& out);
+void build_plain_ell(const RowsView& A, int64_t K, PlainEll& out);
+// rows: int32 rows of the COO entries (sorted); T steps per interval.
+void encode_bro_coo(int64_t nnz, const int32_t* row, const int32_t* col, const uint8_t* vals,
+                    int vsize, int T, int V, CooCode& out);
+void build_plain_coo(int64_t nnz, const int32_t* row, const int32_t* col, const uint8_t* vals,
+                     int vsize, int T, CooCode& out);
+
+// BAR reordering
+void bar_signature_order(int64_t m, const int64_t* row_ptr, const int32_t* col, int64_t* perm);
+bool bar_greedy_order(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col, int vsize,
+                      int64_t* perm, std::string* err);
+
+int num_threads();
+
+}  // namespace bro

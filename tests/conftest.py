@@ -34,3 +34,16 @@ def matrix_A(golden_A):
     row_ptr = np.zeros(m + 1, dtype=np.int64)
     np.cumsum(counts, out=row_ptr[1:])
     return Csr(m, n, row_ptr, cols.astype(np.int32), vals, "paper_A")
+
+
+@pytest.fixture(scope="session")
+def lib():
+    """Build (if stale) and load libbro.so through the Python binding."""
+    import importlib.util
+    spec = importlib.util.spec_from_file_location(
+        "_bro_build", os.path.join(ROOT, "paper_conf_sc_tangtrwckgtw13_b200", "_build.py"))
+    mod = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(mod)
+    mod.build()
+    import paper_conf_sc_tangtrwckgtw13_b200 as P
+    return P
