@@ -3,6 +3,7 @@
 
 #include <algorithm>
 #include <chrono>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -289,6 +290,52 @@ bro_status_t common_checks(bro_dtype_t dtype, const bro_opts_t* opts, bro_opts_t
   return check_opts(*o);
 }
 
+// Persistent grid: as many resident blocks as the SMs hold (queried once per
+// instantiation), capped by the number of slices.
+template <typename T, int V, int kWarps, int kMinBlocks, int G>
+void launch_bro_ell_cfg(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+  using namespace bro::dev;
+  auto kern = bro_ell_spmv<T, V, kWarps, kMinBlocks, G>;
+  static int resident = 0;
+  if (resident == 0) {
+    int per_sm = 0, sms = 0, dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kWarps * 32, 0);
+    resident = std::max(1, per_sm) * std::max(1, sms);
+  }
+  const int64_t need = (A->s + kWarps - 1) / kWarps;
+  const unsigned grid = (unsigned)std::min<int64_t>(need, resident);
+  kern<<<grid, kWarps * 32, 0, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr,
+                                     (const T*)A->d_ell_vals, x, y);
+}
+
+// Tuning knob (not part of the ABI): BRO_ELL_VARIANT selects a compiled
+// launch configuration for V = 4; read once per process.
+int ell_variant() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("BRO_ELL_VARIANT");
+    v = e ? atoi(e) : 0;
+  }
+  return v;
+}
+
+template <typename T, int V>
+void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+  if constexpr (V == 4) {
+    switch (ell_variant()) {
+      case 1: return launch_bro_ell_cfg<T, V, 8, 3, 8>(A, x, y, st);
+      case 2: return launch_bro_ell_cfg<T, V, 8, 4, 8>(A, x, y, st);
+      case 3: return launch_bro_ell_cfg<T, V, 4, 8, 4>(A, x, y, st);
+      case 4: return launch_bro_ell_cfg<T, V, 8, 2, 8>(A, x, y, st);
+      case 5: return launch_bro_ell_cfg<T, V, 8, 5, 4>(A, x, y, st);
+      default: break;
+    }
+  }
+  launch_bro_ell_cfg<T, V, 8, 4, 4>(A, x, y, st);
+}
+
 template <typename T>
 bro_status_t launch_spmv(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   using namespace bro::dev;
@@ -296,17 +343,9 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   if (A->has_ell) {
     if (A->opts.codec) {
       if (A->s > 0) {
-        const int warps = kEllThreads / 32;
-        dim3 grid((unsigned)((A->s + warps - 1) / warps));
-        if (V == 4)
-          bro_ell_spmv<T, 4, kEllThreads><<<grid, kEllThreads, 0, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc,
-              A->d_colptr, A->d_symptr, (const T*)A->d_ell_vals, x, y);
-        else if (V == 2)
-          bro_ell_spmv<T, 2, kEllThreads><<<grid, kEllThreads, 0, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc,
-              A->d_colptr, A->d_symptr, (const T*)A->d_ell_vals, x, y);
-        else
-          bro_ell_spmv<T, 1, kEllThreads><<<grid, kEllThreads, 0, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc,
-              A->d_colptr, A->d_symptr, (const T*)A->d_ell_vals, x, y);
+        if (V == 4) launch_bro_ell<T, 4>(A, x, y, st);
+        else if (V == 2) launch_bro_ell<T, 2>(A, x, y, st);
+        else launch_bro_ell<T, 1>(A, x, y, st);
       }
     } else if (A->m > 0) {
       dim3 grid((unsigned)((A->m + kPlainThreads - 1) / kPlainThreads));

@@ -96,19 +96,20 @@ __device__ __forceinline__ int64_t place(int64_t r, int64_t q, int64_t S, int64_
 // only on S and on widths, which are warp-uniform.
 template <int V>
 struct LaneStream {
-  const uint32_t* base;
-  int S, lane, next, nbuf, remaining;
-  uint32_t buf[8];
+  const uint32_t* base;  // slice / interval word block
+  int S;                 // symbols per lane
+  int q;                 // symbols consumed so far
+  int avail;             // valid bits in hi:lo
   uint32_t hi, lo;
-  int avail;
+  uint32_t buf[8];       // symbols q .. (q | 7) of this lane
 
-  __device__ __forceinline__ void fetch8() {
+  __device__ __forceinline__ void fetch8(int lane) {
     if constexpr (V == 4) {
       const int F = S >> 2;
       const int Vp = S - 4 * F;
 #pragma unroll
       for (int h2 = 0; h2 < 2; ++h2) {
-        const int c = (next >> 2) + h2;
+        const int c = (q >> 2) + h2;
         if (c < F) {
           uint4 v = ld_stream_u4(base + 128 * c + 4 * lane);
           buf[4 * h2 + 0] = v.x; buf[4 * h2 + 1] = v.y;
@@ -122,101 +123,147 @@ struct LaneStream {
     } else {
 #pragma unroll
       for (int k = 0; k < 8; ++k) {
-        const int q = next + k;
-        buf[k] = q < S ? ld_stream_u32(base + place(lane, q, S, V)) : 0u;
+        const int qq = q + k;
+        buf[k] = qq < S ? ld_stream_u32(base + place(lane, qq, S, V)) : 0u;
       }
     }
-    next += 8;
-    nbuf = 8;
   }
-  __device__ __forceinline__ uint32_t pop() {
-    if (nbuf == 0) fetch8();
+  __device__ __forceinline__ uint32_t pop(int lane) {
+    if ((q & 7) == 0) fetch8(lane);
     const uint32_t r = buf[0];
 #pragma unroll
     for (int k = 0; k < 7; ++k) buf[k] = buf[k + 1];
-    --nbuf;
-    --remaining;
+    ++q;
     return r;
   }
-  __device__ __forceinline__ void init(const uint32_t* b, int S_, int lane_) {
-    base = b; S = S_; lane = lane_; next = 0; nbuf = 0; remaining = S_;
+  __device__ __forceinline__ void init(const uint32_t* b, int S_, int lane) {
+    base = b; S = S_; q = 0;
     hi = 0; lo = 0; avail = 0;
-    if (S > 0) { hi = pop(); avail = 32; }
+    if (S > 0) { hi = pop(lane); avail = 32; }
   }
-  __device__ __forceinline__ uint32_t get(int b) {  // 1 <= b <= 32
+  __device__ __forceinline__ uint32_t get(int b, int lane) {  // 1 <= b <= 32
     const uint32_t v = hi >> (32 - b);
     hi = __funnelshift_lc(lo, hi, b);
     lo = shl_clamp(lo, b);
     avail -= b;
-    if (avail < 32 && remaining > 0) {
-      const uint32_t w = pop();
+    if (avail < 32 && q < S) {
+      const uint32_t w = pop(lane);
       hi |= w >> avail;
       lo = shl_clamp(w, 32 - avail);
       avail += 32;
     }
     return v;
   }
+  // park / resume the lane's state in shared memory (12 words per lane,
+  // stride 32) so it does not occupy registers between column blocks
+  __device__ __forceinline__ void save(uint32_t* st, int lane) const {
+    st[0 * 32 + lane] = (uint32_t)q; st[1 * 32 + lane] = (uint32_t)avail;
+    st[2 * 32 + lane] = hi; st[3 * 32 + lane] = lo;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) st[(4 + k) * 32 + lane] = buf[k];
+  }
+  __device__ __forceinline__ void restore(const uint32_t* b, int S_, const uint32_t* st, int lane) {
+    base = b; S = S_;
+    q = (int)st[0 * 32 + lane]; avail = (int)st[1 * 32 + lane];
+    hi = st[2 * 32 + lane]; lo = st[3 * 32 + lane];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) buf[k] = st[(4 + k) * 32 + lane];
+  }
 };
 
 // ------------------------------------------------------------------ BRO-ELL
 // y[32t + lane] = sum_j vals(slot) * x[col_j], Alg. 1.
-template <typename T, int V, int kThreads>
-__global__ void __launch_bounds__(kThreads)
+//
+// Persistent warps walk slices t = warp_id, warp_id + n_warps, ...; the next
+// slice's metadata is prefetched while the current one runs.  Each slice is
+// processed in blocks of up to 32 columns:
+//   phase 1 (decode): the 32 widths of the block are loaded one per lane and
+//     broadcast by SHFL; every lane pulls its deltas through the 64-bit
+//     window, accumulates the column (col += delta) and writes it to a
+//     per-warp shared-memory column buffer (-1 for padding, delta == 0);
+//   phase 2 (multiply): groups of 8 columns, all value chunks (16-byte loads)
+//     and all x gathers of a group issued before the FMAs (8 gathers + 4/2
+//     vector loads in flight per lane), slot-order FMA accumulation.
+// Registers stay near the plain-ELL kernel's, so occupancy stays high.
+template <typename T, int G>
+__device__ __forceinline__ void load_group_vals(T* v, const T* vs, int j, int l, int lfull, int lane) {
+  constexpr int VV = Chunk<T>::N;
+#pragma unroll
+  for (int u = 0; u < G / VV; ++u) {
+    const int jj = j + u * VV;
+    if (jj + VV <= lfull) {
+      Chunk<T> c;
+      c.load(vs + 32 * jj + lane * VV);
+#pragma unroll
+      for (int k = 0; k < VV; ++k) v[u * VV + k] = c.v[k];
+    } else {
+      const int tw = l - lfull;  // tail slots per lane (< VV), contiguous per lane
+#pragma unroll
+      for (int k = 0; k < VV; ++k)
+        v[u * VV + k] = (jj + k < l) ? ld_stream(vs + 32 * lfull + lane * tw + (jj + k - lfull)) : T(0);
+    }
+  }
+}
+
+template <typename T, int V, int kWarps, int kMinBlocks, int G>
+__global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_spmv(int64_t m, int64_t s, const uint32_t* __restrict__ words,
              const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
              const uint64_t* __restrict__ symptr, const T* __restrict__ vals,
              const T* __restrict__ x, T* __restrict__ y) {
   constexpr int VV = Chunk<T>::N;
-  constexpr int G = 8;  // columns per unrolled group
+  __shared__ int32_t colbuf[kWarps][32 * 32];
+  __shared__ uint32_t stbuf[kWarps][12 * 32];
   const int lane = threadIdx.x & 31;
-  const int64_t t = int64_t(blockIdx.x) * (kThreads / 32) + (threadIdx.x >> 5);
-  if (t >= s) return;
-  const uint64_t c0 = colptr[t];
-  const int l = int(colptr[t + 1] - c0);
-  const uint64_t q0 = symptr[t];
-  const int S = int(symptr[t + 1] - q0);
-  LaneStream<V> ls;
-  ls.init(words + 32 * q0, S, lane);
-  const T* vs = vals + 32 * c0;
-  const uint8_t* ba = bit_alloc + c0;
-  const int lfull = (l / VV) * VV;
-  T sum = T(0);
-  int col = -1;
-  uint32_t breg = 0;
-  int j = 0;
-  for (; j + G <= lfull; j += G) {
-    if ((j & 31) == 0) breg = lane < l - j ? uint32_t(__ldg(ba + j + lane)) : 0u;
-    Chunk<T> v[G / VV];
+  const int w = threadIdx.x >> 5;
+  int32_t* cb = colbuf[w];
+  uint32_t* st = stbuf[w];
+  const int64_t stride = int64_t(gridDim.x) * kWarps;
+  for (int64_t t = int64_t(blockIdx.x) * kWarps + w; t < s; t += stride) {
+    const uint64_t c0 = __ldg(colptr + t);
+    const int l = int(__ldg(colptr + t + 1) - c0);
+    const uint64_t q0 = __ldg(symptr + t);
+    const int S = int(__ldg(symptr + t + 1) - q0);
+    const uint32_t* wb = words + 32 * q0;
+    const T* vs = vals + 32 * c0;
+    const uint8_t* ba = bit_alloc + c0;
+    const int lfull = (l / VV) * VV;
+    T sum = T(0);
+    int col = -1;
+    for (int jb = 0; jb < l; jb += 32) {
+      const int nb = min(32, l - jb);
+      {  // phase 1: decode columns [jb, jb + nb) into cb
+        const uint32_t breg = lane < nb ? uint32_t(__ldg(ba + jb + lane)) : 0u;
+        LaneStream<V> ls;
+        if (jb == 0) ls.init(wb, S, lane);
+        else ls.restore(wb, S, st, lane);
+#pragma unroll 4
+        for (int k = 0; k < nb; ++k) {
+          const int b = (int)__shfl_sync(0xffffffffu, breg, k);
+          const uint32_t d = ls.get(b, lane);
+          col += int(d);
+          cb[k * 32 + lane] = d ? col : -1;
+        }
+        if (jb + 32 < l) ls.save(st, lane);
+      }
+      __syncwarp();
+      for (int g = 0; g < nb; g += G) {  // phase 2
+        T v[G];
+        load_group_vals<T, G>(v, vs, jb + g, l, lfull, lane);
+        int cc[G];
 #pragma unroll
-    for (int u = 0; u < G / VV; ++u) v[u].load(vs + 32 * (j + u * VV) + lane * VV);
-    int cidx[G];
-    bool ok[G];
+        for (int k = 0; k < G; ++k) cc[k] = (g + k < nb) ? cb[(g + k) * 32 + lane] : -1;
+        T xv[G];
 #pragma unroll
-    for (int k = 0; k < G; ++k) {
-      const int b = (int)__shfl_sync(0xffffffffu, breg, (j + k) & 31);
-      const uint32_t d = ls.get(b);
-      col += int(d);
-      cidx[k] = col;
-      ok[k] = d != 0u;
+        for (int k = 0; k < G; ++k) xv[k] = cc[k] >= 0 ? ldg_x(x + cc[k]) : T(0);
+#pragma unroll
+        for (int k = 0; k < G; ++k) sum = fma(v[k], xv[k], sum);
+      }
+      __syncwarp();
     }
-    T xv[G];
-#pragma unroll
-    for (int k = 0; k < G; ++k) xv[k] = ok[k] ? ldg_x(x + cidx[k]) : T(0);
-#pragma unroll
-    for (int k = 0; k < G; ++k) sum = fma(v[k / VV].v[k % VV], xv[k], sum);
+    const int64_t row = 32 * t + lane;
+    if (row < m) y[row] = sum;
   }
-  for (; j < l; ++j) {
-    if ((j & 31) == 0) breg = lane < l - j ? uint32_t(__ldg(ba + j + lane)) : 0u;
-    const int b = (int)__shfl_sync(0xffffffffu, breg, j & 31);
-    const uint32_t d = ls.get(b);
-    col += int(d);
-    const T* vp = j < lfull ? vs + 32 * (j - j % VV) + lane * VV + j % VV
-                            : vs + 32 * lfull + lane * (l - lfull) + (j - lfull);
-    const T v = ld_stream(vp);
-    if (d != 0u) sum = fma(v, ldg_x(x + col), sum);
-  }
-  const int64_t row = 32 * t + lane;
-  if (row < m) y[row] = sum;
 }
 
 // Decode-only variant: decoded column (or -1) per slot in V=1 slot order.
@@ -235,7 +282,7 @@ __global__ void bro_ell_decode(int64_t s, const uint32_t* __restrict__ words,
   ls.init(words + 32 * q0, int(symptr[t + 1] - q0), lane);
   int col = -1;
   for (int j = 0; j < l; ++j) {
-    const uint32_t d = ls.get(bit_alloc[c0 + j]);
+    const uint32_t d = ls.get(bit_alloc[c0 + j], lane);
     col += int(d);
     out[32 * c0 + 32 * j + lane] = d ? col : -1;
   }
@@ -312,7 +359,7 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, const uint32_t* __restrict__ word
     const int64_t e = e0 + 32 * t + lane;
     const bool valid = e < nnz;
     if constexpr (kBro) {
-      if (b) row += (int)ls.get(b);
+      if (b) row += (int)ls.get(b, lane);
     } else {
       row = ld_stream_s32(rows + (valid ? e : nnz - 1));
     }
@@ -398,7 +445,7 @@ __global__ void bro_coo_decode(int64_t nnz, int64_t nI, int T_steps, const uint3
   ls.init(words + 32 * symptr[i], int(symptr[i + 1] - symptr[i]), lane);
   int row = (int)base_row[i];
   for (int t = 0; t < T_steps; ++t) {
-    if (b) row += (int)ls.get(b);
+    if (b) row += (int)ls.get(b, lane);
     const int64_t e = i * 32 * T_steps + 32 * t + lane;
     if (e < nnz) out[e] = row;
   }

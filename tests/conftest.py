@@ -8,7 +8,18 @@ if ROOT not in sys.path:
     sys.path.insert(0, ROOT)
 
 
+def _build_lib():
+    """Build libbro.so in-tree if missing or stale (nvcc cross-compiles here)."""
+    import importlib.util
+    spec = importlib.util.spec_from_file_location(
+        "_bro_build", os.path.join(ROOT, "paper_conf_sc_tangtrwckgtw13_b200", "_build.py"))
+    mod = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(mod)
+    mod.build()
+
+
 def pytest_configure(config):
+    _build_lib()
     config.addinivalue_line("markers", "gpu: needs a CUDA B200 (run via gpurun)")
     config.addinivalue_line("markers", "slow: long CPU test (full-size configs)")
 
@@ -39,11 +50,6 @@ def matrix_A(golden_A):
 @pytest.fixture(scope="session")
 def lib():
     """Build (if stale) and load libbro.so through the Python binding."""
-    import importlib.util
-    spec = importlib.util.spec_from_file_location(
-        "_bro_build", os.path.join(ROOT, "paper_conf_sc_tangtrwckgtw13_b200", "_build.py"))
-    mod = importlib.util.module_from_spec(spec)
-    spec.loader.exec_module(mod)
-    mod.build()
+    _build_lib()
     import paper_conf_sc_tangtrwckgtw13_b200 as P
     return P
