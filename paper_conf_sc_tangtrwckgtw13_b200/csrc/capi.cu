@@ -74,6 +74,7 @@ struct bro_matrix_s {
   void* d_xs = nullptr;
   void* d_ys = nullptr;
   int64_t device_bytes = 0;
+  int64_t stage_bytes = 0;  // TMA ring stage size (largest slice: values + symbols + widths window)
   bro_info_t info{};
 };
 
@@ -238,6 +239,15 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
 #define UP(dst, vec) \
   if (st == BRO_OK) st = dev_upload(A, &(dst), (vec).data(), (vec).size() * sizeof(*(vec).data()))
     if (A->has_ell && o.codec) {
+      int64_t need = 0;
+      for (int64_t t = 0; t < A->s; ++t) {
+        const uint64_t c0 = A->ell.colptr[t], c1 = A->ell.colptr[t + 1];
+        const int64_t b = int64_t(32 * (c1 - c0) * A->vsize + 128 * (A->ell.symptr[t + 1] - A->ell.symptr[t]) +
+                                  (((c1 + 15) & ~uint64_t(15)) - (c0 & ~uint64_t(15))));
+        need = std::max(need, b);
+      }
+      A->stage_bytes = (need + 127) / 128 * 128;
+      A->ell.bit_alloc.resize(A->ell.bit_alloc.size() + 16, 0);  // bulk copies read 16-byte windows
       UP(A->d_words, A->ell.words);
       UP(A->d_bit_alloc, A->ell.bit_alloc);
       UP(A->d_colptr, A->ell.colptr);
@@ -310,6 +320,33 @@ void launch_bro_ell_cfg(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
                                      (const T*)A->d_ell_vals, x, y);
 }
 
+// TMA-pipelined BRO-ELL: ring of `nstages` stages of A->stage_bytes in
+// dynamic shared memory, kMinBlocks blocks per SM.  Returns false when the
+// largest slice does not leave room for at least 2 stages.
+template <typename T, int V, int kCons, int kMinBlocks>
+bool launch_bro_ell_tma(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+  using namespace bro::dev;
+  auto kern = bro_ell_spmv_tma<T, V, kCons, kMinBlocks>;
+  constexpr int kSmemPerBlock = (227 * 1024) / kMinBlocks - 1024;
+  static int sms = 0;
+  if (sms == 0) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemPerBlock);
+  }
+  const int64_t hdr = 128;  // rounded per-stage barrier + header bytes, see kernel
+  int nst = (int)std::min<int64_t>(32, (kSmemPerBlock - 32 * 40) / std::max<int64_t>(A->stage_bytes, 1));
+  if (nst < 2) return false;
+  const size_t smem = size_t(((nst * (16 + 16)) + 127) / 128 * 128) + size_t(nst) * A->stage_bytes;
+  (void)hdr;
+  const int64_t grid = std::min<int64_t>(A->s, int64_t(sms) * kMinBlocks);
+  kern<<<(unsigned)grid, (kCons + 1) * 32, smem, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc, A->d_colptr,
+                                                       A->d_symptr, (const T*)A->d_ell_vals, x, y, nst,
+                                                       (int)A->stage_bytes);
+  return true;
+}
+
 // Tuning knob (not part of the ABI): BRO_ELL_VARIANT selects a compiled
 // launch configuration for V = 4; read once per process.
 int ell_variant() {
@@ -325,13 +362,15 @@ template <typename T, int V>
 void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   if constexpr (V == 4) {
     switch (ell_variant()) {
-      case 1: return launch_bro_ell_cfg<T, V, 8, 3, 8>(A, x, y, st);
-      case 2: return launch_bro_ell_cfg<T, V, 8, 4, 8>(A, x, y, st);
-      case 3: return launch_bro_ell_cfg<T, V, 4, 8, 4>(A, x, y, st);
-      case 4: return launch_bro_ell_cfg<T, V, 8, 2, 8>(A, x, y, st);
-      case 5: return launch_bro_ell_cfg<T, V, 8, 5, 4>(A, x, y, st);
+      case 0: if (launch_bro_ell_tma<T, V, 8, 2>(A, x, y, st)) return; break;
+      case 1: if (launch_bro_ell_tma<T, V, 4, 4>(A, x, y, st)) return; break;
+      case 2: if (launch_bro_ell_tma<T, V, 12, 1>(A, x, y, st)) return; break;
+      case 3: if (launch_bro_ell_tma<T, V, 6, 3>(A, x, y, st)) return; break;
+      case 8: return launch_bro_ell_cfg<T, V, 8, 4, 8>(A, x, y, st);
       default: break;
     }
+  } else {
+    if (launch_bro_ell_tma<T, V, 8, 2>(A, x, y, st)) return;
   }
   launch_bro_ell_cfg<T, V, 8, 4, 4>(A, x, y, st);
 }

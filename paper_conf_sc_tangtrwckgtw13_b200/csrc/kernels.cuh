@@ -266,6 +266,224 @@ bro_ell_spmv(int64_t m, int64_t s, const uint32_t* __restrict__ words,
   }
 }
 
+// ------------------------------------------------------------------ BRO-ELL, TMA pipeline
+// Warp-specialised persistent kernel.  Block b owns slices t_k = b + k*gridDim.x.
+// Producer warp: loads the metadata of 32 upcoming slices at once (one slice
+// per lane), then for each slice waits for a free ring stage and issues three
+// bulk async copies (cp.async.bulk, TMA engine) — the slice's values
+// (32*l*sizeof(T) bytes), its multiplexed symbols (128*S bytes) and its
+// widths (16-byte aligned window of bit_alloc) — all completing on the
+// stage's mbarrier.  Consumer warps (one slice each, round robin) wait on the
+// stage, decode the symbols from shared memory, gather x through the
+// read-only path, multiply with the staged values and release the stage.
+// HBM latency is hidden by the ring depth instead of by registers.
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n"
+      "WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra WAIT_%=;\n}\n" :: "r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar,
+                                         uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+      :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(policy) : "memory");
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+
+// One lane's symbols read from shared memory (V-interleaved, 16-byte chunks
+// read with one LDS.128 per 4 symbols), MSB first through a 64-bit window.
+template <int V>
+struct SmemLaneStream {
+  const uint32_t* base;
+  int S, q, avail;
+  uint32_t hi, lo;
+  uint32_t buf[4];
+
+  __device__ __forceinline__ void fetch4(int lane) {
+    if constexpr (V == 4) {
+      const int F = S >> 2;
+      const int c = q >> 2;
+      if (c < F) {
+        const uint4 v = *reinterpret_cast<const uint4*>(base + 128 * c + 4 * lane);
+        buf[0] = v.x; buf[1] = v.y; buf[2] = v.z; buf[3] = v.w;
+      } else {
+        const int Vp = S - 4 * F;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) buf[k] = k < Vp ? base[128 * F + Vp * lane + k] : 0u;
+      }
+    } else {
+#pragma unroll
+      for (int k = 0; k < 4; ++k) buf[k] = (q + k < S) ? base[place(lane, q + k, S, V)] : 0u;
+    }
+  }
+  __device__ __forceinline__ uint32_t pop(int lane) {
+    if ((q & 3) == 0) fetch4(lane);
+    const uint32_t r = buf[0];
+    buf[0] = buf[1]; buf[1] = buf[2]; buf[2] = buf[3];
+    ++q;
+    return r;
+  }
+  __device__ __forceinline__ void init(const uint32_t* b, int S_, int lane) {
+    base = b; S = S_; q = 0; hi = 0; lo = 0; avail = 0;
+    if (S > 0) { hi = pop(lane); avail = 32; }
+  }
+  __device__ __forceinline__ uint32_t get(int b, int lane) {  // 1 <= b <= 32
+    const uint32_t v = hi >> (32 - b);
+    hi = __funnelshift_lc(lo, hi, b);
+    lo = shl_clamp(lo, b);
+    avail -= b;
+    if (avail < 32 && q < S) {
+      const uint32_t w = pop(lane);
+      hi |= w >> avail;
+      lo = shl_clamp(w, 32 - avail);
+      avail += 32;
+    }
+    return v;
+  }
+};
+
+struct StageHdr {
+  int l, S, ba_off, pad;
+};
+
+template <typename T, int V, int kCons, int kMinBlocks>
+__global__ void __launch_bounds__((kCons + 1) * 32, kMinBlocks)
+bro_ell_spmv_tma(int64_t m, int64_t s, const uint32_t* __restrict__ words,
+                 const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
+                 const uint64_t* __restrict__ symptr, const T* __restrict__ vals,
+                 const T* __restrict__ x, T* __restrict__ y, int nstages, int stage_bytes) {
+  constexpr int VV = Chunk<T>::N;
+  constexpr int G = 8;
+  extern __shared__ __align__(128) uint8_t smem[];
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem);
+  uint64_t* empty = full + nstages;
+  StageHdr* hdr = reinterpret_cast<StageHdr*>(empty + nstages);
+  uint8_t* ring = smem + ((nstages * (16 + sizeof(StageHdr)) + 127) / 128) * 128;
+  const int lane = threadIdx.x & 31;
+  const int w = threadIdx.x >> 5;
+  const int64_t G0 = gridDim.x;
+  const int64_t nk = (s > blockIdx.x) ? (s - blockIdx.x + G0 - 1) / G0 : 0;
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < nstages; ++i) {
+      mbar_init(full + i, 1);
+      mbar_init(empty + i, 1);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if (w == kCons) {
+    // ------------------------------------------------ producer warp
+    const uint64_t pol = policy_evict_first();
+    for (int64_t k0 = 0; k0 < nk; k0 += 32) {
+      const int64_t kk = k0 + lane;
+      uint64_t c0 = 0, c1 = 0, q0 = 0, q1 = 0;
+      if (kk < nk) {
+        const int64_t t = blockIdx.x + kk * G0;
+        c0 = __ldg(colptr + t); c1 = __ldg(colptr + t + 1);
+        q0 = __ldg(symptr + t); q1 = __ldg(symptr + t + 1);
+      }
+      const int nb = (int)(nk - k0 < 32 ? nk - k0 : 32);
+      for (int i = 0; i < nb; ++i) {
+        const uint64_t a0 = __shfl_sync(0xffffffffu, c0, i), a1 = __shfl_sync(0xffffffffu, c1, i);
+        const uint64_t b0 = __shfl_sync(0xffffffffu, q0, i), b1 = __shfl_sync(0xffffffffu, q1, i);
+        const int64_t k = k0 + i;
+        const int st = int(k % nstages);
+        const uint32_t ph = uint32_t((k / nstages) & 1);
+        if (lane == 0) {
+          mbar_wait(empty + st, ph ^ 1u);
+          const int l = int(a1 - a0), S = int(b1 - b0);
+          const uint32_t vbytes = uint32_t(32 * l * sizeof(T));
+          const uint32_t wbytes = uint32_t(128 * S);
+          const uint64_t ba_lo = a0 & ~uint64_t(15);
+          const uint32_t bbytes = uint32_t(((a1 + 15) & ~uint64_t(15)) - ba_lo);
+          hdr[st] = StageHdr{l, S, int(a0 - ba_lo), 0};
+          uint8_t* dst = ring + size_t(st) * stage_bytes;
+          mbar_arrive_expect_tx(full + st, vbytes + wbytes + bbytes);
+          if (vbytes) bulk_g2s(dst, vals + 32 * a0, vbytes, full + st, pol);
+          if (wbytes) bulk_g2s(dst + vbytes, words + 32 * b0, wbytes, full + st, pol);
+          if (bbytes) bulk_g2s(dst + vbytes + wbytes, bit_alloc + ba_lo, bbytes, full + st, pol);
+        }
+        __syncwarp();
+      }
+    }
+    return;
+  }
+  // -------------------------------------------------- consumer warps
+  for (int64_t k = w; k < nk; k += kCons) {
+    const int st = int(k % nstages);
+    const uint32_t ph = uint32_t((k / nstages) & 1);
+    mbar_wait(full + st, ph);
+    const StageHdr h = hdr[st];
+    const int l = h.l, S = h.S;
+    const uint8_t* sbase = ring + size_t(st) * stage_bytes;
+    const T* sv = reinterpret_cast<const T*>(sbase);
+    const uint32_t* sw = reinterpret_cast<const uint32_t*>(sbase + 32 * l * sizeof(T));
+    const uint8_t* sb = sbase + 32 * l * sizeof(T) + 128 * S + h.ba_off;
+    const int lfull = (l / VV) * VV;
+    const int tw = l - lfull;
+    SmemLaneStream<V> ls;
+    ls.init(sw, S, lane);
+    T sum = T(0);
+    int col = -1;
+    for (int j0 = 0; j0 < l; j0 += G) {
+      int cc[G];
+#pragma unroll
+      for (int k2 = 0; k2 < G; ++k2) {
+        const int j = j0 + k2;
+        const int b = j < l ? int(sb[j]) : 0;
+        const uint32_t d = b ? ls.get(b, lane) : 0u;
+        col += int(d);
+        cc[k2] = d ? col : -1;
+      }
+      T xv[G];
+#pragma unroll
+      for (int k2 = 0; k2 < G; ++k2) xv[k2] = cc[k2] >= 0 ? ldg_x(x + cc[k2]) : T(0);
+      T v[G];
+#pragma unroll
+      for (int u = 0; u < G / VV; ++u) {
+        const int jj = j0 + u * VV;
+        if (jj + VV <= lfull) {
+          if constexpr (VV == 2) {
+            const double2 c2 = *reinterpret_cast<const double2*>(sv + 32 * jj + lane * VV);
+            v[u * VV] = c2.x; v[u * VV + 1] = c2.y;
+          } else {
+            const float4 c4 = *reinterpret_cast<const float4*>(sv + 32 * jj + lane * VV);
+            v[u * VV] = c4.x; v[u * VV + 1] = c4.y; v[u * VV + 2] = c4.z; v[u * VV + 3] = c4.w;
+          }
+        } else {
+#pragma unroll
+          for (int q2 = 0; q2 < VV; ++q2)
+            v[u * VV + q2] = (jj + q2 < l) ? sv[32 * lfull + lane * tw + (jj + q2 - lfull)] : T(0);
+        }
+      }
+#pragma unroll
+      for (int k2 = 0; k2 < G; ++k2) sum = fma(v[k2], xv[k2], sum);
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(empty + st);
+    const int64_t row = 32 * (blockIdx.x + k * G0) + lane;
+    if (row < m) y[row] = sum;
+  }
+}
+
 // Decode-only variant: decoded column (or -1) per slot in V=1 slot order.
 template <int V>
 __global__ void bro_ell_decode(int64_t s, const uint32_t* __restrict__ words,
