@@ -320,11 +320,12 @@ void launch_bro_ell_cfg(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
                                      (const T*)A->d_ell_vals, x, y);
 }
 
-// TMA-pipelined BRO-ELL: ring of `nstages` stages of A->stage_bytes in
-// dynamic shared memory, kMinBlocks blocks per SM.  Returns false when the
-// largest slice does not leave room for at least 2 stages.
+// TMA-pipelined BRO-ELL.  The ring holds ncons * spc stages of
+// A->stage_bytes (the largest slice) in dynamic shared memory; ncons
+// consumer warps are active (<= kCons) so that each owns spc >= kMinSpc
+// stages.  Returns false when even one consumer cannot get kMinSpc stages.
 template <typename T, int V, int kCons, int kMinBlocks>
-bool launch_bro_ell_tma(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+bool launch_bro_ell_tma(bro_matrix_s* A, const T* x, T* y, cudaStream_t st, int min_spc = 2) {
   using namespace bro::dev;
   auto kern = bro_ell_spmv_tma<T, V, kCons, kMinBlocks>;
   constexpr int kSmemPerBlock = (227 * 1024) / kMinBlocks - 1024;
@@ -335,15 +336,17 @@ bool launch_bro_ell_tma(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemPerBlock);
   }
-  const int64_t hdr = 128;  // rounded per-stage barrier + header bytes, see kernel
-  int nst = (int)std::min<int64_t>(32, (kSmemPerBlock - 32 * 40) / std::max<int64_t>(A->stage_bytes, 1));
-  if (nst < 2) return false;
-  const size_t smem = size_t(((nst * (16 + 16)) + 127) / 128 * 128) + size_t(nst) * A->stage_bytes;
-  (void)hdr;
+  const int64_t sb = std::max<int64_t>(A->stage_bytes, 128);
+  const int64_t fit = (kSmemPerBlock - 2048) / sb;           // stages that fit
+  const int ncons = (int)std::min<int64_t>(kCons, fit / min_spc);
+  if (ncons < 1) return false;
+  const int spc = (int)std::min<int64_t>(fit / ncons, 8);
+  const int nst = ncons * spc;
+  const size_t smem = size_t(((nst * (16 + 16)) + 127) / 128 * 128) + size_t(nst) * sb;
   const int64_t grid = std::min<int64_t>(A->s, int64_t(sms) * kMinBlocks);
   kern<<<(unsigned)grid, (kCons + 1) * 32, smem, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc, A->d_colptr,
-                                                       A->d_symptr, (const T*)A->d_ell_vals, x, y, nst,
-                                                       (int)A->stage_bytes);
+                                                       A->d_symptr, (const T*)A->d_ell_vals, x, y, ncons, spc,
+                                                       (int)sb);
   return true;
 }
 
@@ -362,15 +365,20 @@ template <typename T, int V>
 void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   if constexpr (V == 4) {
     switch (ell_variant()) {
-      case 0: if (launch_bro_ell_tma<T, V, 8, 2>(A, x, y, st)) return; break;
+      case 0:
+        if (launch_bro_ell_tma<T, V, 8, 2>(A, x, y, st)) return;
+        if (launch_bro_ell_tma<T, V, 8, 1>(A, x, y, st)) return;
+        break;
       case 1: if (launch_bro_ell_tma<T, V, 4, 4>(A, x, y, st)) return; break;
-      case 2: if (launch_bro_ell_tma<T, V, 12, 1>(A, x, y, st)) return; break;
+      case 2: if (launch_bro_ell_tma<T, V, 8, 2>(A, x, y, st, 3)) return; break;
       case 3: if (launch_bro_ell_tma<T, V, 6, 3>(A, x, y, st)) return; break;
+      case 4: if (launch_bro_ell_tma<T, V, 8, 1>(A, x, y, st, 3)) return; break;
       case 8: return launch_bro_ell_cfg<T, V, 8, 4, 8>(A, x, y, st);
       default: break;
     }
   } else {
     if (launch_bro_ell_tma<T, V, 8, 2>(A, x, y, st)) return;
+    if (launch_bro_ell_tma<T, V, 8, 1>(A, x, y, st)) return;
   }
   launch_bro_ell_cfg<T, V, 8, 4, 4>(A, x, y, st);
 }

@@ -364,12 +364,18 @@ struct StageHdr {
   int l, S, ba_off, pad;
 };
 
+// Stage ownership: item k (the block's k-th slice) goes to consumer
+// w = k % ncons, its j = k / ncons -th item, in the consumer's private stage
+// w * spc + j % spc, phase (j / spc) & 1.  A consumer therefore never waits
+// on a stage more than one phase ahead (mbarrier parity cannot alias), and
+// the producer, which runs in item order, never either.
 template <typename T, int V, int kCons, int kMinBlocks>
 __global__ void __launch_bounds__((kCons + 1) * 32, kMinBlocks)
 bro_ell_spmv_tma(int64_t m, int64_t s, const uint32_t* __restrict__ words,
                  const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
                  const uint64_t* __restrict__ symptr, const T* __restrict__ vals,
-                 const T* __restrict__ x, T* __restrict__ y, int nstages, int stage_bytes) {
+                 const T* __restrict__ x, T* __restrict__ y, int ncons, int spc, int stage_bytes) {
+  const int nstages = ncons * spc;
   constexpr int VV = Chunk<T>::N;
   constexpr int G = 8;
   extern __shared__ __align__(128) uint8_t smem[];
@@ -405,8 +411,9 @@ bro_ell_spmv_tma(int64_t m, int64_t s, const uint32_t* __restrict__ words,
         const uint64_t a0 = __shfl_sync(0xffffffffu, c0, i), a1 = __shfl_sync(0xffffffffu, c1, i);
         const uint64_t b0 = __shfl_sync(0xffffffffu, q0, i), b1 = __shfl_sync(0xffffffffu, q1, i);
         const int64_t k = k0 + i;
-        const int st = int(k % nstages);
-        const uint32_t ph = uint32_t((k / nstages) & 1);
+        const int64_t jj = k / ncons;
+        const int st = int(k - jj * ncons) * spc + int(jj % spc);
+        const uint32_t ph = uint32_t((jj / spc) & 1);
         if (lane == 0) {
           mbar_wait(empty + st, ph ^ 1u);
           const int l = int(a1 - a0), S = int(b1 - b0);
@@ -427,9 +434,11 @@ bro_ell_spmv_tma(int64_t m, int64_t s, const uint32_t* __restrict__ words,
     return;
   }
   // -------------------------------------------------- consumer warps
-  for (int64_t k = w; k < nk; k += kCons) {
-    const int st = int(k % nstages);
-    const uint32_t ph = uint32_t((k / nstages) & 1);
+  if (w >= ncons) return;
+  int64_t jj = 0;
+  for (int64_t k = w; k < nk; k += ncons, ++jj) {
+    const int st = w * spc + int(jj % spc);
+    const uint32_t ph = uint32_t((jj / spc) & 1);
     mbar_wait(full + st, ph);
     const StageHdr h = hdr[st];
     const int l = h.l, S = h.S;

@@ -1,7 +1,8 @@
 #!/usr/bin/env python
 """Tuning sweep (GPU box): run bench.py for each BRO_ELL_VARIANT x workload x
 dtype in subprocesses and print one compact line per run.
-usage: python scripts/sweep.py OUTDIR "0 1 2" "C5:f64 C5:f32 C2:f64"
+usage: python scripts/sweep.py OUTDIR "0 1 2" "C5:f64 C5:f32:0,8 C2:f64"
+(a case may carry its own comma-separated variant list)
 """
 import json
 import os
@@ -14,8 +15,9 @@ cases = sys.argv[3].split()
 extra = sys.argv[4:] if len(sys.argv) > 4 else []
 os.makedirs(out, exist_ok=True)
 for case in cases:
-    wl, dt = case.split(":")
-    for v in variants:
+    parts = case.split(":")
+    wl, dt = parts[0], parts[1]
+    for v in (parts[2].split(",") if len(parts) > 2 else variants):
         env = dict(os.environ, BRO_ELL_VARIANT=v)
         cmd = [sys.executable, "bench.py", "--workload", wl, "--dtype", dt, "--steps", "300",
                "--no-cpu-baseline", "--no-e2e"] + extra
