@@ -350,6 +350,24 @@ bool launch_bro_ell_tma(bro_matrix_s* A, const T* x, T* y, cudaStream_t st, int 
   return true;
 }
 
+template <typename T, int V, int kWarps, int kMinBlocks>
+void launch_bro_ell_od(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+  using namespace bro::dev;
+  auto kern = bro_ell_spmv_od<T, V, kWarps, kMinBlocks>;
+  static int resident = 0;
+  if (resident == 0) {
+    int per_sm = 0, sms = 0, dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kWarps * 32, 0);
+    resident = std::max(1, per_sm) * std::max(1, sms);
+  }
+  const int64_t need = (A->s + kWarps - 1) / kWarps;
+  const unsigned grid = (unsigned)std::min<int64_t>(need, resident);
+  kern<<<grid, kWarps * 32, 0, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr,
+                                     (const T*)A->d_ell_vals, x, y);
+}
+
 // Tuning knob (not part of the ABI): BRO_ELL_VARIANT selects a compiled
 // launch configuration for V = 4; read once per process.
 int ell_variant() {
@@ -365,22 +383,21 @@ template <typename T, int V>
 void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   if constexpr (V == 4) {
     switch (ell_variant()) {
-      case 0:
+      case 0: return launch_bro_ell_od<T, V, 8, 4>(A, x, y, st);
+      case 1: return launch_bro_ell_od<T, V, 8, 3>(A, x, y, st);
+      case 2: return launch_bro_ell_od<T, V, 8, 5>(A, x, y, st);
+      case 3: return launch_bro_ell_od<T, V, 4, 8>(A, x, y, st);
+      case 5:
         if (launch_bro_ell_tma<T, V, 8, 2>(A, x, y, st)) return;
         if (launch_bro_ell_tma<T, V, 8, 1>(A, x, y, st)) return;
         break;
-      case 1: if (launch_bro_ell_tma<T, V, 4, 4>(A, x, y, st)) return; break;
-      case 2: if (launch_bro_ell_tma<T, V, 8, 2>(A, x, y, st, 3)) return; break;
-      case 3: if (launch_bro_ell_tma<T, V, 6, 3>(A, x, y, st)) return; break;
-      case 4: if (launch_bro_ell_tma<T, V, 8, 1>(A, x, y, st, 3)) return; break;
       case 8: return launch_bro_ell_cfg<T, V, 8, 4, 8>(A, x, y, st);
       default: break;
     }
-  } else {
-    if (launch_bro_ell_tma<T, V, 8, 2>(A, x, y, st)) return;
-    if (launch_bro_ell_tma<T, V, 8, 1>(A, x, y, st)) return;
+    launch_bro_ell_cfg<T, V, 8, 4, 4>(A, x, y, st);
+    return;
   }
-  launch_bro_ell_cfg<T, V, 8, 4, 4>(A, x, y, st);
+  launch_bro_ell_od<T, V, 8, 4>(A, x, y, st);
 }
 
 template <typename T>

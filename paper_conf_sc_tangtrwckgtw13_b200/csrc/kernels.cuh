@@ -266,6 +266,144 @@ bro_ell_spmv(int64_t m, int64_t s, const uint32_t* __restrict__ words,
   }
 }
 
+// ------------------------------------------------------------------ BRO-ELL, offset decode
+// Widths are warp-uniform (one per slice column), so the bit offset
+// of column j inside every row stream is the same for all 32 lanes:
+// o_j = sum_{i<j} b_i.  Per block of up to 32 columns the warp computes the
+// offsets with one SHFL scan, stages the block's symbols (<= 33 per lane) in
+// a per-warp shared window as [row][lane] (conflict-free), and then each
+// column's delta is a branch-free extraction
+//     delta = funnelshift(w[q+1], w[q], o mod 32) >> (32 - b),   q = o / 32
+// fused with the x gather and the FMA (8 columns in flight per group).
+__device__ __forceinline__ uint32_t shr_clamp(uint32_t v, uint32_t s) {
+  uint32_t r;
+  asm("shr.b32 %0, %1, %2;" : "=r"(r) : "r"(v), "r"(s));
+  return r;
+}
+
+// Copy symbol rows [qa, qa + nrows) of this lane into win[(q - qa) * 32 + lane]
+// (zeros past S) plus one zero guard row.
+template <int V>
+__device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __restrict__ wb, int S, int qa,
+                                              int nrows, int lane) {
+  if constexpr (V == 1) {
+    for (int r = 0; r < nrows; ++r) {
+      const int q = qa + r;
+      win[r * 32 + lane] = q < S ? __ldg(wb + 32 * q + lane) : 0u;
+    }
+  } else if constexpr (V == 4) {
+    const int F = S >> 2;
+    const int c_lo = qa >> 2, c_hi = (qa + nrows - 1) >> 2;
+    for (int c = c_lo; c <= c_hi; ++c) {
+      uint32_t w4[4];
+      if (c < F) {
+        const uint4 v = ld_stream_u4(wb + 128 * c + 4 * lane);
+        w4[0] = v.x; w4[1] = v.y; w4[2] = v.z; w4[3] = v.w;
+      } else {
+        const int Vp = S - 4 * F;
+#pragma unroll
+        for (int k = 0; k < 4; ++k) w4[k] = (c == F && k < Vp) ? ld_stream_u32(wb + 128 * F + Vp * lane + k) : 0u;
+      }
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const int r = 4 * c + k - qa;
+        if (r >= 0 && r < nrows) win[r * 32 + lane] = w4[k];
+      }
+    }
+  } else {
+    for (int r = 0; r < nrows; ++r) {
+      const int q = qa + r;
+      win[r * 32 + lane] = q < S ? ld_stream_u32(wb + place(lane, q, S, V)) : 0u;
+    }
+  }
+  win[nrows * 32 + lane] = 0u;
+}
+
+template <typename T, int V, int kWarps, int kMinBlocks>
+__global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
+bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
+                const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
+                const uint64_t* __restrict__ symptr, const T* __restrict__ vals,
+                const T* __restrict__ x, T* __restrict__ y) {
+  constexpr int G = 8;
+  constexpr int kRows = 34;
+  __shared__ uint32_t window[kWarps][kRows * 32];
+  __shared__ uint2 colmeta[kWarps][32];  // per column of the block: {byte offset of its word row, r | (32-b) << 8}
+  const int lane = threadIdx.x & 31;
+  const int w = threadIdx.x >> 5;
+  uint32_t* win = window[w];
+  const uint2* cm = colmeta[w];
+  const char* win_lane = reinterpret_cast<const char*>(win + lane);
+  const int64_t stride = int64_t(gridDim.x) * kWarps;
+  for (int64_t t = int64_t(blockIdx.x) * kWarps + w; t < s; t += stride) {
+    const uint64_t c0 = __ldg(colptr + t);
+    const int l = int(__ldg(colptr + t + 1) - c0);
+    const uint64_t q0 = __ldg(symptr + t);
+    const int S = int(__ldg(symptr + t + 1) - q0);
+    const uint32_t* wb = words + 32 * q0;
+    const T* vs = vals + 32 * c0;
+    const uint8_t* ba = bit_alloc + c0;
+    const int lfull = (l / Chunk<T>::N) * Chunk<T>::N;
+    T sum = T(0);
+    int col = -1;
+    int obase = 0;  // bit offset of the current block inside every row stream
+    for (int jb = 0; jb < l; jb += 32) {
+      const int nb = min(32, l - jb);
+      const int b = lane < nb ? int(__ldg(ba + jb + lane)) : 0;
+      int incl = b;  // inclusive scan of the widths over the block
+#pragma unroll
+      for (int off = 1; off < 32; off <<= 1) {
+        const int o = __shfl_up_sync(0xffffffffu, incl, off);
+        if (lane >= off) incl += o;
+      }
+      const int tot = __shfl_sync(0xffffffffu, incl, 31);
+      const int qa = obase >> 5;
+      const int nrows = tot > 0 ? ((obase + tot - 1) >> 5) - qa + 1 : 0;
+      __syncwarp();
+      stage_symbols<V>(win, wb, S, qa, nrows, lane);
+      {
+        const int rel = b ? obase + incl - b - 32 * qa : 0;  // column jb+lane inside the window
+        colmeta[w][lane] = make_uint2(uint32_t(rel >> 5) * 128u, uint32_t(rel & 31) | ((32u - uint32_t(b)) << 8));
+      }
+      __syncwarp();
+      for (int g = 0; g < nb; g += G) {
+        T v[G];
+        if (jb + g + G <= lfull) {  // all chunks of the group are full 16-byte chunks
+#pragma unroll
+          for (int u = 0; u < G / Chunk<T>::N; ++u) {
+            Chunk<T> c;
+            c.load(vs + 32 * (jb + g + u * Chunk<T>::N) + lane * Chunk<T>::N);
+#pragma unroll
+            for (int q = 0; q < Chunk<T>::N; ++q) v[u * Chunk<T>::N + q] = c.v[q];
+          }
+        } else {
+          load_group_vals<T, G>(v, vs, jb + g, l, lfull, lane);
+        }
+        int cidx[G];
+        bool ok[G];
+#pragma unroll
+        for (int k = 0; k < G; ++k) {
+          const uint2 mm = cm[g + k];  // broadcast
+          const uint32_t* wp = reinterpret_cast<const uint32_t*>(win_lane + mm.x);
+          // funnelshift_l uses the low 5 bits of mm.y (= r); bits 8.. hold 32-b
+          const uint32_t d = shr_clamp(__funnelshift_l(wp[32], wp[0], mm.y), mm.y >> 8);
+          col += int(d);
+          cidx[k] = col;
+          ok[k] = d != 0u;
+        }
+        T xv[G];
+#pragma unroll
+        for (int k = 0; k < G; ++k) xv[k] = ok[k] ? ldg_x(x + cidx[k]) : T(0);
+#pragma unroll
+        for (int k = 0; k < G; ++k) sum = fma(v[k], xv[k], sum);
+      }
+      obase += tot;
+    }
+    const int64_t row = 32 * t + lane;
+    if (row < m) y[row] = sum;
+  }
+}
+
 // ------------------------------------------------------------------ BRO-ELL, TMA pipeline
 // Warp-specialised persistent kernel.  Block b owns slices t_k = b + k*gridDim.x.
 // Producer warp: loads the metadata of 32 upcoming slices at once (one slice
