@@ -49,7 +49,7 @@ def parse_args():
     ap.add_argument("--workload", default="C5", choices=sorted(WORKLOADS))
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--vec-words", type=int, default=1)
+    ap.add_argument("--vec-words", type=int, default=4)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--flush-l2", action="store_true", help="write a 2xL2 buffer between steps")
@@ -354,8 +354,7 @@ def main():
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
                      "peak_kind": peak_kind,
-                     "kernel": (f"bro_ell_spmv_pf<{'double' if dtype == np.float64 else 'float'}>" if args.vec_words == 1 else
-                                f"bro_ell_spmv_od<{'double' if dtype == np.float64 else 'float'},V={args.vec_words}>")
+                     "kernel": f"bro_ell_spmv_od<{'double' if dtype == np.float64 else 'float'},V={args.vec_words}>"
                      if fmt == "ell" else "bro_ell_spmv + coo_spmv + coo_fixup",
                      "algorithmic_bytes_per_launch": alg_bytes, "kernel_ms": kern_ms,
                      "frac_of_8TBps_spec": achieved / 8000.0},

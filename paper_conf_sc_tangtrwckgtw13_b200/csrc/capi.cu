@@ -368,26 +368,6 @@ void launch_bro_ell_od(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
                                      (const T*)A->d_ell_vals, x, y);
 }
 
-template <typename T, int kWarps, int kMinBlocks>
-void launch_bro_ell_pf(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
-  using namespace bro::dev;
-  auto kern = bro_ell_spmv_pf<T, kWarps, kMinBlocks>;
-  constexpr int smem = kWarps * kPfWarpBytes;
-  static int resident = 0;
-  if (resident == 0) {
-    int per_sm = 0, sms = 0, dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kWarps * 32, smem);
-    resident = std::max(1, per_sm) * std::max(1, sms);
-  }
-  const int64_t need = (A->s + kWarps - 1) / kWarps;
-  const unsigned grid = (unsigned)std::min<int64_t>(need, resident);
-  kern<<<grid, kWarps * 32, smem, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr,
-                                        (const T*)A->d_ell_vals, x, y);
-}
-
 // Tuning knob (not part of the ABI): BRO_ELL_VARIANT selects a compiled
 // launch configuration for V = 4; read once per process.
 int ell_variant() {
@@ -401,14 +381,7 @@ int ell_variant() {
 
 template <typename T, int V>
 void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
-  if constexpr (V == 1) {
-    switch (ell_variant()) {
-      case 1: return launch_bro_ell_pf<T, 8, 2>(A, x, y, st);
-      case 2: return launch_bro_ell_pf<T, 4, 6>(A, x, y, st);
-      case 3: return launch_bro_ell_od<T, V, 8, 4>(A, x, y, st);
-      default: return launch_bro_ell_pf<T, 8, 3>(A, x, y, st);
-    }
-  } else if constexpr (V == 4) {
+  if constexpr (V == 4) {
     switch (ell_variant()) {
       case 5:
         if (launch_bro_ell_tma<T, V, 8, 2>(A, x, y, st)) return;
@@ -513,7 +486,7 @@ void bro_opts_default(bro_opts_t* o) {
   if (!o) return;
   o->slice_h = 32;
   o->sym_bits = 32;
-  o->vec_words = 1;
+  o->vec_words = 4;
   o->coo_T = 32;
   o->hyb_K = -1;
   o->codec = 1;

@@ -408,168 +408,6 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
   }
 }
 
-// ------------------------------------------------------------------ BRO-ELL, offset decode + prefetch (V = 1)
-// Same decode as bro_ell_spmv_od, for the paper's multiplexing (V = 1: symbol
-// q of lane r at 32*q + r, so a slice's symbols are contiguous 128-byte rows).
-// While slice t is multiplied, the warp already has slice t+1's symbol rows
-// and first-block widths in flight into the other half of a double-buffered
-// shared window (16-byte cp.async, zero-filled past S), and slice t+2's
-// metadata in registers: the per-slice chain metadata -> widths/symbols ->
-// scan no longer stalls the warp.
-__device__ __forceinline__ void cp_async16(void* dst, const void* src, uint32_t src_bytes) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;"
-               :: "r"(smem_u32(dst)), "l"(src), "r"(src_bytes) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" :: "n"(N) : "memory"); }
-
-struct SliceMeta {
-  uint64_t c0, q0;
-  int l, S;
-};
-
-__device__ __forceinline__ SliceMeta load_meta(const uint64_t* __restrict__ colptr,
-                                               const uint64_t* __restrict__ symptr, int64_t t) {
-  SliceMeta mt;
-  mt.c0 = __ldg(colptr + t);
-  mt.l = int(__ldg(colptr + t + 1) - mt.c0);
-  mt.q0 = __ldg(symptr + t);
-  mt.S = int(__ldg(symptr + t + 1) - mt.q0);
-  return mt;
-}
-
-constexpr int kPfRows = 34;                       // symbol rows per window (33 + guard)
-constexpr int kPfWinBytes = kPfRows * 32 * 4;     // 4352
-constexpr int kPfWarpBytes = 2 * kPfWinBytes + 2 * 64 + 32 * 8;
-
-// Issue the copies of slice mt's first symbol window (rows [0, min(S+1, R)),
-// rows >= S zero-filled) and of its first-block widths (16-byte window).
-__device__ __forceinline__ void pf_issue(const SliceMeta& mt, const uint32_t* __restrict__ words,
-                                         const uint8_t* __restrict__ bit_alloc, uint32_t* win,
-                                         uint8_t* bab, int lane) {
-  const int nr = min(mt.S + 1, kPfRows);
-  const uint32_t* wb = words + 32 * mt.q0;
-  for (int p = lane; p < nr * 8; p += 32) {
-    const int row = p >> 3;
-    cp_async16(win + 4 * p, row < mt.S ? wb + 4 * p : wb, row < mt.S ? 16u : 0u);
-  }
-  if (mt.l > 0) {
-    const uint64_t lo = mt.c0 & ~uint64_t(15);
-    const uint64_t hi = (mt.c0 + uint64_t(min(mt.l, 32)) + 15) & ~uint64_t(15);
-    if (lane < int((hi - lo) >> 4)) cp_async16(bab + 16 * lane, bit_alloc + lo + 16 * lane, 16u);
-  }
-}
-
-template <typename T, int kWarps, int kMinBlocks>
-__global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
-bro_ell_spmv_pf(int64_t m, int64_t s, const uint32_t* __restrict__ words,
-                const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
-                const uint64_t* __restrict__ symptr, const T* __restrict__ vals,
-                const T* __restrict__ x, T* __restrict__ y) {
-  constexpr int G = 8;
-  constexpr int VV = Chunk<T>::N;
-  extern __shared__ __align__(16) uint8_t dsm[];
-  const int lane = threadIdx.x & 31;
-  const int w = threadIdx.x >> 5;
-  uint8_t* wbase = dsm + size_t(w) * kPfWarpBytes;
-  uint2* cm = reinterpret_cast<uint2*>(wbase + 2 * kPfWinBytes + 128);
-  const int64_t stride = int64_t(gridDim.x) * kWarps;
-  int64_t t = int64_t(blockIdx.x) * kWarps + w;
-  if (t >= s) return;
-  SliceMeta cur = load_meta(colptr, symptr, t);
-  pf_issue(cur, words, bit_alloc, reinterpret_cast<uint32_t*>(wbase), wbase + 2 * kPfWinBytes, lane);
-  cp_async_commit();
-  SliceMeta nxt{0, 0, 0, 0};
-  if (t + stride < s) nxt = load_meta(colptr, symptr, t + stride);
-  int buf = 0;
-  for (; t < s; t += stride, buf ^= 1) {
-    SliceMeta nn{0, 0, 0, 0};
-    if (t + 2 * stride < s) nn = load_meta(colptr, symptr, t + 2 * stride);
-    if (t + stride < s)
-      pf_issue(nxt, words, bit_alloc, reinterpret_cast<uint32_t*>(wbase + (buf ^ 1) * kPfWinBytes),
-               wbase + 2 * kPfWinBytes + 64 * (buf ^ 1), lane);
-    cp_async_commit();
-    cp_async_wait<1>();  // this slice's copies (all but the newest group) have landed
-    __syncwarp();
-    uint32_t* win = reinterpret_cast<uint32_t*>(wbase + buf * kPfWinBytes);
-    const uint8_t* bab = wbase + 2 * kPfWinBytes + 64 * buf;
-    const char* win_lane = reinterpret_cast<const char*>(win + lane);
-    const int l = cur.l, S = cur.S;
-    const T* vs = vals + 32 * cur.c0;
-    const uint8_t* ba = bit_alloc + cur.c0;
-    const int lfull = (l / VV) * VV;
-    int wq0 = 0, wvalid = min(S + 1, kPfRows);
-    T sum = T(0);
-    int col = -1;
-    int obase = 0;
-    for (int jb = 0; jb < l; jb += 32) {
-      const int nb = min(32, l - jb);
-      int b = 0;
-      if (lane < nb) b = jb == 0 ? int(bab[int(cur.c0 & 15) + lane]) : int(__ldg(ba + jb + lane));
-      int incl = b;
-#pragma unroll
-      for (int off = 1; off < 32; off <<= 1) {
-        const int o = __shfl_up_sync(0xffffffffu, incl, off);
-        if (lane >= off) incl += o;
-      }
-      const int tot = __shfl_sync(0xffffffffu, incl, 31);
-      const int qa = obase >> 5;
-      const int nrows = tot > 0 ? ((obase + tot - 1) >> 5) - qa + 1 : 0;
-      if (qa < wq0 || qa + nrows + 1 > wq0 + wvalid) {  // block outside the staged window: reload
-        __syncwarp();
-        const uint32_t* wb = words + 32 * cur.q0;
-        for (int r = 0; r < nrows; ++r) win[r * 32 + lane] = (qa + r < S) ? __ldg(wb + 32 * (qa + r) + lane) : 0u;
-        win[nrows * 32 + lane] = 0u;
-        wq0 = qa;
-        wvalid = nrows + 1;
-      }
-      {
-        const int rel = b ? obase + incl - b - 32 * wq0 : 0;
-        cm[lane] = make_uint2(uint32_t(rel >> 5) * 128u, uint32_t(rel & 31) | ((32u - uint32_t(b)) << 8));
-      }
-      __syncwarp();
-      for (int g = 0; g < nb; g += G) {
-        T v[G];
-        if (jb + g + G <= lfull) {
-#pragma unroll
-          for (int u = 0; u < G / VV; ++u) {
-            Chunk<T> c;
-            c.load(vs + 32 * (jb + g + u * VV) + lane * VV);
-#pragma unroll
-            for (int q = 0; q < VV; ++q) v[u * VV + q] = c.v[q];
-          }
-        } else {
-          load_group_vals<T, G>(v, vs, jb + g, l, lfull, lane);
-        }
-        int cidx[G];
-        bool ok[G];
-#pragma unroll
-        for (int k = 0; k < G; ++k) {
-          const uint2 mm = cm[g + k];
-          const uint32_t* wp = reinterpret_cast<const uint32_t*>(win_lane + mm.x);
-          const uint32_t d = shr_clamp(__funnelshift_l(wp[32], wp[0], mm.y), mm.y >> 8);
-          col += int(d);
-          cidx[k] = col;
-          ok[k] = d != 0u;
-        }
-        T xv[G];
-#pragma unroll
-        for (int k = 0; k < G; ++k) xv[k] = ok[k] ? ldg_x(x + cidx[k]) : T(0);
-#pragma unroll
-        for (int k = 0; k < G; ++k) sum = fma(v[k], xv[k], sum);
-      }
-      obase += tot;
-      __syncwarp();
-    }
-    const int64_t row = 32 * t + lane;
-    if (row < m) y[row] = sum;
-    cur = nxt;
-    nxt = nn;
-  }
-  cp_async_wait<0>();
-}
-
 // ------------------------------------------------------------------ BRO-ELL, TMA pipeline
 // Warp-specialised persistent kernel.  Block b owns slices t_k = b + k*gridDim.x.
 // Producer warp: loads the metadata of 32 upcoming slices at once (one slice

@@ -22,7 +22,7 @@ def dev():
     return torch.device("cuda:0")
 
 
-def _run(lib, A, fmt, codec, dtype, dev, V=1, x=None, stream=None):
+def _run(lib, A, fmt, codec, dtype, dev, V=4, x=None, stream=None):
     M = lib.BroMatrix(A, fmt=fmt, codec=codec, device=0, dtype=dtype, vec_words=V)
     if x is None:
         x = make_x(A.n, 3, dtype)
