@@ -331,20 +331,32 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
                 const T* __restrict__ x, T* __restrict__ y) {
   constexpr int G = 8;
   constexpr int kRows = 34;
+  struct Meta { uint64_t c0, q0; int l, S; };
   __shared__ uint32_t window[kWarps][kRows * 32];
   __shared__ uint2 colmeta[kWarps][32];  // per column of the block: {byte offset of its word row, r | (32-b) << 8}
+  __shared__ Meta metas[kWarps][32];     // metadata of this warp's next 32 slices
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
   uint32_t* win = window[w];
   const uint2* cm = colmeta[w];
   const char* win_lane = reinterpret_cast<const char*>(win + lane);
   const int64_t stride = int64_t(gridDim.x) * kWarps;
-  for (int64_t t = int64_t(blockIdx.x) * kWarps + w; t < s; t += stride) {
-    const uint64_t c0 = __ldg(colptr + t);
-    const int l = int(__ldg(colptr + t + 1) - c0);
-    const uint64_t q0 = __ldg(symptr + t);
-    const int S = int(__ldg(symptr + t + 1) - q0);
-    const uint32_t* wb = words + 32 * q0;
+  int k32 = 0;
+  for (int64_t t = int64_t(blockIdx.x) * kWarps + w; t < s; t += stride, k32 = (k32 + 1) & 31) {
+    __syncwarp();
+    if (k32 == 0) {  // one round trip fetches the metadata of the next 32 slices
+      const int64_t tl = t + lane * stride;
+      if (tl < s) {
+        const uint64_t c0l = __ldg(colptr + tl), q0l = __ldg(symptr + tl);
+        metas[w][lane] = Meta{c0l, q0l, int(__ldg(colptr + tl + 1) - c0l), int(__ldg(symptr + tl + 1) - q0l)};
+      }
+      __syncwarp();
+    }
+    const Meta mt = metas[w][k32];
+    const uint64_t c0 = mt.c0;
+    const int l = mt.l;
+    const int S = mt.S;
+    const uint32_t* wb = words + 32 * mt.q0;
     const T* vs = vals + 32 * c0;
     const uint8_t* ba = bit_alloc + c0;
     const int lfull = (l / Chunk<T>::N) * Chunk<T>::N;
@@ -354,6 +366,10 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
     for (int jb = 0; jb < l; jb += 32) {
       const int nb = min(32, l - jb);
       const int b = lane < nb ? int(__ldg(ba + jb + lane)) : 0;
+      if (jb == 0) {  // first block starts at symbol 0: stage without waiting for the scan
+        __syncwarp();
+        stage_symbols<V>(win, wb, S, 0, min(S, kRows - 1), lane);
+      }
       int incl = b;  // inclusive scan of the widths over the block
 #pragma unroll
       for (int off = 1; off < 32; off <<= 1) {
@@ -361,10 +377,12 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
         if (lane >= off) incl += o;
       }
       const int tot = __shfl_sync(0xffffffffu, incl, 31);
-      const int qa = obase >> 5;
+      const int qa = jb == 0 ? 0 : obase >> 5;
       const int nrows = tot > 0 ? ((obase + tot - 1) >> 5) - qa + 1 : 0;
-      __syncwarp();
-      stage_symbols<V>(win, wb, S, qa, nrows, lane);
+      if (jb > 0) {
+        __syncwarp();
+        stage_symbols<V>(win, wb, S, qa, nrows, lane);
+      }
       {
         const int rel = b ? obase + incl - b - 32 * qa : 0;  // column jb+lane inside the window
         colmeta[w][lane] = make_uint2(uint32_t(rel >> 5) * 128u, uint32_t(rel & 31) | ((32u - uint32_t(b)) << 8));
@@ -397,9 +415,11 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
         }
         T xv[G];
 #pragma unroll
-        for (int k = 0; k < G; ++k) xv[k] = ok[k] ? ldg_x(x + cidx[k]) : T(0);
+        for (int k = 0; k < G; ++k)
+          if (ok[k]) xv[k] = ldg_x(x + cidx[k]);
 #pragma unroll
-        for (int k = 0; k < G; ++k) sum = fma(v[k], xv[k], sum);
+        for (int k = 0; k < G; ++k)
+          if (ok[k]) sum = fma(v[k], xv[k], sum);  // padding slots (delta 0) are skipped, Alg. 1 line 17
       }
       obase += tot;
     }
@@ -721,42 +741,56 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, const uint32_t* __restrict__ word
   }
   T carry = T(0);
   int crow = first;
-  for (int t = 0; t < T_steps; ++t) {
-    const int64_t e = e0 + 32 * t + lane;
-    const bool valid = e < nnz;
-    if constexpr (kBro) {
-      if (b) row += (int)ls.get(b, lane);
-    } else {
-      row = ld_stream_s32(rows + (valid ? e : nnz - 1));
-    }
-    T p = T(0);
-    if (valid) p = ld_stream(vals + e) * ldg_x(x + ld_stream_s32(col + e));
-    // the carried row ended at the previous step's last lane
-    const int row0 = __shfl_sync(0xffffffffu, row, 0);
-    if (row0 != crow) {
-      if (lane == 0) {
-        if (crow == first) carry_first[i] = carry;
-        else y[crow] += carry;
-      }
-      carry = T(0);
-      crow = row0;
-    }
-    // inclusive segmented scan over lanes (rows are non-decreasing)
-    T sc = p;
+  constexpr int TB = 8;  // steps whose loads are all in flight before the scans
+  for (int t0 = 0; t0 < T_steps; t0 += TB) {
+    int rw[TB], cl[TB];
+    T vl[TB], xv[TB];
 #pragma unroll
-    for (int off = 1; off < 32; off <<= 1) {
-      const T o = __shfl_up_sync(0xffffffffu, sc, off);
-      const int ro = __shfl_up_sync(0xffffffffu, row, off);
-      if (lane >= off && ro == row) sc += o;
+    for (int k = 0; k < TB; ++k) {  // rows (decode or load), columns, values
+      const int64_t e = e0 + 32 * (t0 + k) + lane;
+      const bool valid = e < nnz;
+      if constexpr (kBro) {
+        if (b) row += (int)ls.get(b, lane);
+        rw[k] = row;
+      } else {
+        rw[k] = ld_stream_s32(rows + (valid ? e : nnz - 1));
+      }
+      cl[k] = valid ? ld_stream_s32(col + e) : -1;
+      vl[k] = valid ? ld_stream(vals + e) : T(0);
     }
-    if (row == crow) sc += carry;
-    const int rn = __shfl_down_sync(0xffffffffu, row, 1);
-    if (lane != 31 && rn != row) {
-      if (row == first) carry_first[i] = sc;
-      else y[row] += sc;
+#pragma unroll
+    for (int k = 0; k < TB; ++k) xv[k] = cl[k] >= 0 ? ldg_x(x + cl[k]) : T(0);
+#pragma unroll
+    for (int k = 0; k < TB; ++k) {
+      const T p = vl[k] * xv[k];
+      const int row = rw[k];
+      // the carried row ended at the previous step's last lane
+      const int row0 = __shfl_sync(0xffffffffu, row, 0);
+      if (row0 != crow) {
+        if (lane == 0) {
+          if (crow == first) carry_first[i] = carry;
+          else y[crow] += carry;
+        }
+        carry = T(0);
+        crow = row0;
+      }
+      // inclusive segmented scan over lanes (rows are non-decreasing)
+      T sc = p;
+#pragma unroll
+      for (int off = 1; off < 32; off <<= 1) {
+        const T o = __shfl_up_sync(0xffffffffu, sc, off);
+        const int ro = __shfl_up_sync(0xffffffffu, row, off);
+        if (lane >= off && ro == row) sc += o;
+      }
+      if (row == crow) sc += carry;
+      const int rn = __shfl_down_sync(0xffffffffu, row, 1);
+      if (lane != 31 && rn != row) {
+        if (row == first) carry_first[i] = sc;
+        else y[row] += sc;
+      }
+      carry = __shfl_sync(0xffffffffu, sc, 31);
+      crow = __shfl_sync(0xffffffffu, row, 31);
     }
-    carry = __shfl_sync(0xffffffffu, sc, 31);
-    crow = __shfl_sync(0xffffffffu, row, 31);
   }
   if (lane == 0) {
     last_row[i] = crow;
