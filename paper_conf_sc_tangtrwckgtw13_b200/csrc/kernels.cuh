@@ -715,9 +715,38 @@ __global__ void ell_decode(int64_t m, int64_t K, int64_t pitch, const int32_t* _
 }
 
 // ------------------------------------------------------------------ (BRO-)COO
-// One warp per interval of 32*T entries.  Entry e0 + 32t + lane is element
-// (t, lane).  Rows of fully-contained rows are added into y directly; the
-// first row's and last row's partial sums go to carry arrays for the fix-up.
+// One warp per interval of 32*T entries.  BRO row deltas are laid
+// out per (step t, lane) (element (t, lane) = entry e0 + 32t + lane), so each
+// lane first decodes its rows for 8 steps into a per-warp shared buffer.  The
+// multiply is then done TRANSPOSED: lane l owns the 8 consecutive entries
+// 8l .. 8l+7 of the 256-entry batch (16-byte loads of col / vals, which are in
+// plain COO order), reduces them sequentially, and one warp-level segmented
+// scan over the lanes' trailing partials (the "parallel scan primitive" of
+// P:L343) links segments that cross lanes.  Complete segments of rows other
+// than the interval's first row are added into y directly (each such row
+// lives in exactly one interval); the first and last rows' partials go to
+// carry arrays for the deterministic fix-up kernel.
+template <typename T>
+struct Vec8 {  // 8 consecutive values of one lane, loaded as 16-byte chunks
+  T v[8];
+  __device__ __forceinline__ void load(const T* p) {
+#pragma unroll
+    for (int u = 0; u < 8 / Chunk<T>::N; ++u) {
+      Chunk<T> c;
+      c.load(p + u * Chunk<T>::N);
+#pragma unroll
+      for (int q = 0; q < Chunk<T>::N; ++q) v[u * Chunk<T>::N + q] = c.v[q];
+    }
+  }
+};
+
+__device__ __forceinline__ void load8_s32(int* d, const int32_t* p) {
+  const uint4 a = ld_stream_u4(reinterpret_cast<const uint32_t*>(p));
+  const uint4 b = ld_stream_u4(reinterpret_cast<const uint32_t*>(p) + 4);
+  d[0] = int(a.x); d[1] = int(a.y); d[2] = int(a.z); d[3] = int(a.w);
+  d[4] = int(b.x); d[5] = int(b.y); d[6] = int(b.z); d[7] = int(b.w);
+}
+
 template <typename T, int V, bool kBro, int kThreads>
 __global__ void __launch_bounds__(kThreads)
 coo_spmv(int64_t nnz, int64_t nI, int T_steps, const uint32_t* __restrict__ words,
@@ -726,9 +755,13 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, const uint32_t* __restrict__ word
          const int32_t* __restrict__ col, const T* __restrict__ vals, const T* __restrict__ x,
          T* __restrict__ y, T* __restrict__ carry_first, T* __restrict__ carry_last,
          int32_t* __restrict__ last_row) {
+  constexpr int TB = 8;
+  __shared__ __align__(16) int32_t rowbuf[kThreads / 32][TB * 32];
   const int lane = threadIdx.x & 31;
-  const int64_t i = int64_t(blockIdx.x) * (kThreads / 32) + (threadIdx.x >> 5);
+  const int w = threadIdx.x >> 5;
+  const int64_t i = int64_t(blockIdx.x) * (kThreads / 32) + w;
   if (i >= nI) return;
+  int32_t* rb = rowbuf[w];
   const int64_t e0 = i * 32 * T_steps;
   const int first = (int)base_row[i];
   int row = first;
@@ -739,58 +772,95 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, const uint32_t* __restrict__ word
     const uint64_t q0 = symptr[i];
     ls.init(words + 32 * q0, int(symptr[i + 1] - q0), lane);
   }
-  T carry = T(0);
+  T carry = T(0);   // partial of row crow carried from earlier batches (not yet written)
   int crow = first;
-  constexpr int TB = 8;  // steps whose loads are all in flight before the scans
+  auto emit = [&](int r, T v) {  // a complete segment of row r
+    if (r == first) carry_first[i] = v;
+    else y[r] += v;
+  };
   for (int t0 = 0; t0 < T_steps; t0 += TB) {
-    int rw[TB], cl[TB];
-    T vl[TB], xv[TB];
+    const int64_t eb = e0 + 32 * t0;            // first entry of the batch
+    const int64_t el = eb + TB * lane;          // this lane's first entry (transposed)
+    int r[TB], c[TB];
+    T v[TB];
+    if constexpr (kBro) {
 #pragma unroll
-    for (int k = 0; k < TB; ++k) {  // rows (decode or load), columns, values
-      const int64_t e = e0 + 32 * (t0 + k) + lane;
-      const bool valid = e < nnz;
-      if constexpr (kBro) {
+      for (int k = 0; k < TB; ++k) {  // decode rows of steps t0..t0+7 for (t, lane)
         if (b) row += (int)ls.get(b, lane);
-        rw[k] = row;
-      } else {
-        rw[k] = ld_stream_s32(rows + (valid ? e : nnz - 1));
+        rb[k * 32 + lane] = row;
       }
-      cl[k] = valid ? ld_stream_s32(col + e) : -1;
-      vl[k] = valid ? ld_stream(vals + e) : T(0);
+      __syncwarp();
+      const int4 ra = *reinterpret_cast<const int4*>(rb + TB * lane);
+      const int4 rc = *reinterpret_cast<const int4*>(rb + TB * lane + 4);
+      r[0] = ra.x; r[1] = ra.y; r[2] = ra.z; r[3] = ra.w;
+      r[4] = rc.x; r[5] = rc.y; r[6] = rc.z; r[7] = rc.w;
+      __syncwarp();
     }
+    if (el + TB <= nnz) {
+      if constexpr (!kBro) load8_s32(r, rows + el);
+      load8_s32(c, col + el);
+      Vec8<T> vv;
+      vv.load(vals + el);
 #pragma unroll
-    for (int k = 0; k < TB; ++k) xv[k] = cl[k] >= 0 ? ldg_x(x + cl[k]) : T(0);
+      for (int k = 0; k < TB; ++k) v[k] = vv.v[k];
+    } else {  // tail of the last interval: entries past nnz repeat the last row with value 0
+#pragma unroll
+      for (int k = 0; k < TB; ++k) {
+        const bool ok = el + k < nnz;
+        if constexpr (!kBro) r[k] = ld_stream_s32(rows + (ok ? el + k : nnz - 1));
+        c[k] = ok ? ld_stream_s32(col + el + k) : -1;
+        v[k] = ok ? ld_stream(vals + el + k) : T(0);
+      }
+    }
+    T xv[TB];
+#pragma unroll
+    for (int k = 0; k < TB; ++k) xv[k] = c[k] >= 0 ? ldg_x(x + c[k]) : T(0);
+    // sequential pass over the lane's 8 entries
+    const int f = r[0];
+    T A = T(0), cur = T(0);
+    bool one = true;
+    int cr = f;
 #pragma unroll
     for (int k = 0; k < TB; ++k) {
-      const T p = vl[k] * xv[k];
-      const int row = rw[k];
-      // the carried row ended at the previous step's last lane
-      const int row0 = __shfl_sync(0xffffffffu, row, 0);
-      if (row0 != crow) {
-        if (lane == 0) {
-          if (crow == first) carry_first[i] = carry;
-          else y[crow] += carry;
-        }
-        carry = T(0);
-        crow = row0;
+      const T p = v[k] * xv[k];
+      if (r[k] != cr) {           // the segment of row cr ends inside this lane
+        if (one) { A = cur; one = false; }
+        else emit(cr, cur);       // interior segment: complete, row unique to this lane
+        cr = r[k];
+        cur = p;
+      } else {
+        cur += p;
       }
-      // inclusive segmented scan over lanes (rows are non-decreasing)
-      T sc = p;
-#pragma unroll
-      for (int off = 1; off < 32; off <<= 1) {
-        const T o = __shfl_up_sync(0xffffffffu, sc, off);
-        const int ro = __shfl_up_sync(0xffffffffu, row, off);
-        if (lane >= off && ro == row) sc += o;
-      }
-      if (row == crow) sc += carry;
-      const int rn = __shfl_down_sync(0xffffffffu, row, 1);
-      if (lane != 31 && rn != row) {
-        if (row == first) carry_first[i] = sc;
-        else y[row] += sc;
-      }
-      carry = __shfl_sync(0xffffffffu, sc, 31);
-      crow = __shfl_sync(0xffffffffu, row, 31);
     }
+    if (one) A = cur;
+    const int L = cr;             // trailing segment: row L, partial cur
+    // carry-in from earlier lanes (or earlier batches for lane 0)
+    const int Lprev = __shfl_up_sync(0xffffffffu, L, 1);
+    const bool link = lane == 0 ? (crow == f) : (Lprev == f);
+    // C_out(l) = B_l + [one_l && link_l] * C_out(l-1): segmented scan
+    T co = cur;
+    bool open = one && link;      // this lane's partial continues an earlier one
+    if (lane == 0 && open) co += carry;
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+      const T o = __shfl_up_sync(0xffffffffu, co, off);
+      const int op = __shfl_up_sync(0xffffffffu, int(open), off);
+      if (lane >= off && open) co += o;
+      if (lane >= off) open = open && op;
+    }
+    // C_in = C_out(l-1) if linked; lane 0 takes the batch carry
+    T cin = __shfl_up_sync(0xffffffffu, co, 1);
+    if (lane == 0) cin = carry;
+    if (!link) cin = T(0);
+    if (lane == 0 && !link && crow != f) {
+      // the carried row ended before this batch
+      emit(crow, carry);
+    }
+    if (!one) emit(f, A + cin);   // first segment complete inside this lane
+    const int fnext = __shfl_down_sync(0xffffffffu, f, 1);
+    if (lane < 31 && fnext != L) emit(L, co);  // trailing segment complete at this lane
+    carry = __shfl_sync(0xffffffffu, co, 31);
+    crow = __shfl_sync(0xffffffffu, L, 31);
   }
   if (lane == 0) {
     last_row[i] = crow;
