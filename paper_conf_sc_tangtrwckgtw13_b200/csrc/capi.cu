@@ -3,7 +3,6 @@
 
 #include <algorithm>
 #include <chrono>
-#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -21,7 +20,6 @@ bro_status_t fail(bro_status_t s, const std::string& msg) {
   return s;
 }
 
-constexpr int kEllThreads = 256;
 constexpr int kCooThreads = 256;
 constexpr int kPlainThreads = 256;
 
@@ -74,7 +72,6 @@ struct bro_matrix_s {
   void* d_xs = nullptr;
   void* d_ys = nullptr;
   int64_t device_bytes = 0;
-  int64_t stage_bytes = 0;  // TMA ring stage size (largest slice: values + symbols + widths window)
   bro_info_t info{};
 };
 
@@ -239,15 +236,6 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
 #define UP(dst, vec) \
   if (st == BRO_OK) st = dev_upload(A, &(dst), (vec).data(), (vec).size() * sizeof(*(vec).data()))
     if (A->has_ell && o.codec) {
-      int64_t need = 0;
-      for (int64_t t = 0; t < A->s; ++t) {
-        const uint64_t c0 = A->ell.colptr[t], c1 = A->ell.colptr[t + 1];
-        const int64_t b = int64_t(32 * (c1 - c0) * A->vsize + 128 * (A->ell.symptr[t + 1] - A->ell.symptr[t]) +
-                                  (((c1 + 15) & ~uint64_t(15)) - (c0 & ~uint64_t(15))));
-        need = std::max(need, b);
-      }
-      A->stage_bytes = (need + 127) / 128 * 128;
-      A->ell.bit_alloc.resize(A->ell.bit_alloc.size() + 16, 0);  // bulk copies read 16-byte windows
       UP(A->d_words, A->ell.words);
       UP(A->d_bit_alloc, A->ell.bit_alloc);
       UP(A->d_colptr, A->ell.colptr);
@@ -302,54 +290,6 @@ bro_status_t common_checks(bro_dtype_t dtype, const bro_opts_t* opts, bro_opts_t
 
 // Persistent grid: as many resident blocks as the SMs hold (queried once per
 // instantiation), capped by the number of slices.
-template <typename T, int V, int kWarps, int kMinBlocks, int G>
-void launch_bro_ell_cfg(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
-  using namespace bro::dev;
-  auto kern = bro_ell_spmv<T, V, kWarps, kMinBlocks, G>;
-  static int resident = 0;
-  if (resident == 0) {
-    int per_sm = 0, sms = 0, dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kWarps * 32, 0);
-    resident = std::max(1, per_sm) * std::max(1, sms);
-  }
-  const int64_t need = (A->s + kWarps - 1) / kWarps;
-  const unsigned grid = (unsigned)std::min<int64_t>(need, resident);
-  kern<<<grid, kWarps * 32, 0, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr,
-                                     (const T*)A->d_ell_vals, x, y);
-}
-
-// TMA-pipelined BRO-ELL.  The ring holds ncons * spc stages of
-// A->stage_bytes (the largest slice) in dynamic shared memory; ncons
-// consumer warps are active (<= kCons) so that each owns spc >= kMinSpc
-// stages.  Returns false when even one consumer cannot get kMinSpc stages.
-template <typename T, int V, int kCons, int kMinBlocks>
-bool launch_bro_ell_tma(bro_matrix_s* A, const T* x, T* y, cudaStream_t st, int min_spc = 2) {
-  using namespace bro::dev;
-  auto kern = bro_ell_spmv_tma<T, V, kCons, kMinBlocks>;
-  constexpr int kSmemPerBlock = (227 * 1024) / kMinBlocks - 1024;
-  static int sms = 0;
-  if (sms == 0) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemPerBlock);
-  }
-  const int64_t sb = std::max<int64_t>(A->stage_bytes, 128);
-  const int64_t fit = (kSmemPerBlock - 2048) / sb;           // stages that fit
-  const int ncons = (int)std::min<int64_t>(kCons, fit / min_spc);
-  if (ncons < 1) return false;
-  const int spc = (int)std::min<int64_t>(fit / ncons, 8);
-  const int nst = ncons * spc;
-  const size_t smem = size_t(((nst * (16 + 16)) + 127) / 128 * 128) + size_t(nst) * sb;
-  const int64_t grid = std::min<int64_t>(A->s, int64_t(sms) * kMinBlocks);
-  kern<<<(unsigned)grid, (kCons + 1) * 32, smem, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc, A->d_colptr,
-                                                       A->d_symptr, (const T*)A->d_ell_vals, x, y, ncons, spc,
-                                                       (int)sb);
-  return true;
-}
-
 template <typename T, int V, int kWarps, int kMinBlocks>
 void launch_bro_ell_od(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   using namespace bro::dev;
@@ -368,30 +308,12 @@ void launch_bro_ell_od(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
                                      (const T*)A->d_ell_vals, x, y);
 }
 
-// Tuning knob (not part of the ABI): BRO_ELL_VARIANT selects a compiled
-// launch configuration for V = 4; read once per process.
-int ell_variant() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("BRO_ELL_VARIANT");
-    v = e ? atoi(e) : 0;
-  }
-  return v;
-}
+constexpr int kEllWarps = 8;      // slices per block
+constexpr int kEllMinBlocks = 4;  // 32 resident warps per SM (64 registers)
 
 template <typename T, int V>
 void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
-  if constexpr (V == 4) {
-    switch (ell_variant()) {
-      case 5:
-        if (launch_bro_ell_tma<T, V, 8, 2>(A, x, y, st)) return;
-        if (launch_bro_ell_tma<T, V, 8, 1>(A, x, y, st)) return;
-        break;
-      case 8: return launch_bro_ell_cfg<T, V, 8, 4, 8>(A, x, y, st);
-      default: break;
-    }
-  }
-  launch_bro_ell_od<T, V, 8, 4>(A, x, y, st);
+  launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks>(A, x, y, st);
 }
 
 template <typename T>

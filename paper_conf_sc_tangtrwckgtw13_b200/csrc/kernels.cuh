@@ -3,20 +3,24 @@
 //
 // Mapping (B200-first; the paper's Fermi/Kepler mapping of one 256-thread
 // block per slice, is prior art):
-//   * BRO-ELL: one WARP per 32-row slice, one lane per row (h = 32).  Every
-//     per-column quantity of Alg. 1 (b = bit_alloc[c], rb, the refill branch)
-//     is warp-uniform, so decode has no divergence.  A lane's
-//     symbols are V-interleaved 16-byte chunks -> 128-bit loads; its values
-//     are 16-byte chunks too.  The 32 widths of a column block live one per
-//     lane and are broadcast with SHFL (replaces constant memory).
-//     Decoding uses a 64-bit window (hi:lo) instead of Alg. 1's sym/rb pair
-//     (reading R5/R6: no read past the row stream, no shift by sym_len).
-//   * BRO-COO: one warp per interval of 32*T entries, a warp-shuffle
-//     segmented scan per step (the "parallel scan primitive") with a
-//     running carry, and a deterministic fix-up kernel for rows crossing
-//     interval boundaries (the "extra kernel invocation for data reduction").
+//   * BRO-ELL (bro_ell_spmv_od): one WARP per 32-row slice, one lane per row
+//     (h = 32), persistent warps.  Widths are warp-uniform, so every
+//     column's bit offset is uniform too: a SHFL scan of the widths gives the
+//     offsets of a 32-column block, the block's symbols are staged in a
+//     per-warp shared window, and each delta is a branch-free funnel-shift
+//     extraction, fused with the x gather and the FMA (the load-decode-compute
+//     cycle of Alg. 1 without its per-column branch).
+//   * BRO-COO (coo_spmv<kBro=true>): one warp per interval of 32*T entries
+//     (P:L140); rows decoded per (step, lane), then a transposed 256-entry
+//     batch per iteration (lane owns 8 consecutive entries), sequential lane
+//     reduction + one warp segmented scan (the "parallel scan primitive",
+//     P:L343) and a deterministic fix-up kernel for rows crossing intervals
+//     (the "extra kernel invocation for data reduction").
+//   * Uncompressed baselines: ell_spmv (thread per row, column-major ELLPACK)
+//     and coo_spmv<kBro=false> (same COO traversal, explicit rows).
 //   * Streamed arrays (symbols, values, COO col/row) are read with
-//     ld.global.nc.L1::no_allocate; x is gathered through the read-only path.
+//     ld.global.nc.L1::no_allocate 16-byte loads; x is gathered through the
+//     read-only path.
 #pragma once
 #include <cstdint>
 #include <cuda_runtime.h>
@@ -158,37 +162,10 @@ struct LaneStream {
     }
     return v;
   }
-  // park / resume the lane's state in shared memory (12 words per lane,
-  // stride 32) so it does not occupy registers between column blocks
-  __device__ __forceinline__ void save(uint32_t* st, int lane) const {
-    st[0 * 32 + lane] = (uint32_t)q; st[1 * 32 + lane] = (uint32_t)avail;
-    st[2 * 32 + lane] = hi; st[3 * 32 + lane] = lo;
-#pragma unroll
-    for (int k = 0; k < 8; ++k) st[(4 + k) * 32 + lane] = buf[k];
-  }
-  __device__ __forceinline__ void restore(const uint32_t* b, int S_, const uint32_t* st, int lane) {
-    base = b; S = S_;
-    q = (int)st[0 * 32 + lane]; avail = (int)st[1 * 32 + lane];
-    hi = st[2 * 32 + lane]; lo = st[3 * 32 + lane];
-#pragma unroll
-    for (int k = 0; k < 8; ++k) buf[k] = st[(4 + k) * 32 + lane];
-  }
 };
 
-// ------------------------------------------------------------------ BRO-ELL
-// y[32t + lane] = sum_j vals(slot) * x[col_j], Alg. 1.
-//
-// Persistent warps walk slices t = warp_id, warp_id + n_warps, ...; the next
-// slice's metadata is prefetched while the current one runs.  Each slice is
-// processed in blocks of up to 32 columns:
-//   phase 1 (decode): the 32 widths of the block are loaded one per lane and
-//     broadcast by SHFL; every lane pulls its deltas through the 64-bit
-//     window, accumulates the column (col += delta) and writes it to a
-//     per-warp shared-memory column buffer (-1 for padding, delta == 0);
-//   phase 2 (multiply): groups of 8 columns, all value chunks (16-byte loads)
-//     and all x gathers of a group issued before the FMAs (8 gathers + 4/2
-//     vector loads in flight per lane), slot-order FMA accumulation.
-// Registers stay near the plain-ELL kernel's, so occupancy stays high.
+// Values of 8 consecutive slice columns j .. j+7 of this lane (16-byte
+// chunks where the chunk is full, scalar loads in the tail chunk, 0 past l).
 template <typename T, int G>
 __device__ __forceinline__ void load_group_vals(T* v, const T* vs, int j, int l, int lfull, int lane) {
   constexpr int VV = Chunk<T>::N;
@@ -206,67 +183,6 @@ __device__ __forceinline__ void load_group_vals(T* v, const T* vs, int j, int l,
       for (int k = 0; k < VV; ++k)
         v[u * VV + k] = (jj + k < l) ? ld_stream(vs + 32 * lfull + lane * tw + (jj + k - lfull)) : T(0);
     }
-  }
-}
-
-template <typename T, int V, int kWarps, int kMinBlocks, int G>
-__global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
-bro_ell_spmv(int64_t m, int64_t s, const uint32_t* __restrict__ words,
-             const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
-             const uint64_t* __restrict__ symptr, const T* __restrict__ vals,
-             const T* __restrict__ x, T* __restrict__ y) {
-  constexpr int VV = Chunk<T>::N;
-  __shared__ int32_t colbuf[kWarps][32 * 32];
-  __shared__ uint32_t stbuf[kWarps][12 * 32];
-  const int lane = threadIdx.x & 31;
-  const int w = threadIdx.x >> 5;
-  int32_t* cb = colbuf[w];
-  uint32_t* st = stbuf[w];
-  const int64_t stride = int64_t(gridDim.x) * kWarps;
-  for (int64_t t = int64_t(blockIdx.x) * kWarps + w; t < s; t += stride) {
-    const uint64_t c0 = __ldg(colptr + t);
-    const int l = int(__ldg(colptr + t + 1) - c0);
-    const uint64_t q0 = __ldg(symptr + t);
-    const int S = int(__ldg(symptr + t + 1) - q0);
-    const uint32_t* wb = words + 32 * q0;
-    const T* vs = vals + 32 * c0;
-    const uint8_t* ba = bit_alloc + c0;
-    const int lfull = (l / VV) * VV;
-    T sum = T(0);
-    int col = -1;
-    for (int jb = 0; jb < l; jb += 32) {
-      const int nb = min(32, l - jb);
-      {  // phase 1: decode columns [jb, jb + nb) into cb
-        const uint32_t breg = lane < nb ? uint32_t(__ldg(ba + jb + lane)) : 0u;
-        LaneStream<V> ls;
-        if (jb == 0) ls.init(wb, S, lane);
-        else ls.restore(wb, S, st, lane);
-#pragma unroll 4
-        for (int k = 0; k < nb; ++k) {
-          const int b = (int)__shfl_sync(0xffffffffu, breg, k);
-          const uint32_t d = ls.get(b, lane);
-          col += int(d);
-          cb[k * 32 + lane] = d ? col : -1;
-        }
-        if (jb + 32 < l) ls.save(st, lane);
-      }
-      __syncwarp();
-      for (int g = 0; g < nb; g += G) {  // phase 2
-        T v[G];
-        load_group_vals<T, G>(v, vs, jb + g, l, lfull, lane);
-        int cc[G];
-#pragma unroll
-        for (int k = 0; k < G; ++k) cc[k] = (g + k < nb) ? cb[(g + k) * 32 + lane] : -1;
-        T xv[G];
-#pragma unroll
-        for (int k = 0; k < G; ++k) xv[k] = cc[k] >= 0 ? ldg_x(x + cc[k]) : T(0);
-#pragma unroll
-        for (int k = 0; k < G; ++k) sum = fma(v[k], xv[k], sum);
-      }
-      __syncwarp();
-    }
-    const int64_t row = 32 * t + lane;
-    if (row < m) y[row] = sum;
   }
 }
 
@@ -424,230 +340,6 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
       obase += tot;
     }
     const int64_t row = 32 * t + lane;
-    if (row < m) y[row] = sum;
-  }
-}
-
-// ------------------------------------------------------------------ BRO-ELL, TMA pipeline
-// Warp-specialised persistent kernel.  Block b owns slices t_k = b + k*gridDim.x.
-// Producer warp: loads the metadata of 32 upcoming slices at once (one slice
-// per lane), then for each slice waits for a free ring stage and issues three
-// bulk async copies (cp.async.bulk, TMA engine) — the slice's values
-// (32*l*sizeof(T) bytes), its multiplexed symbols (128*S bytes) and its
-// widths (16-byte aligned window of bit_alloc) — all completing on the
-// stage's mbarrier.  Consumer warps (one slice each, round robin) wait on the
-// stage, decode the symbols from shared memory, gather x through the
-// read-only path, multiply with the staged values and release the stage.
-// HBM latency is hidden by the ring depth instead of by registers.
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count));
-}
-__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(bar)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  asm volatile(
-      "{\n .reg .pred p;\n"
-      "WAIT_%=:\n"
-      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      " @!p bra WAIT_%=;\n}\n" :: "r"(smem_u32(bar)), "r"(parity) : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar,
-                                         uint64_t policy) {
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
-      :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(policy) : "memory");
-}
-__device__ __forceinline__ uint64_t policy_evict_first() {
-  uint64_t p;
-  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-  return p;
-}
-
-// One lane's symbols read from shared memory (V-interleaved, 16-byte chunks
-// read with one LDS.128 per 4 symbols), MSB first through a 64-bit window.
-template <int V>
-struct SmemLaneStream {
-  const uint32_t* base;
-  int S, q, avail;
-  uint32_t hi, lo;
-  uint32_t buf[4];
-
-  __device__ __forceinline__ void fetch4(int lane) {
-    if constexpr (V == 4) {
-      const int F = S >> 2;
-      const int c = q >> 2;
-      if (c < F) {
-        const uint4 v = *reinterpret_cast<const uint4*>(base + 128 * c + 4 * lane);
-        buf[0] = v.x; buf[1] = v.y; buf[2] = v.z; buf[3] = v.w;
-      } else {
-        const int Vp = S - 4 * F;
-#pragma unroll
-        for (int k = 0; k < 4; ++k) buf[k] = k < Vp ? base[128 * F + Vp * lane + k] : 0u;
-      }
-    } else {
-#pragma unroll
-      for (int k = 0; k < 4; ++k) buf[k] = (q + k < S) ? base[place(lane, q + k, S, V)] : 0u;
-    }
-  }
-  __device__ __forceinline__ uint32_t pop(int lane) {
-    if ((q & 3) == 0) fetch4(lane);
-    const uint32_t r = buf[0];
-    buf[0] = buf[1]; buf[1] = buf[2]; buf[2] = buf[3];
-    ++q;
-    return r;
-  }
-  __device__ __forceinline__ void init(const uint32_t* b, int S_, int lane) {
-    base = b; S = S_; q = 0; hi = 0; lo = 0; avail = 0;
-    if (S > 0) { hi = pop(lane); avail = 32; }
-  }
-  __device__ __forceinline__ uint32_t get(int b, int lane) {  // 1 <= b <= 32
-    const uint32_t v = hi >> (32 - b);
-    hi = __funnelshift_lc(lo, hi, b);
-    lo = shl_clamp(lo, b);
-    avail -= b;
-    if (avail < 32 && q < S) {
-      const uint32_t w = pop(lane);
-      hi |= w >> avail;
-      lo = shl_clamp(w, 32 - avail);
-      avail += 32;
-    }
-    return v;
-  }
-};
-
-struct StageHdr {
-  int l, S, ba_off, pad;
-};
-
-// Stage ownership: item k (the block's k-th slice) goes to consumer
-// w = k % ncons, its j = k / ncons -th item, in the consumer's private stage
-// w * spc + j % spc, phase (j / spc) & 1.  A consumer therefore never waits
-// on a stage more than one phase ahead (mbarrier parity cannot alias), and
-// the producer, which runs in item order, never either.
-template <typename T, int V, int kCons, int kMinBlocks>
-__global__ void __launch_bounds__((kCons + 1) * 32, kMinBlocks)
-bro_ell_spmv_tma(int64_t m, int64_t s, const uint32_t* __restrict__ words,
-                 const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
-                 const uint64_t* __restrict__ symptr, const T* __restrict__ vals,
-                 const T* __restrict__ x, T* __restrict__ y, int ncons, int spc, int stage_bytes) {
-  const int nstages = ncons * spc;
-  constexpr int VV = Chunk<T>::N;
-  constexpr int G = 8;
-  extern __shared__ __align__(128) uint8_t smem[];
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem);
-  uint64_t* empty = full + nstages;
-  StageHdr* hdr = reinterpret_cast<StageHdr*>(empty + nstages);
-  uint8_t* ring = smem + ((nstages * (16 + sizeof(StageHdr)) + 127) / 128) * 128;
-  const int lane = threadIdx.x & 31;
-  const int w = threadIdx.x >> 5;
-  const int64_t G0 = gridDim.x;
-  const int64_t nk = (s > blockIdx.x) ? (s - blockIdx.x + G0 - 1) / G0 : 0;
-  if (threadIdx.x == 0) {
-    for (int i = 0; i < nstages; ++i) {
-      mbar_init(full + i, 1);
-      mbar_init(empty + i, 1);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  if (w == kCons) {
-    // ------------------------------------------------ producer warp
-    const uint64_t pol = policy_evict_first();
-    for (int64_t k0 = 0; k0 < nk; k0 += 32) {
-      const int64_t kk = k0 + lane;
-      uint64_t c0 = 0, c1 = 0, q0 = 0, q1 = 0;
-      if (kk < nk) {
-        const int64_t t = blockIdx.x + kk * G0;
-        c0 = __ldg(colptr + t); c1 = __ldg(colptr + t + 1);
-        q0 = __ldg(symptr + t); q1 = __ldg(symptr + t + 1);
-      }
-      const int nb = (int)(nk - k0 < 32 ? nk - k0 : 32);
-      for (int i = 0; i < nb; ++i) {
-        const uint64_t a0 = __shfl_sync(0xffffffffu, c0, i), a1 = __shfl_sync(0xffffffffu, c1, i);
-        const uint64_t b0 = __shfl_sync(0xffffffffu, q0, i), b1 = __shfl_sync(0xffffffffu, q1, i);
-        const int64_t k = k0 + i;
-        const int64_t jj = k / ncons;
-        const int st = int(k - jj * ncons) * spc + int(jj % spc);
-        const uint32_t ph = uint32_t((jj / spc) & 1);
-        if (lane == 0) {
-          mbar_wait(empty + st, ph ^ 1u);
-          const int l = int(a1 - a0), S = int(b1 - b0);
-          const uint32_t vbytes = uint32_t(32 * l * sizeof(T));
-          const uint32_t wbytes = uint32_t(128 * S);
-          const uint64_t ba_lo = a0 & ~uint64_t(15);
-          const uint32_t bbytes = uint32_t(((a1 + 15) & ~uint64_t(15)) - ba_lo);
-          hdr[st] = StageHdr{l, S, int(a0 - ba_lo), 0};
-          uint8_t* dst = ring + size_t(st) * stage_bytes;
-          mbar_arrive_expect_tx(full + st, vbytes + wbytes + bbytes);
-          if (vbytes) bulk_g2s(dst, vals + 32 * a0, vbytes, full + st, pol);
-          if (wbytes) bulk_g2s(dst + vbytes, words + 32 * b0, wbytes, full + st, pol);
-          if (bbytes) bulk_g2s(dst + vbytes + wbytes, bit_alloc + ba_lo, bbytes, full + st, pol);
-        }
-        __syncwarp();
-      }
-    }
-    return;
-  }
-  // -------------------------------------------------- consumer warps
-  if (w >= ncons) return;
-  int64_t jj = 0;
-  for (int64_t k = w; k < nk; k += ncons, ++jj) {
-    const int st = w * spc + int(jj % spc);
-    const uint32_t ph = uint32_t((jj / spc) & 1);
-    mbar_wait(full + st, ph);
-    const StageHdr h = hdr[st];
-    const int l = h.l, S = h.S;
-    const uint8_t* sbase = ring + size_t(st) * stage_bytes;
-    const T* sv = reinterpret_cast<const T*>(sbase);
-    const uint32_t* sw = reinterpret_cast<const uint32_t*>(sbase + 32 * l * sizeof(T));
-    const uint8_t* sb = sbase + 32 * l * sizeof(T) + 128 * S + h.ba_off;
-    const int lfull = (l / VV) * VV;
-    const int tw = l - lfull;
-    SmemLaneStream<V> ls;
-    ls.init(sw, S, lane);
-    T sum = T(0);
-    int col = -1;
-    for (int j0 = 0; j0 < l; j0 += G) {
-      int cc[G];
-#pragma unroll
-      for (int k2 = 0; k2 < G; ++k2) {
-        const int j = j0 + k2;
-        const int b = j < l ? int(sb[j]) : 0;
-        const uint32_t d = b ? ls.get(b, lane) : 0u;
-        col += int(d);
-        cc[k2] = d ? col : -1;
-      }
-      T xv[G];
-#pragma unroll
-      for (int k2 = 0; k2 < G; ++k2) xv[k2] = cc[k2] >= 0 ? ldg_x(x + cc[k2]) : T(0);
-      T v[G];
-#pragma unroll
-      for (int u = 0; u < G / VV; ++u) {
-        const int jj = j0 + u * VV;
-        if (jj + VV <= lfull) {
-          if constexpr (VV == 2) {
-            const double2 c2 = *reinterpret_cast<const double2*>(sv + 32 * jj + lane * VV);
-            v[u * VV] = c2.x; v[u * VV + 1] = c2.y;
-          } else {
-            const float4 c4 = *reinterpret_cast<const float4*>(sv + 32 * jj + lane * VV);
-            v[u * VV] = c4.x; v[u * VV + 1] = c4.y; v[u * VV + 2] = c4.z; v[u * VV + 3] = c4.w;
-          }
-        } else {
-#pragma unroll
-          for (int q2 = 0; q2 < VV; ++q2)
-            v[u * VV + q2] = (jj + q2 < l) ? sv[32 * lfull + lane * tw + (jj + q2 - lfull)] : T(0);
-        }
-      }
-#pragma unroll
-      for (int k2 = 0; k2 < G; ++k2) sum = fma(v[k2], xv[k2], sum);
-    }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(empty + st);
-    const int64_t row = 32 * (blockIdx.x + k * G0) + lane;
     if (row < m) y[row] = sum;
   }
 }
