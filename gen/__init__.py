@@ -18,6 +18,7 @@ from .matrices import (  # noqa: F401
     webbase_like,
     random_block,
     random_csr,
+    dense_band,
     permute_rows,
     row_block,
 )

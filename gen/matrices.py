@@ -339,3 +339,13 @@ def make_config(i: int, dtype=np.float64) -> Csr:
         raise ValueError(f"no config {i}")
     A.name = f"C{i}:" + A.name
     return A.astype(dtype) if dtype != np.float64 else A
+
+
+def dense_band(m: int, k: int = 32, seed: int = 7) -> Csr:
+    """Dense m x k matrix (every row holds columns 0..k-1), vals U[-1,1):
+    the Fig. 3 workload ('a dense matrix was used ... to avoid
+    variations in performance due to cache effects when reading x')."""
+    rng = np.random.default_rng(seed)
+    row_ptr = np.arange(m + 1, dtype=np.int64) * k
+    col = np.tile(np.arange(k, dtype=np.int32), m)
+    return Csr(m, k, row_ptr, col, rng.uniform(-1.0, 1.0, m * k), f"dense_{m}x{k}")

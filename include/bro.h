@@ -90,7 +90,10 @@ typedef struct {
   int32_t coo_T;     /* BRO-COO steps per interval (interval = 32*T entries). Must be 32. */
   int64_t hyb_K;     /* HYB dividing column; -1 = the "less than a third" rule. */
   int32_t codec;     /* 1 = BRO compressed formats; 0 = uncompressed ELL/COO/HYB baseline. */
-  int32_t reserved;  /* must be 0 */
+  int32_t min_bits;  /* 0 = natural widths; k in [1, 31] forces every BRO-ELL width
+                        b_j = max(Gamma, k) — the simulated compression ratios of the
+                        Fig. 3 experiment ("the number of bits allocated to each
+                        index value ... was varied"). */
 } bro_opts_t;
 
 typedef struct {

@@ -85,16 +85,19 @@ class SliceCode:
     symbols: list          # h lists of S ints
 
 
-def encode_slice(rows_cols, h: int, sym_len: int) -> SliceCode:
+def encode_slice(rows_cols, h: int, sym_len: int, min_bits: int = 0) -> SliceCode:
     """Steps 1-6 for one slice.  rows_cols: h column lists (0-based, sorted
-    strictly increasing); rows past the matrix end are empty lists."""
+    strictly increasing); rows past the matrix end are empty lists.
+    min_bits > 0 forces every width up to min_bits: the simulated compression
+    ratios of the Fig. 3 experiment ("the number of bits allocated to each
+    index value of a non-zero entry was varied")."""
     assert len(rows_cols) == h
     l = max((len(c) for c in rows_cols), default=0)                # step 3
     deltas = []
     for cols in rows_cols:                                          # step 1
         d = row_deltas(cols)
         deltas.append(d + [0] * (l - len(d)))                       # 0 = invalid
-    widths = [max(gamma(deltas[r][j]) for r in range(h)) for j in range(l)]  # step 4
+    widths = [max([min_bits] + [gamma(deltas[r][j]) for r in range(h)]) for j in range(l)]  # step 4
     L = sum(widths)
     S = -(-L // sym_len)                                            # step 5
     b_p = sym_len * S - L
@@ -146,7 +149,7 @@ def _slice_rows(row_ptr, col, t, h, m):
     return out
 
 
-def slice_shapes(row_ptr, col, m, h=32, sym_len=32):
+def slice_shapes(row_ptr, col, m, h=32, sym_len=32, min_bits=0):
     """(num_col, S, widths-flat) for ALL slices, vectorised over the matrix.
     Same rules as encode_slice (steps 1, 3-5); a separate code path used to
     place sampled slices of full-size matrices (pinned against encode_slice
@@ -172,6 +175,7 @@ def slice_shapes(row_ptr, col, m, h=32, sym_len=32):
     g = gamma_np(delta)
     widths = np.zeros(int(colptr[-1]), dtype=np.int64)
     np.maximum.at(widths, colptr[rows // h] + pos, g)
+    widths = np.maximum(widths, min_bits)
     cw = np.zeros(widths.size + 1, dtype=np.int64)
     np.cumsum(widths, out=cw[1:])
     L = cw[colptr[1:]] - cw[colptr[:-1]]          # sum_j b_j per slice (exact ints)
@@ -179,7 +183,8 @@ def slice_shapes(row_ptr, col, m, h=32, sym_len=32):
     return num_col, S, widths
 
 
-def encode(row_ptr, col, vals, m, n, h=32, sym_len=32, V=4, Vv=None, slices=None) -> BroEll:
+def encode(row_ptr, col, vals, m, n, h=32, sym_len=32, V=4, Vv=None, slices=None,
+           min_bits=0) -> BroEll:
     """BRO-ELL of the CSR matrix.  `slices=None` encodes every slice; a list
     encodes only those slices (placed at their global offsets, other words
     left 0) so full-size matrices can be checked on samples."""
@@ -188,7 +193,7 @@ def encode(row_ptr, col, vals, m, n, h=32, sym_len=32, V=4, Vv=None, slices=None
     if Vv is None:
         Vv = value_chunk(vals.dtype.itemsize)
     s = -(-m // h)
-    num_col, S, widths_flat = slice_shapes(row_ptr, col, m, h, sym_len)
+    num_col, S, widths_flat = slice_shapes(row_ptr, col, m, h, sym_len, min_bits)
     colptr = np.zeros(s + 1, dtype=np.uint64)
     np.cumsum(num_col, out=colptr[1:])
     symptr = np.zeros(s + 1, dtype=np.uint64)
@@ -200,7 +205,7 @@ def encode(row_ptr, col, vals, m, n, h=32, sym_len=32, V=4, Vv=None, slices=None
     todo = range(s) if slices is None else slices
     codes = {}
     for t in todo:
-        sc = encode_slice(_slice_rows(row_ptr, col, t, h, m), h, sym_len)
+        sc = encode_slice(_slice_rows(row_ptr, col, t, h, m), h, sym_len, min_bits)
         assert sc.l == num_col[t] and sc.S == S[t]
         bit_alloc[int(colptr[t]):int(colptr[t + 1])] = sc.widths
         wb = h * int(symptr[t])

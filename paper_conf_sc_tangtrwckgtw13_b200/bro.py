@@ -33,7 +33,7 @@ FORMATS = {0: "ELL", 1: "COO", 2: "HYB"}
 class bro_opts_t(C.Structure):
     _fields_ = [("slice_h", C.c_int32), ("sym_bits", C.c_int32), ("vec_words", C.c_int32),
                 ("coo_T", C.c_int32), ("hyb_K", C.c_int64), ("codec", C.c_int32),
-                ("reserved", C.c_int32)]
+                ("min_bits", C.c_int32)]
 
 
 class bro_info_t(C.Structure):
@@ -225,11 +225,11 @@ class BroMatrix:
     """Owns one libbro handle.  `fmt` in {"ell", "hyb", "coo"}; codec=1 gives
     BRO-ELL / BRO-HYB / BRO-COO, codec=0 the uncompressed baseline."""
 
-    def __init__(self, A, fmt="ell", codec=1, device=0, dtype=None, vec_words=4, hyb_K=-1):
+    def __init__(self, A, fmt="ell", codec=1, device=0, dtype=None, vec_words=4, hyb_K=-1, min_bits=0):
         vals = A.vals if dtype is None else A.vals.astype(dtype)
         self.dtype = np.dtype(vals.dtype)
         self.m, self.n, self.fmt, self.device = A.m, A.n, fmt, device
-        opts = bro_opts_default(codec=codec, vec_words=vec_words, hyb_K=hyb_K)
+        opts = bro_opts_default(codec=codec, vec_words=vec_words, hyb_K=hyb_K, min_bits=min_bits)
         if fmt == "ell":
             self.h = bro_create_ell(device, A.m, A.n, A.row_ptr, A.col, vals, opts)
         elif fmt == "hyb":

@@ -111,7 +111,7 @@ bro_status_t check_opts(const bro_opts_t& o) {
   if (o.coo_T != 32) return fail(BRO_ERR_UNSUPPORTED, "coo_T must be 32");
   if (o.codec != 0 && o.codec != 1) return fail(BRO_ERR_ARG, "codec must be 0 or 1");
   if (o.hyb_K < -1) return fail(BRO_ERR_ARG, "hyb_K must be >= -1");
-  if (o.reserved != 0) return fail(BRO_ERR_ARG, "reserved must be 0");
+  if (o.min_bits < 0 || o.min_bits > 31) return fail(BRO_ERR_ARG, "min_bits must be in [0, 31]");
   return BRO_OK;
 }
 
@@ -189,7 +189,7 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
       for (int64_t i = 0; i < m; ++i) ne += rv.len(i);
       A->nnz_ell = ne;
       if (o.codec) {
-        bro::encode_bro_ell(rv, o.vec_words, 16 / A->vsize, A->ell);
+        bro::encode_bro_ell(rv, o.vec_words, 16 / A->vsize, o.min_bits, A->ell);
         A->s = A->ell.s;
         A->ell_words = (int64_t)A->ell.words.size();
         A->ell_slots = (int64_t)(A->ell.vals.size() / A->vsize);
@@ -412,7 +412,7 @@ void bro_opts_default(bro_opts_t* o) {
   o->coo_T = 32;
   o->hyb_K = -1;
   o->codec = 1;
-  o->reserved = 0;
+  o->min_bits = 0;
 }
 
 bro_status_t bro_create_ell(int device, bro_dtype_t dtype, int64_t m, int64_t n, const int64_t* row_ptr,

@@ -139,7 +139,7 @@ struct SymbolWriter {
   }
 };
 
-void encode_bro_ell(const RowsView& A, int V, int VV, EllCode& out) {
+void encode_bro_ell(const RowsView& A, int V, int VV, int min_bits, EllCode& out) {
   const int64_t m = A.m;
   const int64_t s = (m + kH - 1) / kH;
   out.s = s;
@@ -171,7 +171,10 @@ void encode_bro_ell(const RowsView& A, int V, int VV, EllCode& out) {
         }
       }
       uint64_t L = 0;
-      for (uint64_t j = 0; j < ncol[t]; ++j) L += ba[j];
+      for (uint64_t j = 0; j < ncol[t]; ++j) {
+        if (ba[j] < min_bits) ba[j] = (uint8_t)min_bits;  // forced widths (Fig. 3)
+        L += ba[j];
+      }
       nsym[t] = (L + kSym - 1) / kSym;
     }
   });

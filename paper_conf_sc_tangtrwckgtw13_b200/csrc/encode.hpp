@@ -78,7 +78,7 @@ std::string check_coo(int64_t m, int64_t n, int64_t nnz, const int32_t* row, con
 
 int64_t hyb_K(int64_t m, const int64_t* row_ptr);
 
-void encode_bro_ell(const RowsView& A, int V, int value_chunk, EllCode& out);
+void encode_bro_ell(const RowsView& A, int V, int value_chunk, int min_bits, EllCode& out);
 void build_plain_ell(const RowsView& A, int64_t K, PlainEll& out);
 // rows: int32 rows of the COO entries (sorted); T steps per interval.
 void encode_bro_coo(int64_t nnz, const int32_t* row, const int32_t* col, const uint8_t* vals,

@@ -255,3 +255,33 @@ def test_bar_algorithm2_matches_oracle(lib, seed):
         perm = lib.bro_reorder_bar(M.m, M.n, M.row_ptr, M.col, method=1)
         ref = bar.algorithm2(M.row_ptr, M.col, M.m, h=32)
         assert np.array_equal(perm, ref)
+
+
+@pytest.mark.parametrize("min_bits", [3, 9, 31])
+def test_forced_widths_bytes_match_oracle(lib, min_bits):
+    """min_bits (Fig. 3 forced widths): C++ bytes == oracle bytes."""
+    A = random_csr(120, 700, 4, max_len=40, empty_frac=0.1)
+    o = lib.bro_opts_default(min_bits=min_bits)
+    h = lib.bro_create_ell(HOST, A.m, A.n, A.row_ptr, A.col, A.vals, o)
+    try:
+        parts = {p: lib.bro_export_encoded(h, p, np.float64) for p in
+                 ("ell_words", "ell_bit_alloc", "ell_colptr", "ell_symptr", "ell_vals")}
+    finally:
+        lib.bro_destroy(h)
+    E = bro_ell.encode(A.row_ptr, A.col, A.vals, A.m, A.n, min_bits=min_bits)
+    _assert_ell_equal(parts, E)
+    assert bro_ell.decode(E) == [A.col[A.row_ptr[i]:A.row_ptr[i + 1]].tolist() for i in range(A.m)]
+
+
+def test_dense_band_eta_closed_form(lib):
+    """Dense 32-column rows with every width forced to b: each row stream is
+    exactly b symbols of 32 bits, so eta = 1 - b/32."""
+    from gen import dense_band
+    A = dense_band(320, 32)
+    for b in (1, 4, 16, 31):
+        h = lib.bro_create_ell(HOST, A.m, A.n, A.row_ptr, A.col, A.vals, lib.bro_opts_default(min_bits=b))
+        try:
+            info = lib.bro_get_info(h)
+        finally:
+            lib.bro_destroy(h)
+        assert info["eta_stream"] == pytest.approx(1 - b / 32)
