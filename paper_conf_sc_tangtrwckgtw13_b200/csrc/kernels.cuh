@@ -195,6 +195,11 @@ __device__ __forceinline__ void load_group_vals(T* v, const T* vs, int j, int l,
 // column's delta is a branch-free extraction
 //     delta = funnelshift(w[q+1], w[q], o mod 32) >> (32 - b),   q = o / 32
 // fused with the x gather and the FMA (8 columns in flight per group).
+// Bulk (TMA engine) prefetch of [p, p + bytes) into L2; p and bytes multiples of 16.
+__device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(p), "r"(bytes) : "memory");
+}
+
 __device__ __forceinline__ uint32_t shr_clamp(uint32_t v, uint32_t s) {
   uint32_t r;
   asm("shr.b32 %0, %1, %2;" : "=r"(r) : "r"(v), "r"(s));
@@ -239,7 +244,7 @@ __device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __r
   win[nrows * 32 + lane] = 0u;
 }
 
-template <typename T, int V, int kWarps, int kMinBlocks>
+template <typename T, int V, int kWarps, int kMinBlocks, bool kPrefetch>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
                 const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
@@ -269,6 +274,14 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
       __syncwarp();
     }
     const Meta mt = metas[w][k32];
+    if (kPrefetch && lane == 0 && k32 < 31 && t + stride < s) {
+      // TMA prefetch of the next slice's values and symbols into L2: the
+      // next iteration's loads then hit L2 instead of DRAM (no registers or
+      // shared memory held while they are in flight)
+      const Meta mn = metas[w][k32 + 1];
+      if (mn.l) prefetch_l2(vals + 32 * mn.c0, uint32_t(32 * mn.l * sizeof(T)));
+      if (mn.S) prefetch_l2(words + 32 * mn.q0, uint32_t(128 * mn.S));
+    }
     const uint64_t c0 = mt.c0;
     const int l = mt.l;
     const int S = mt.S;
@@ -455,6 +468,15 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, const uint32_t* __restrict__ word
   if (i >= nI) return;
   int32_t* rb = rowbuf[w];
   const int64_t e0 = i * 32 * T_steps;
+  if (lane == 0) {  // L2 prefetch (TMA engine) of the batches after the first one
+    const int64_t p0 = e0 + 32 * TB;
+    const int64_t p1 = min(e0 + 32 * int64_t(T_steps), nnz) & ~int64_t(3);
+    if (p1 > p0) {
+      prefetch_l2(col + p0, uint32_t((p1 - p0) * 4));
+      prefetch_l2(vals + p0, uint32_t((p1 - p0) * sizeof(T)));
+      if constexpr (!kBro) prefetch_l2(rows + p0, uint32_t((p1 - p0) * 4));
+    }
+  }
   const int first = (int)base_row[i];
   int row = first;
   int b = 0;
