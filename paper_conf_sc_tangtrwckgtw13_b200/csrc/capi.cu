@@ -291,10 +291,10 @@ bro_status_t common_checks(bro_dtype_t dtype, const bro_opts_t* opts, bro_opts_t
 
 // Persistent grid: as many resident blocks as the SMs hold (queried once per
 // instantiation), capped by the number of slices.
-template <typename T, int V, int kWarps, int kMinBlocks, bool kPrefetch>
+template <typename T, int V, int kWarps, int kMinBlocks>
 void launch_bro_ell_od(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   using namespace bro::dev;
-  auto kern = bro_ell_spmv_od<T, V, kWarps, kMinBlocks, kPrefetch>;
+  auto kern = bro_ell_spmv_od<T, V, kWarps, kMinBlocks>;
   static int resident = 0;
   if (resident == 0) {
     int per_sm = 0, sms = 0, dev = 0;
@@ -312,20 +312,9 @@ void launch_bro_ell_od(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
 constexpr int kEllWarps = 8;      // slices per block
 constexpr int kEllMinBlocks = 4;  // 32 resident warps per SM (64 registers)
 
-// A/B switch for tuning runs only (BRO_ELL_VARIANT=1 disables the L2 prefetch).
-static int ell_variant() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("BRO_ELL_VARIANT");
-    v = e ? atoi(e) : 0;
-  }
-  return v;
-}
-
 template <typename T, int V>
 void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
-  if (ell_variant() == 1) return launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks, false>(A, x, y, st);
-  launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks, true>(A, x, y, st);
+  launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks>(A, x, y, st);
 }
 
 template <typename T>

@@ -186,6 +186,24 @@ __device__ __forceinline__ void load_group_vals(T* v, const T* vs, int j, int l,
   }
 }
 
+// Group values: straight 16-byte loads when the whole group lies in full
+// chunks (the common case), else the tail-aware path.
+template <typename T, int G>
+__device__ __forceinline__ void load_vals(T* v, const T* vs, int j, int l, int lfull, int lane) {
+  constexpr int VV = Chunk<T>::N;
+  if (j + G <= lfull) {
+#pragma unroll
+    for (int u = 0; u < G / VV; ++u) {
+      Chunk<T> c;
+      c.load(vs + 32 * (j + u * VV) + lane * VV);
+#pragma unroll
+      for (int q = 0; q < VV; ++q) v[u * VV + q] = c.v[q];
+    }
+  } else {
+    load_group_vals<T, G>(v, vs, j, l, lfull, lane);
+  }
+}
+
 // ------------------------------------------------------------------ BRO-ELL, offset decode
 // Widths are warp-uniform (one per slice column), so the bit offset
 // of column j inside every row stream is the same for all 32 lanes:
@@ -244,7 +262,7 @@ __device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __r
   win[nrows * 32 + lane] = 0u;
 }
 
-template <typename T, int V, int kWarps, int kMinBlocks, bool kPrefetch>
+template <typename T, int V, int kWarps, int kMinBlocks>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
                 const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
@@ -274,14 +292,6 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
       __syncwarp();
     }
     const Meta mt = metas[w][k32];
-    if (kPrefetch && lane == 0 && k32 < 31 && t + stride < s) {
-      // TMA prefetch of the next slice's values and symbols into L2: the
-      // next iteration's loads then hit L2 instead of DRAM (no registers or
-      // shared memory held while they are in flight)
-      const Meta mn = metas[w][k32 + 1];
-      if (mn.l) prefetch_l2(vals + 32 * mn.c0, uint32_t(32 * mn.l * sizeof(T)));
-      if (mn.S) prefetch_l2(words + 32 * mn.q0, uint32_t(128 * mn.S));
-    }
     const uint64_t c0 = mt.c0;
     const int l = mt.l;
     const int S = mt.S;
@@ -292,6 +302,10 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
     T sum = T(0);
     int col = -1;
     int obase = 0;  // bit offset of the current block inside every row stream
+    T v[G];         // values of the group being multiplied
+    // the first group's values do not depend on decoding: issue them before
+    // the width scan and the symbol staging so both latencies overlap
+    if (l > 0) load_vals<T, G>(v, vs, 0, l, lfull, lane);
     for (int jb = 0; jb < l; jb += 32) {
       const int nb = min(32, l - jb);
       const int b = lane < nb ? int(__ldg(ba + jb + lane)) : 0;
@@ -318,18 +332,7 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
       }
       __syncwarp();
       for (int g = 0; g < nb; g += G) {
-        T v[G];
-        if (jb + g + G <= lfull) {  // all chunks of the group are full 16-byte chunks
-#pragma unroll
-          for (int u = 0; u < G / Chunk<T>::N; ++u) {
-            Chunk<T> c;
-            c.load(vs + 32 * (jb + g + u * Chunk<T>::N) + lane * Chunk<T>::N);
-#pragma unroll
-            for (int q = 0; q < Chunk<T>::N; ++q) v[u * Chunk<T>::N + q] = c.v[q];
-          }
-        } else {
-          load_group_vals<T, G>(v, vs, jb + g, l, lfull, lane);
-        }
+        if (jb + g > 0) load_vals<T, G>(v, vs, jb + g, l, lfull, lane);
         int cidx[G];
         bool ok[G];
 #pragma unroll
@@ -488,9 +491,14 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, const uint32_t* __restrict__ word
   }
   T carry = T(0);   // partial of row crow carried from earlier batches (not yet written)
   int crow = first;
-  auto emit = [&](int r, T v) {  // a complete segment of row r
+  // A complete segment of row r.  Every row other than the interval's first
+  // and last rows is complete in exactly one place of the whole launch, so it
+  // receives exactly one addition: a fire-and-forget RED (atomicAdd with the
+  // result unused) is as deterministic as y[r] += v but does not serialize
+  // the warp on a load -> store chain per segment.
+  auto emit = [&](int r, T v) {
     if (r == first) carry_first[i] = v;
-    else y[r] += v;
+    else atomicAdd(y + r, v);
   };
   for (int t0 = 0; t0 < T_steps; t0 += TB) {
     const int64_t eb = e0 + 32 * t0;            // first entry of the batch
