@@ -302,10 +302,6 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
     T sum = T(0);
     int col = -1;
     int obase = 0;  // bit offset of the current block inside every row stream
-    T v[G];         // values of the group being multiplied
-    // the first group's values do not depend on decoding: issue them before
-    // the width scan and the symbol staging so both latencies overlap
-    if (l > 0) load_vals<T, G>(v, vs, 0, l, lfull, lane);
     for (int jb = 0; jb < l; jb += 32) {
       const int nb = min(32, l - jb);
       const int b = lane < nb ? int(__ldg(ba + jb + lane)) : 0;
@@ -332,7 +328,8 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
       }
       __syncwarp();
       for (int g = 0; g < nb; g += G) {
-        if (jb + g > 0) load_vals<T, G>(v, vs, jb + g, l, lfull, lane);
+        T v[G];
+        load_vals<T, G>(v, vs, jb + g, l, lfull, lane);
         int cidx[G];
         bool ok[G];
 #pragma unroll
