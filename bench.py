@@ -53,6 +53,8 @@ def parse_args():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--flush-l2", action="store_true", help="write a 2xL2 buffer between steps")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="gloo only for functional checks of the N>1 path on one GPU")
     return ap.parse_args()
 
 
@@ -169,6 +171,15 @@ def time_steps(fn, steps, warmup, stream, flush=None):
     return np.array([s.elapsed_time(e) for s, e in ev])
 
 
+def max_over_ranks(vals, dev, backend):
+    """Element-wise max over ranks (device times are compared as the max)."""
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor(vals, dtype=torch.float64, device=dev if backend == "nccl" else "cpu")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return [float(v) for v in t.cpu()]
+
+
 def run_reference(args):
     """--impl reference: the CPU oracle (the only reference this paper-only
     tier has), as it stands, on the host cores; rank 0 only."""
@@ -216,10 +227,16 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus and world > 1:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    # one process per GPU; ranks wrap around only in the gloo functional
+    # check of the N > 1 path on a single-GPU box (never with NCCL)
+    local = local % max(1, torch.cuda.device_count()) if args.dist_backend == "gloo" else local
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
 
     import paper_conf_sc_tangtrwckgtw13_b200 as P
     from paper_conf_sc_tangtrwckgtw13_b200.dist import RowBlockSpmv, choose_partition
@@ -275,9 +292,7 @@ def main():
     base_kern_ms = float(np.mean(time_steps(lambda: base.spmv(x, stream), min(args.steps, 500), 3,
                                             stream, flush)))
     if world > 1:
-        t = torch.tensor([total_ms, base_ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms, base_ms = float(t[0]), float(t[1])
+        total_ms, base_ms = max_over_ranks([total_ms, base_ms], dev, args.dist_backend)
 
     # --- end to end through the C ABI with pinned host buffers (rank 0 / N=1 path)
     e2e = None
@@ -297,9 +312,7 @@ def main():
         torch.cuda.synchronize()
         e2e_ms = t0e.elapsed_time(t1e) / e2e_steps
         if world > 1:
-            t = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            e2e_ms = float(t[0])
+            (e2e_ms,) = max_over_ranks([e2e_ms], dev, args.dist_backend)
         isz = np.dtype(dtype).itemsize
         e2e = {"value": 2.0 * A.nnz / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s",
                "h2d_bytes_per_step": int(A.n * isz), "d2h_bytes_per_step": int(blk.mat.m * isz),
