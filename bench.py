@@ -361,7 +361,7 @@ def main():
             "vec_words": args.vec_words,
             "l2": ("flushed (2x L2 write) before every step" if args.flush_l2 else
                    ("inputs larger than L2" if alg_bytes > 2 * L2_BYTES else "L2-resident (warm)")),
-            "parallelism": f"row-block x{world}" + (f" + {args.dist_backend} allgather of y per step" if world > 1 else ""),
+            "parallelism": f"row-block x{world}" + (" + NCCL allgather of y per step" if world > 1 else ""),
             "eta_stream": info["eta_stream"], "eta_total": info["eta_total"],
         },
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

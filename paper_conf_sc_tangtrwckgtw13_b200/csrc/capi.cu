@@ -21,7 +21,7 @@ bro_status_t fail(bro_status_t s, const std::string& msg) {
   return s;
 }
 
-constexpr int kCooThreads = 128;  // 4 warps: per-warp staging is 9-16 KB of shared memory
+constexpr int kCooThreads = 256;
 constexpr int kPlainThreads = 256;
 
 struct DeviceGuard {
@@ -249,11 +249,6 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
     }
     if (A->has_coo) {
       UP(A->d_coo_base, A->coo.base_row);
-      // the COO kernel stages each interval with 16-byte-rounded bulk copies:
-      // pad the streamed arrays so the last interval's copy stays in bounds
-      A->coo.col.resize(A->coo.col.size() + 4, 0);
-      A->coo.vals.v.resize(A->coo.vals.size() + 16, 0);
-      if (!o.codec) A->coo.row.resize(A->coo.row.size() + 4, 0);
       UP(A->d_coo_col, A->coo.col);
       if (st == BRO_OK) st = dev_upload(A, &A->d_coo_vals, A->coo.vals.data(), A->coo.vals.size());
       if (o.codec) {
@@ -322,25 +317,6 @@ void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks>(A, x, y, st);
 }
 
-// (BRO-)COO: one warp per 1024-entry interval, the interval's arrays staged
-// in dynamic shared memory (CooSmem) by bulk copies.
-template <typename T, int V, bool kBro>
-void launch_coo(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
-  using namespace bro::dev;
-  auto kern = coo_spmv<T, V, kBro, kCooThreads>;
-  constexpr int smem = (kCooThreads / 32) * CooSmem<T, kBro>::kWarp;
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    attr = true;
-  }
-  const int warps = kCooThreads / 32;
-  dim3 grid((unsigned)((A->nI + warps - 1) / warps));
-  kern<<<grid, kCooThreads, smem, st>>>(A->nnz_coo, A->nI, A->opts.coo_T, A->d_coo_words, A->d_coo_base,
-                                        A->d_coo_width, A->d_coo_symptr, A->d_coo_row, A->d_coo_col,
-                                        (const T*)A->d_coo_vals, x, y, (T*)A->d_cf, (T*)A->d_cl, A->d_last_row);
-}
-
 template <typename T>
 bro_status_t launch_spmv(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   using namespace bro::dev;
@@ -361,12 +337,26 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
     cudaMemsetAsync(y, 0, size_t(A->m) * sizeof(T), st);
   }
   if (A->has_coo && A->nI > 0) {
+    const int warps = kCooThreads / 32;
+    dim3 grid((unsigned)((A->nI + warps - 1) / warps));
+    const int T_ = A->opts.coo_T;
     if (A->opts.codec) {
-      if (V == 4) launch_coo<T, 4, true>(A, x, y, st);
-      else if (V == 2) launch_coo<T, 2, true>(A, x, y, st);
-      else launch_coo<T, 1, true>(A, x, y, st);
+      if (V == 4)
+        coo_spmv<T, 4, true, kCooThreads><<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, A->d_coo_words,
+            A->d_coo_base, A->d_coo_width, A->d_coo_symptr, nullptr, A->d_coo_col, (const T*)A->d_coo_vals, x, y,
+            (T*)A->d_cf, (T*)A->d_cl, A->d_last_row);
+      else if (V == 2)
+        coo_spmv<T, 2, true, kCooThreads><<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, A->d_coo_words,
+            A->d_coo_base, A->d_coo_width, A->d_coo_symptr, nullptr, A->d_coo_col, (const T*)A->d_coo_vals, x, y,
+            (T*)A->d_cf, (T*)A->d_cl, A->d_last_row);
+      else
+        coo_spmv<T, 1, true, kCooThreads><<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, A->d_coo_words,
+            A->d_coo_base, A->d_coo_width, A->d_coo_symptr, nullptr, A->d_coo_col, (const T*)A->d_coo_vals, x, y,
+            (T*)A->d_cf, (T*)A->d_cl, A->d_last_row);
     } else {
-      launch_coo<T, 4, false>(A, x, y, st);
+      coo_spmv<T, 4, false, kCooThreads><<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, nullptr,
+          A->d_coo_base, nullptr, nullptr, A->d_coo_row, A->d_coo_col, (const T*)A->d_coo_vals, x, y,
+          (T*)A->d_cf, (T*)A->d_cl, A->d_last_row);
     }
     dim3 g2((unsigned)((A->nI + 255) / 256));
     coo_fixup<T><<<g2, 256, 0, st>>>(A->nI, A->d_coo_base, A->d_last_row, (const T*)A->d_cf,

@@ -218,26 +218,6 @@ __device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
   asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(p), "r"(bytes) : "memory");
 }
 
-// mbarrier + bulk async copy (TMA engine) global -> shared
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count) : "memory");
-  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-}
-__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  asm volatile(
-      "{\n .reg .pred p;\n"
-      "WAIT_%=:\n"
-      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      " @!p bra WAIT_%=;\n}\n" :: "r"(smem_u32(bar)), "r"(parity) : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-               :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
-}
-
 __device__ __forceinline__ uint32_t shr_clamp(uint32_t v, uint32_t s) {
   uint32_t r;
   asm("shr.b32 %0, %1, %2;" : "=r"(r) : "r"(v), "r"(s));
@@ -451,16 +431,26 @@ __global__ void ell_decode(int64_t m, int64_t K, int64_t pitch, const int32_t* _
 // than the interval's first row are added into y directly (each such row
 // lives in exactly one interval); the first and last rows' partials go to
 // carry arrays for the deterministic fix-up kernel.
-// Per-warp shared memory of coo_spmv (interval = 1024 entries): values,
-// columns, rows (plain COO only), the decoded-row buffer (BRO only), mbarrier.
-template <typename T, bool kBro>
-struct CooSmem {
-  static constexpr int kCol = 1024 * int(sizeof(T));
-  static constexpr int kRow = kCol + 4096;
-  static constexpr int kBuf = kRow + (kBro ? 0 : 4096);
-  static constexpr int kBar = kBuf + (kBro ? 1024 : 0);
-  static constexpr int kWarp = kBar + 16;
+template <typename T>
+struct Vec8 {  // 8 consecutive values of one lane, loaded as 16-byte chunks
+  T v[8];
+  __device__ __forceinline__ void load(const T* p) {
+#pragma unroll
+    for (int u = 0; u < 8 / Chunk<T>::N; ++u) {
+      Chunk<T> c;
+      c.load(p + u * Chunk<T>::N);
+#pragma unroll
+      for (int q = 0; q < Chunk<T>::N; ++q) v[u * Chunk<T>::N + q] = c.v[q];
+    }
+  }
 };
+
+__device__ __forceinline__ void load8_s32(int* d, const int32_t* p) {
+  const uint4 a = ld_stream_u4(reinterpret_cast<const uint32_t*>(p));
+  const uint4 b = ld_stream_u4(reinterpret_cast<const uint32_t*>(p) + 4);
+  d[0] = int(a.x); d[1] = int(a.y); d[2] = int(a.z); d[3] = int(a.w);
+  d[4] = int(b.x); d[5] = int(b.y); d[6] = int(b.z); d[7] = int(b.w);
+}
 
 template <typename T, int V, bool kBro, int kThreads>
 __global__ void __launch_bounds__(kThreads)
@@ -471,31 +461,22 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, const uint32_t* __restrict__ word
          T* __restrict__ y, T* __restrict__ carry_first, T* __restrict__ carry_last,
          int32_t* __restrict__ last_row) {
   constexpr int TB = 8;
-  extern __shared__ __align__(16) uint8_t dsm[];
+  __shared__ __align__(16) int32_t rowbuf[kThreads / 32][TB * 32];
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
   const int64_t i = int64_t(blockIdx.x) * (kThreads / 32) + w;
   if (i >= nI) return;
-  // per-warp staging area: the interval's values, columns (and rows for plain COO)
-  uint8_t* ws = dsm + size_t(w) * CooSmem<T, kBro>::kWarp;
-  T* sv = reinterpret_cast<T*>(ws);
-  int32_t* sc = reinterpret_cast<int32_t*>(ws + CooSmem<T, kBro>::kCol);
-  int32_t* sr = reinterpret_cast<int32_t*>(ws + CooSmem<T, kBro>::kRow);
-  int32_t* rb = reinterpret_cast<int32_t*>(ws + CooSmem<T, kBro>::kBuf);
-  uint64_t* bar = reinterpret_cast<uint64_t*>(ws + CooSmem<T, kBro>::kBar);
+  int32_t* rb = rowbuf[w];
   const int64_t e0 = i * 32 * T_steps;
-  const int64_t rest = nnz - e0;
-  const int ne = int(rest < 32 * int64_t(T_steps) ? rest : 32 * int64_t(T_steps));  // entries here
-  if (lane == 0) {  // one bulk copy per array (TMA engine); sizes rounded up to 16 bytes
-    mbar_init(bar, 1);
-    const uint32_t vb = (uint32_t(ne) * sizeof(T) + 15u) & ~15u;
-    const uint32_t cb = (uint32_t(ne) * 4u + 15u) & ~15u;
-    mbar_arrive_expect_tx(bar, vb + cb + (kBro ? 0u : cb));
-    bulk_g2s(sv, vals + e0, vb, bar);
-    bulk_g2s(sc, col + e0, cb, bar);
-    if constexpr (!kBro) bulk_g2s(sr, rows + e0, cb, bar);
+  if (lane == 0) {  // L2 prefetch (TMA engine) of the batches after the first one
+    const int64_t p0 = e0 + 32 * TB;
+    const int64_t p1 = min(e0 + 32 * int64_t(T_steps), nnz) & ~int64_t(3);
+    if (p1 > p0) {
+      prefetch_l2(col + p0, uint32_t((p1 - p0) * 4));
+      prefetch_l2(vals + p0, uint32_t((p1 - p0) * sizeof(T)));
+      if constexpr (!kBro) prefetch_l2(rows + p0, uint32_t((p1 - p0) * 4));
+    }
   }
-  __syncwarp();
   const int first = (int)base_row[i];
   int row = first;
   int b = 0;
@@ -534,38 +515,20 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, const uint32_t* __restrict__ word
       r[4] = rc.x; r[5] = rc.y; r[6] = rc.z; r[7] = rc.w;
       __syncwarp();
     }
-    if (t0 == 0) mbar_wait(bar, 0);             // the interval's arrays have landed
-    const int j0 = int(el - e0);                 // this lane's first entry inside the interval
-    {
-      const int4 c0v = *reinterpret_cast<const int4*>(sc + j0);
-      const int4 c1v = *reinterpret_cast<const int4*>(sc + j0 + 4);
-      c[0] = c0v.x; c[1] = c0v.y; c[2] = c0v.z; c[3] = c0v.w;
-      c[4] = c1v.x; c[5] = c1v.y; c[6] = c1v.z; c[7] = c1v.w;
-      if constexpr (!kBro) {
-        const int4 r0v = *reinterpret_cast<const int4*>(sr + j0);
-        const int4 r1v = *reinterpret_cast<const int4*>(sr + j0 + 4);
-        r[0] = r0v.x; r[1] = r0v.y; r[2] = r0v.z; r[3] = r0v.w;
-        r[4] = r1v.x; r[5] = r1v.y; r[6] = r1v.z; r[7] = r1v.w;
-      }
+    if (el + TB <= nnz) {
+      if constexpr (!kBro) load8_s32(r, rows + el);
+      load8_s32(c, col + el);
+      Vec8<T> vv;
+      vv.load(vals + el);
 #pragma unroll
-      for (int u = 0; u < TB / Chunk<T>::N; ++u) {
-        if constexpr (Chunk<T>::N == 2) {
-          const double2 q = *reinterpret_cast<const double2*>(sv + j0 + 2 * u);
-          v[2 * u] = q.x; v[2 * u + 1] = q.y;
-        } else {
-          const float4 q = *reinterpret_cast<const float4*>(sv + j0 + 4 * u);
-          v[4 * u] = q.x; v[4 * u + 1] = q.y; v[4 * u + 2] = q.z; v[4 * u + 3] = q.w;
-        }
-      }
-    }
-    if (j0 + TB > ne) {  // tail of the last interval: entries past nnz repeat the last row, value 0
+      for (int k = 0; k < TB; ++k) v[k] = vv.v[k];
+    } else {  // tail of the last interval: entries past nnz repeat the last row with value 0
 #pragma unroll
       for (int k = 0; k < TB; ++k) {
-        if (j0 + k >= ne) {
-          if constexpr (!kBro) r[k] = sr[ne - 1];
-          c[k] = -1;
-          v[k] = T(0);
-        }
+        const bool ok = el + k < nnz;
+        if constexpr (!kBro) r[k] = ld_stream_s32(rows + (ok ? el + k : nnz - 1));
+        c[k] = ok ? ld_stream_s32(col + el + k) : -1;
+        v[k] = ok ? ld_stream(vals + el + k) : T(0);
       }
     }
     T xv[TB];
