@@ -31,18 +31,19 @@ namespace dev {
 constexpr int kWarp = 32;
 
 // ------------------------------------------------------------------ loads
-// Streamed arrays use the ld.global.cs (cache-streaming, evict-first)
-// intrinsics: the compiler treats them as real loads, so guarded tail loads
-// (cond ? ld(p) : 0) are never if-converted into unconditional out-of-bounds
-// reads (a pure inline-asm load was, compute-sanitizer memcheck caught it),
-// while they still schedule freely (an asm volatile load cost 14% on C5 fp32).
+// Streamed arrays go through the non-coherent read-only path (ld.global.nc,
+// the __ldg builtin).  The builtin is a real load to the compiler, so guarded
+// tail loads (cond ? ld(p) : 0) are never if-converted into unconditional
+// out-of-bounds reads, which a pure inline-asm load was (compute-sanitizer
+// memcheck caught it); the generic-path streaming loads (__ldcs,
+// ld.global.cs) were measured 14% slower on C5 fp32.
 __device__ __forceinline__ uint4 ld_stream_u4(const uint32_t* p) {
-  return __ldcs(reinterpret_cast<const uint4*>(p));
+  return __ldg(reinterpret_cast<const uint4*>(p));
 }
-__device__ __forceinline__ uint32_t ld_stream_u32(const uint32_t* p) { return __ldcs(p); }
-__device__ __forceinline__ int32_t ld_stream_s32(const int32_t* p) { return __ldcs(p); }
-__device__ __forceinline__ double ld_stream(const double* p) { return __ldcs(p); }
-__device__ __forceinline__ float ld_stream(const float* p) { return __ldcs(p); }
+__device__ __forceinline__ uint32_t ld_stream_u32(const uint32_t* p) { return __ldg(p); }
+__device__ __forceinline__ int32_t ld_stream_s32(const int32_t* p) { return __ldg(p); }
+__device__ __forceinline__ double ld_stream(const double* p) { return __ldg(p); }
+__device__ __forceinline__ float ld_stream(const float* p) { return __ldg(p); }
 
 // 16-byte value chunk: 2 doubles or 4 floats
 template <typename T> struct Chunk;
@@ -50,7 +51,7 @@ template <> struct Chunk<double> {
   double v[2];
   static constexpr int N = 2;
   __device__ __forceinline__ void load(const double* p) {
-    const double2 q = __ldcs(reinterpret_cast<const double2*>(p));
+    const double2 q = __ldg(reinterpret_cast<const double2*>(p));
     v[0] = q.x; v[1] = q.y;
   }
 };
@@ -58,7 +59,7 @@ template <> struct Chunk<float> {
   float v[4];
   static constexpr int N = 4;
   __device__ __forceinline__ void load(const float* p) {
-    const float4 q = __ldcs(reinterpret_cast<const float4*>(p));
+    const float4 q = __ldg(reinterpret_cast<const float4*>(p));
     v[0] = q.x; v[1] = q.y; v[2] = q.z; v[3] = q.w;
   }
 };
