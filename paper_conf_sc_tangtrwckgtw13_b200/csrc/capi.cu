@@ -83,14 +83,19 @@ bro_status_t dev_upload(bro_matrix_s* A, P** dst, const void* src, size_t bytes)
   *dst = nullptr;
   if (bytes == 0) return BRO_OK;
   void* p = nullptr;
-  cudaError_t e = cudaMalloc(&p, bytes);
+  // every array carries kStreamPad zeroed bytes past its end: the kernels'
+  // 16-byte chunk loads may be issued speculatively (see kernels.cuh "loads")
+  const size_t pad = bro::dev::kStreamPad;
+  cudaError_t e = cudaMalloc(&p, bytes + pad);
   if (e != cudaSuccess) return fail(BRO_ERR_OOM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
-  A->device_bytes += (int64_t)bytes;
+  A->device_bytes += (int64_t)(bytes + pad);
   *dst = static_cast<P*>(p);
   if (src) {
     e = cudaMemcpy(p, src, bytes, cudaMemcpyHostToDevice);
     if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("cudaMemcpy H2D: ") + cudaGetErrorString(e));
   }
+  e = cudaMemset(static_cast<char*>(p) + bytes, 0, pad);
+  if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("cudaMemset: ") + cudaGetErrorString(e));
   return BRO_OK;
 }
 
