@@ -338,20 +338,9 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
         colmeta[w][lane] = make_uint2(uint32_t(rel >> 5) * 128u, uint32_t(rel & 31) | ((32u - uint32_t(b)) << 8));
       }
       __syncwarp();
-      // fp32: the next group's values are loaded one group ahead (software
-      // pipelining, 8 extra registers); fp64 has no register room for it
-      constexpr bool kPipe = sizeof(T) == 4;
-      T vn[G];
-      if (kPipe) load_vals<T, G>(vn, vs, jb, l, lfull, lane);
       for (int g = 0; g < nb; g += G) {
         T v[G];
-        if (kPipe) {
-#pragma unroll
-          for (int k = 0; k < G; ++k) v[k] = vn[k];
-          if (g + G < nb) load_vals<T, G>(vn, vs, jb + g + G, l, lfull, lane);
-        } else {
-          load_vals<T, G>(v, vs, jb + g, l, lfull, lane);
-        }
+        load_vals<T, G>(v, vs, jb + g, l, lfull, lane);
         int cidx[G];
         bool ok[G];
 #pragma unroll
