@@ -73,6 +73,7 @@ struct bro_matrix_s {
   void* d_xs = nullptr;
   void* d_ys = nullptr;
   int64_t device_bytes = 0;
+  uint32_t bulk_unit_max = 0;  // largest staged slice of the bulk BRO-ELL kernel (bytes)
   bro_info_t info{};
 };
 
@@ -199,6 +200,10 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
         A->s = A->ell.s;
         A->ell_words = (int64_t)A->ell.words.size();
         A->ell_slots = (int64_t)(A->ell.vals.size() / A->vsize);
+        for (int64_t t = 0; t < A->s; ++t)
+          A->bulk_unit_max = std::max(A->bulk_unit_max,
+              bro::dev::bulk_unit_bytes(A->ell.colptr[t], int(A->ell.colptr[t + 1] - A->ell.colptr[t]),
+                                        int(A->ell.symptr[t + 1] - A->ell.symptr[t]), A->vsize));
       } else {
         bro::build_plain_ell(rv, K, A->pell);
         A->pitch = A->pell.pitch;
@@ -317,8 +322,53 @@ void launch_bro_ell_od(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
 constexpr int kEllWarps = 8;      // slices per block
 constexpr int kEllMinBlocks = 4;  // 32 resident warps per SM (64 registers)
 
+// Bulk-staged BRO-ELL (V = 1 only): per-warp ring of nslot slots, each
+// holding one whole slice.  Ring bytes per warp: BRO_RING_KB (tuning; default
+// kBulkRingKB).  Returns false when a slice does not fit twice in the ring
+// (then the register-staged kernel runs).
+constexpr int kBulkWarps = 4;
+constexpr int kBulkRingKB = 16;
+constexpr int kBulkG = 16;
+constexpr int kMaxSmemPerBlock = 227 * 1024;
+
+int env_int(const char* name, int dflt) {
+  const char* v = std::getenv(name);
+  return v && *v ? std::atoi(v) : dflt;
+}
+
+template <typename T>
+bool launch_bro_ell_bulk(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+  using namespace bro::dev;
+  using L = BulkSmem<kBulkWarps>;
+  const int unit = int((A->bulk_unit_max + 127) / 128 * 128);
+  if (unit == 0) return false;
+  // at least two slots per warp (one in flight while one is consumed)
+  const int ring = std::max(env_int("BRO_RING_KB", kBulkRingKB) * 1024, 2 * unit);
+  const int fit = (kMaxSmemPerBlock - L::bytes(0, unit)) / (kBulkWarps * unit);  // slots the block can hold
+  const int nslot = std::min({kBulkMaxSlots, ring / unit, fit});
+  if (nslot < 2) return false;
+  const int smem = L::bytes(nslot, unit);
+  auto kern = bro_ell_spmv_bulk<T, kBulkWarps, kBulkG, 1>;
+  static int configured = 0;
+  if (smem > configured) {
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) return false;
+    configured = smem;
+  }
+  int per_sm = 0, sms = 0, dev = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kBulkWarps * 32, smem);
+  if (per_sm < 1) return false;
+  const int64_t need = (A->s + kBulkWarps - 1) / kBulkWarps;
+  const unsigned grid = (unsigned)std::min<int64_t>(need, int64_t(per_sm) * sms);
+  kern<<<grid, kBulkWarps * 32, smem, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr,
+                                            (const T*)A->d_ell_vals, x, y, nslot, unit);
+  return true;
+}
+
 template <typename T, int V>
 void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+  if (V == 1 && env_int("BRO_ELL_KERNEL", 0) != 1 && launch_bro_ell_bulk<T>(A, x, y, st)) return;
   launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks>(A, x, y, st);
 }
 

@@ -368,6 +368,216 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
   }
 }
 
+// ------------------------------------------------------------------ BRO-ELL, bulk-staged
+// Same offset decode, but every byte of a slice (its values, its symbol
+// stream in the paper's V = 1 multiplexing comp_str[q*h + tid], and
+// its widths) is moved into shared memory by the TMA engine
+// (cp.async.bulk, completion on an mbarrier) while the warp works on an
+// earlier slice.  Each warp owns a ring of `nslot` slots (one slice each);
+// with nslot - 1 slices in flight per warp the bytes in flight no longer
+// depend on registers, and the register budget goes to x gathers instead
+// (G per group).  V = 1 is what makes staging free: symbol row q of the
+// slice is the 128-byte row [q][lane] of the window (conflict-free), so the
+// slot IS the decode window (no copy), and each delta is
+//     delta = funnelshift(w[q+1], w[q], o mod 32) >> (32 - b),  q = o / 32.
+// Metadata of 32 upcoming slices is fetched per round trip (one per lane).
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n"
+      "WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra WAIT_%=;\n}\n" :: "r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar,
+                                         uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+      :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(policy) : "memory");
+}
+__device__ __forceinline__ uint64_t policy_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ void prefetch_l2_line(const void* p) {
+  asm volatile("prefetch.global.L2 [%0];" :: "l"(p));
+}
+
+constexpr int kBulkMaxSlots = 8;
+constexpr int kBulkMetaRing = 64;
+struct BulkMeta { uint64_t c0, q0; int l, S; };
+
+// Bytes of one staged slice (host and device agree on this).
+__host__ __device__ __forceinline__ uint32_t bulk_unit_bytes(uint64_t c0, int l, int S, int vsize) {
+  const uint64_t ba_lo = c0 & ~uint64_t(15);
+  const uint64_t ba_hi = (c0 + uint64_t(l) + 15) & ~uint64_t(15);
+  return uint32_t(32 * l * vsize + 128 * S + (ba_hi - ba_lo));
+}
+
+// Dynamic shared memory layout of one block (per warp: slot barriers, meta
+// ring, column metadata; then the warps' slot rings; 128 bytes of slack so
+// the decode's w[q+1] read of the last symbol row stays inside).
+template <int kWarps>
+struct BulkSmem {
+  static constexpr int kBarOff = 0;
+  static constexpr int kMetaOff = kBarOff + kWarps * kBulkMaxSlots * 8;
+  static constexpr int kColOff = kMetaOff + kWarps * kBulkMetaRing * int(sizeof(BulkMeta));
+  static constexpr int kRingOff = ((kColOff + kWarps * 32 * 8) + 127) / 128 * 128;
+  static __host__ __device__ int bytes(int nslot, int slot_bytes) {
+    return kRingOff + kWarps * nslot * slot_bytes + 128;
+  }
+};
+
+template <typename T, int kWarps, int G, int kMinBlocks>
+__global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
+bro_ell_spmv_bulk(int64_t m, int64_t s, const uint32_t* __restrict__ words,
+                  const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
+                  const uint64_t* __restrict__ symptr, const T* __restrict__ vals,
+                  const T* __restrict__ x, T* __restrict__ y, int nslot, int slot_bytes) {
+  using L = BulkSmem<kWarps>;
+  constexpr int VV = Chunk<T>::N;
+  extern __shared__ __align__(128) uint8_t smem[];
+  const int lane = threadIdx.x & 31;
+  const int w = threadIdx.x / 32;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L::kBarOff) + w * kBulkMaxSlots;
+  BulkMeta* metas = reinterpret_cast<BulkMeta*>(smem + L::kMetaOff) + w * kBulkMetaRing;
+  uint2* cm = reinterpret_cast<uint2*>(smem + L::kColOff) + w * 32;
+  uint8_t* ring = smem + L::kRingOff + size_t(w) * nslot * slot_bytes;
+
+  const int64_t stride = int64_t(gridDim.x) * kWarps;
+  const int64_t t0 = int64_t(blockIdx.x) * kWarps + w;
+  const int nk = t0 < s ? int((s - t0 + stride - 1) / stride) : 0;
+  if (lane == 0) {
+    for (int i = 0; i < nslot; ++i) mbar_init(bars + i, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncwarp();
+  const uint64_t pol = policy_evict_first();
+
+  // metadata of units [kb, kb + 32) into the meta ring (all lanes); the
+  // next batch's lines are prefetched into L2 half a batch ahead.
+  auto load_metas = [&](int kb) {
+    const int k = kb + lane;
+    if (k < nk) {
+      const int64_t t = t0 + k * stride;
+      const uint64_t c0 = __ldg(colptr + t), q0 = __ldg(symptr + t);
+      metas[k & (kBulkMetaRing - 1)] =
+          BulkMeta{c0, q0, int(__ldg(colptr + t + 1) - c0), int(__ldg(symptr + t + 1) - q0)};
+    }
+    __syncwarp();
+  };
+  auto issue = [&](int k, int slot) {  // uniform across the warp
+    if ((k & 31) == 0) load_metas(k);
+    if ((k & 31) == 16) {
+      const int kn = (k & ~31) + 32 + lane;
+      if (kn < nk) {
+        const int64_t t = t0 + kn * stride;
+        prefetch_l2_line(colptr + t);
+        prefetch_l2_line(symptr + t);
+      }
+    }
+    if (lane == 0) {
+      const BulkMeta mt = metas[k & (kBulkMetaRing - 1)];
+      uint8_t* dst = ring + size_t(slot) * slot_bytes;
+      const uint32_t vb = uint32_t(32 * mt.l * int(sizeof(T)));
+      const uint32_t sb = uint32_t(128 * mt.S);
+      const uint64_t ba_lo = mt.c0 & ~uint64_t(15);
+      const uint32_t bb = uint32_t(((mt.c0 + uint64_t(mt.l) + 15) & ~uint64_t(15)) - ba_lo);
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      mbar_arrive_expect_tx(bars + slot, vb + sb + bb);
+      if (vb) bulk_g2s(dst, vals + 32 * mt.c0, vb, bars + slot, pol);
+      if (sb) bulk_g2s(dst + vb, words + 32 * mt.q0, sb, bars + slot, pol);
+      if (bb) bulk_g2s(dst + vb + sb, bit_alloc + ba_lo, bb, bars + slot, pol);
+    }
+  };
+
+  const int npre = min(nslot - 1, nk);
+  for (int k = 0; k < npre; ++k) issue(k, k);
+  int slot = 0, phase = 0;           // consumer position
+  int islot = nslot - 1;             // slot of unit k + nslot - 1 (= slot of unit k - 1)
+  for (int k = 0; k < nk; ++k) {
+    if (k + nslot - 1 < nk) issue(k + nslot - 1, islot);  // into the slot freed by unit k - 1
+    islot = slot;
+    mbar_wait(bars + slot, uint32_t(phase));
+    const BulkMeta mt = metas[k & (kBulkMetaRing - 1)];
+    const int l = mt.l;
+    const uint8_t* base = ring + size_t(slot) * slot_bytes;
+    const T* sv = reinterpret_cast<const T*>(base);
+    const char* sw_lane = reinterpret_cast<const char*>(base + 32 * l * sizeof(T)) + 4 * lane;
+    const uint8_t* sb = base + 32 * l * sizeof(T) + 128 * mt.S + (mt.c0 & 15);
+    const int lfull = (l / VV) * VV;
+    const int tw = l - lfull;
+    T sum = T(0);
+    int col = -1;
+    int obase = 0;
+    for (int jb = 0; jb < l; jb += 32) {
+      const int nb = min(32, l - jb);
+      const int b = lane < nb ? int(sb[jb + lane]) : 0;
+      int incl = b;
+#pragma unroll
+      for (int off = 1; off < 32; off <<= 1) {
+        const int o = __shfl_up_sync(0xffffffffu, incl, off);
+        if (lane >= off) incl += o;
+      }
+      const int tot = __shfl_sync(0xffffffffu, incl, 31);
+      {
+        const int rel = b ? obase + incl - b : 0;  // bit offset of column jb+lane in every row stream
+        cm[lane] = make_uint2(uint32_t(rel >> 5) * 128u, uint32_t(rel & 31) | ((32u - uint32_t(b)) << 8));
+      }
+      __syncwarp();
+      for (int g = 0; g < nb; g += G) {
+        int cidx[G];
+        bool ok[G];
+#pragma unroll
+        for (int k2 = 0; k2 < G; ++k2) {
+          const uint2 mm = cm[g + k2];  // broadcast
+          const uint32_t* wp = reinterpret_cast<const uint32_t*>(sw_lane + mm.x);
+          const uint32_t d = shr_clamp(__funnelshift_l(wp[32], wp[0], mm.y), mm.y >> 8);
+          col += int(d);
+          cidx[k2] = col;
+          ok[k2] = d != 0u;
+        }
+        T xv[G];
+#pragma unroll
+        for (int k2 = 0; k2 < G; ++k2) xv[k2] = ok[k2] ? ldg_x(x + cidx[k2]) : T(0);
+        const int j0 = jb + g;
+#pragma unroll
+        for (int u = 0; u < G / VV; ++u) {
+          const int jj = j0 + u * VV;
+          T v[VV];
+          if (jj + VV <= lfull) {
+            if constexpr (VV == 2) {
+              const double2 c2 = *reinterpret_cast<const double2*>(sv + 32 * jj + lane * VV);
+              v[0] = c2.x; v[1] = c2.y;
+            } else {
+              const float4 c4 = *reinterpret_cast<const float4*>(sv + 32 * jj + lane * VV);
+              v[0] = c4.x; v[1] = c4.y; v[2] = c4.z; v[3] = c4.w;
+            }
+          } else {
+#pragma unroll
+            for (int q = 0; q < VV; ++q)
+              v[q] = (jj + q < l) ? sv[32 * lfull + lane * tw + (jj + q - lfull)] : T(0);
+          }
+#pragma unroll
+          for (int q = 0; q < VV; ++q) sum = fma(v[q], xv[u * VV + q], sum);  // padding: v = 0, x = 0
+        }
+      }
+      obase += tot;
+      __syncwarp();
+    }
+    const int64_t row = 32 * (t0 + int64_t(k) * stride) + lane;
+    if (row < m) y[row] = sum;
+    if (++slot == nslot) { slot = 0; phase ^= 1; }
+  }
+}
+
 // Decode-only variant: decoded column (or -1) per slot in V=1 slot order.
 template <int V>
 __global__ void bro_ell_decode(int64_t s, const uint32_t* __restrict__ words,

@@ -68,6 +68,30 @@ def test_vec_words_variants(lib, dev, V):
         M.close()
 
 
+BULK_CASES = CASES + [
+    ("multiblock", lambda: random_csr(3000, 4000, 12, max_len=90, empty_frac=0.05)),
+    ("short", lambda: random_csr(5000, 7000, 13, max_len=3, empty_frac=0.1)),
+]
+
+
+@pytest.mark.parametrize("kernel", ["bulk", "od"])
+@pytest.mark.parametrize("ring_kb", ["", "1", "64"])
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_bro_ell_v1_kernels(lib, dev, kernel, ring_kb, dtype, monkeypatch):
+    """V = 1 (the paper's multiplexing): the bulk-staged kernel (TMA ring of
+    whole slices, 2..8 slots per warp depending on BRO_RING_KB) and the
+    register-staged kernel give the oracle's y on every case, including slices
+    with several 32-column blocks and slices too large to stage."""
+    monkeypatch.setenv("BRO_ELL_KERNEL", "1" if kernel == "od" else "0")
+    monkeypatch.setenv("BRO_RING_KB", ring_kb)
+    for _, mk in BULK_CASES:
+        A = mk()
+        for fmt in ("ell", "hyb"):
+            M, x, y = _run(lib, A, fmt, 1, dtype, dev, V=1)
+            _check_y(A, x, y, dtype)
+            M.close()
+
+
 def test_empty_matrix(lib, dev):
     A = Csr(0, 5, np.zeros(1, np.int64), np.zeros(0, np.int32), np.zeros(0), "empty")
     M = lib.BroMatrix(A, fmt="hyb", device=0)
