@@ -328,7 +328,7 @@ constexpr int kEllMinBlocks = 4;  // 32 resident warps per SM (64 registers)
 // (then the register-staged kernel runs).
 constexpr int kBulkWarps = 4;
 constexpr int kBulkRingKB = 16;
-constexpr int kBulkG = 16;
+constexpr int kBulkG = 32;
 constexpr int kMaxSmemPerBlock = 227 * 1024;
 
 int env_int(const char* name, int dflt) {
@@ -336,8 +336,8 @@ int env_int(const char* name, int dflt) {
   return v && *v ? std::atoi(v) : dflt;
 }
 
-template <typename T>
-bool launch_bro_ell_bulk(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+template <typename T, int G>
+bool launch_bro_ell_bulk_g(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   using namespace bro::dev;
   using L = BulkSmem<kBulkWarps>;
   const int unit = int((A->bulk_unit_max + 127) / 128 * 128);
@@ -348,7 +348,7 @@ bool launch_bro_ell_bulk(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   const int nslot = std::min({kBulkMaxSlots, ring / unit, fit});
   if (nslot < 2) return false;
   const int smem = L::bytes(nslot, unit);
-  auto kern = bro_ell_spmv_bulk<T, kBulkWarps, kBulkG, 1>;
+  auto kern = bro_ell_spmv_bulk<T, kBulkWarps, G, 1>;
   static int configured = 0;
   if (smem > configured) {
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess) return false;
@@ -364,6 +364,12 @@ bool launch_bro_ell_bulk(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   kern<<<grid, kBulkWarps * 32, smem, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr,
                                             (const T*)A->d_ell_vals, x, y, nslot, unit);
   return true;
+}
+
+template <typename T>
+bool launch_bro_ell_bulk(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+  if (env_int("BRO_BULK_G", kBulkG) == 16) return launch_bro_ell_bulk_g<T, 16>(A, x, y, st);
+  return launch_bro_ell_bulk_g<T, 32>(A, x, y, st);
 }
 
 template <typename T, int V>
