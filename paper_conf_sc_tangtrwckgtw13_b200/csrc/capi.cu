@@ -22,6 +22,8 @@ bro_status_t fail(bro_status_t s, const std::string& msg) {
 }
 
 constexpr int kCooThreads = 256;
+constexpr int kCooMaxUpi = 4;   // work units per COO interval (8 steps = 256 entries each at 4)
+constexpr int kCooUpi = 4;
 constexpr int kPlainThreads = 256;
 
 struct DeviceGuard {
@@ -70,6 +72,7 @@ struct bro_matrix_s {
   void* d_cf = nullptr;
   void* d_cl = nullptr;
   int32_t* d_last_row = nullptr;
+  int32_t* d_first_row = nullptr;
   void* d_xs = nullptr;
   void* d_ys = nullptr;
   int64_t device_bytes = 0;
@@ -105,7 +108,7 @@ void free_device(bro_matrix_s* A) {
   DeviceGuard g(A->device);
   void* ps[] = {A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr, A->d_ell_vals, A->d_pell_col,
                 A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr, A->d_coo_row,
-                A->d_coo_col, A->d_coo_vals, A->d_cf, A->d_cl, A->d_last_row, A->d_xs, A->d_ys};
+                A->d_coo_col, A->d_coo_vals, A->d_cf, A->d_cl, A->d_last_row, A->d_first_row, A->d_xs, A->d_ys};
   for (void* p : ps)
     if (p) cudaFree(p);
 }
@@ -268,9 +271,12 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
       } else {
         UP(A->d_coo_row, A->coo.row);
       }
-      if (st == BRO_OK) st = dev_upload(A, &A->d_cf, nullptr, size_t(A->nI) * A->vsize);
-      if (st == BRO_OK) st = dev_upload(A, &A->d_cl, nullptr, size_t(A->nI) * A->vsize);
-      if (st == BRO_OK) st = dev_upload(A, &A->d_last_row, nullptr, size_t(A->nI) * 4);
+      // per-work-unit carries (up to kCooMaxUpi units per interval)
+      const size_t nU = size_t(A->nI) * kCooMaxUpi;
+      if (st == BRO_OK) st = dev_upload(A, &A->d_cf, nullptr, nU * A->vsize);
+      if (st == BRO_OK) st = dev_upload(A, &A->d_cl, nullptr, nU * A->vsize);
+      if (st == BRO_OK) st = dev_upload(A, &A->d_last_row, nullptr, nU * 4);
+      if (st == BRO_OK) st = dev_upload(A, &A->d_first_row, nullptr, nU * 4);
     }
 #undef UP
     if (st != BRO_OK) {
@@ -399,28 +405,25 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   }
   if (A->has_coo && A->nI > 0) {
     const int warps = kCooThreads / 32;
-    dim3 grid((unsigned)((A->nI + warps - 1) / warps));
+    const int upi = std::max(1, std::min(kCooMaxUpi, env_int("BRO_COO_UPI", kCooUpi)));
+    const int64_t nU = A->nI * upi;
+    dim3 grid((unsigned)((nU + warps - 1) / warps));
     const int T_ = A->opts.coo_T;
+    auto args = [&](auto kern) {
+      kern<<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, upi, A->d_coo_words, A->d_coo_base,
+                                         A->d_coo_width, A->d_coo_symptr, A->d_coo_row, A->d_coo_col,
+                                         (const T*)A->d_coo_vals, x, y, (T*)A->d_cf, (T*)A->d_cl,
+                                         A->d_first_row, A->d_last_row);
+    };
     if (A->opts.codec) {
-      if (V == 4)
-        coo_spmv<T, 4, true, kCooThreads><<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, A->d_coo_words,
-            A->d_coo_base, A->d_coo_width, A->d_coo_symptr, nullptr, A->d_coo_col, (const T*)A->d_coo_vals, x, y,
-            (T*)A->d_cf, (T*)A->d_cl, A->d_last_row);
-      else if (V == 2)
-        coo_spmv<T, 2, true, kCooThreads><<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, A->d_coo_words,
-            A->d_coo_base, A->d_coo_width, A->d_coo_symptr, nullptr, A->d_coo_col, (const T*)A->d_coo_vals, x, y,
-            (T*)A->d_cf, (T*)A->d_cl, A->d_last_row);
-      else
-        coo_spmv<T, 1, true, kCooThreads><<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, A->d_coo_words,
-            A->d_coo_base, A->d_coo_width, A->d_coo_symptr, nullptr, A->d_coo_col, (const T*)A->d_coo_vals, x, y,
-            (T*)A->d_cf, (T*)A->d_cl, A->d_last_row);
+      if (V == 4) args(coo_spmv<T, 4, true, kCooThreads>);
+      else if (V == 2) args(coo_spmv<T, 2, true, kCooThreads>);
+      else args(coo_spmv<T, 1, true, kCooThreads>);
     } else {
-      coo_spmv<T, 4, false, kCooThreads><<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, nullptr,
-          A->d_coo_base, nullptr, nullptr, A->d_coo_row, A->d_coo_col, (const T*)A->d_coo_vals, x, y,
-          (T*)A->d_cf, (T*)A->d_cl, A->d_last_row);
+      args(coo_spmv<T, 4, false, kCooThreads>);
     }
-    dim3 g2((unsigned)((A->nI + 255) / 256));
-    coo_fixup<T><<<g2, 256, 0, st>>>(A->nI, A->d_coo_base, A->d_last_row, (const T*)A->d_cf,
+    dim3 g2((unsigned)((nU + 255) / 256));
+    coo_fixup<T><<<g2, 256, 0, st>>>(nU, A->d_first_row, A->d_last_row, (const T*)A->d_cf,
                                      (const T*)A->d_cl, y);
   }
   cudaError_t e = cudaGetLastError();

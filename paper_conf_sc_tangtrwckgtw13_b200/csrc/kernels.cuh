@@ -675,50 +675,59 @@ __device__ __forceinline__ void load8_s32(int* d, const int32_t* p) {
 
 template <typename T, int V, bool kBro, int kThreads>
 __global__ void __launch_bounds__(kThreads)
-coo_spmv(int64_t nnz, int64_t nI, int T_steps, const uint32_t* __restrict__ words,
+coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restrict__ words,
          const uint32_t* __restrict__ base_row, const uint8_t* __restrict__ width,
          const uint64_t* __restrict__ symptr, const int32_t* __restrict__ rows,
          const int32_t* __restrict__ col, const T* __restrict__ vals, const T* __restrict__ x,
          T* __restrict__ y, T* __restrict__ carry_first, T* __restrict__ carry_last,
-         int32_t* __restrict__ last_row) {
+         int32_t* __restrict__ first_row, int32_t* __restrict__ last_row) {
   constexpr int TB = 8;
   __shared__ __align__(16) int32_t rowbuf[kThreads / 32][TB * 32];
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
-  const int64_t i = int64_t(blockIdx.x) * (kThreads / 32) + w;
+  // work unit = steps [ts, ts + T_steps / upi) of interval i (upi units per interval)
+  const int64_t u = int64_t(blockIdx.x) * (kThreads / 32) + w;
+  const int64_t i = u / upi;
   if (i >= nI) return;
+  const int steps = T_steps / upi;
+  const int ts = int(u - i * upi) * steps;
   int32_t* rb = rowbuf[w];
   const int64_t e0 = i * 32 * T_steps;
-  if (lane == 0) {  // L2 prefetch (TMA engine) of the batches after the first one
-    const int64_t p0 = e0 + 32 * TB;
-    const int64_t p1 = min(e0 + 32 * int64_t(T_steps), nnz) & ~int64_t(3);
+  if (lane == 0) {  // L2 prefetch (TMA engine) of the unit's batches after the first one
+    const int64_t p0 = e0 + 32 * (ts + TB);
+    const int64_t p1 = min(e0 + 32 * int64_t(ts + steps), nnz) & ~int64_t(3);
     if (p1 > p0) {
       prefetch_l2(col + p0, uint32_t((p1 - p0) * 4));
       prefetch_l2(vals + p0, uint32_t((p1 - p0) * sizeof(T)));
       if constexpr (!kBro) prefetch_l2(rows + p0, uint32_t((p1 - p0) * 4));
     }
   }
-  const int first = (int)base_row[i];
-  int row = first;
+  int row = (int)base_row[i];
   int b = 0;
   LaneStream<V> ls;
   if constexpr (kBro) {
     b = width[i];
     const uint64_t q0 = symptr[i];
     ls.init(words + 32 * q0, int(symptr[i + 1] - q0), lane);
+    if (b)
+      for (int t = 0; t < ts; ++t) row += (int)ls.get(b, lane);  // rows of the steps before the unit
   }
+  // row of the unit's first entry (element (ts, 0))
+  int first = 0;
+  if constexpr (!kBro) first = rows[min(e0 + 32 * ts, nnz - 1)];
+  bool first_pending = kBro;  // kBro: lane 0's row at step ts is known only after the first decode
   T carry = T(0);   // partial of row crow carried from earlier batches (not yet written)
   int crow = first;
-  // A complete segment of row r.  Every row other than the interval's first
-  // and last rows is complete in exactly one place of the whole launch, so it
+  // A complete segment of row r.  Every row other than the unit's first and
+  // last rows is complete in exactly one place of the whole launch, so it
   // receives exactly one addition: a fire-and-forget RED (atomicAdd with the
   // result unused) is as deterministic as y[r] += v but does not serialize
   // the warp on a load -> store chain per segment.
   auto emit = [&](int r, T v) {
-    if (r == first) carry_first[i] = v;
+    if (r == first) carry_first[u] = v;
     else atomicAdd(y + r, v);
   };
-  for (int t0 = 0; t0 < T_steps; t0 += TB) {
+  for (int t0 = ts; t0 < ts + steps; t0 += TB) {
     const int64_t eb = e0 + 32 * t0;            // first entry of the batch
     const int64_t el = eb + TB * lane;          // this lane's first entry (transposed)
     int r[TB], c[TB];
@@ -734,6 +743,11 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, const uint32_t* __restrict__ word
       const int4 rc = *reinterpret_cast<const int4*>(rb + TB * lane + 4);
       r[0] = ra.x; r[1] = ra.y; r[2] = ra.z; r[3] = ra.w;
       r[4] = rc.x; r[5] = rc.y; r[6] = rc.z; r[7] = rc.w;
+      if (first_pending) {
+        first = rb[0];
+        crow = first;
+        first_pending = false;
+      }
       __syncwarp();
     }
     if (el + TB <= nnz) {
@@ -803,38 +817,41 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, const uint32_t* __restrict__ word
     crow = __shfl_sync(0xffffffffu, L, 31);
   }
   if (lane == 0) {
-    last_row[i] = crow;
+    first_row[u] = first;
+    last_row[u] = crow;
     if (crow == first) {
-      carry_first[i] = carry;
-      carry_last[i] = T(0);
+      carry_first[u] = carry;
+      carry_last[u] = T(0);
     } else {
-      carry_last[i] = carry;
+      carry_last[u] = carry;
     }
   }
 }
 
-// Deterministic application of interval carries (one thread per interval,
-// fixed summation order = interval order).
+// Deterministic application of the units' carries (one thread per unit,
+// fixed summation order = unit order).  first[u] / last[u] = rows of the
+// unit's first and last entries; cf = partial of the first row (the whole
+// unit if first == last), cl = partial of the last row.
 template <typename T>
-__global__ void coo_fixup(int64_t nI, const uint32_t* __restrict__ first,
+__global__ void coo_fixup(int64_t nU, const int32_t* __restrict__ first,
                           const int32_t* __restrict__ last_row, const T* __restrict__ cf,
                           const T* __restrict__ cl, T* __restrict__ y) {
   const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-  if (i >= nI) return;
-  const int F = (int)first[i];
+  if (i >= nU) return;
+  const int F = first[i];
   const int L = last_row[i];
-  if (L != F) {  // interval i is the first one holding row L
+  if (L != F) {  // unit i is the first one holding row L
     T acc = cl[i];
-    for (int64_t j = i + 1; j < nI && (int)first[j] == L; ++j) {
+    for (int64_t j = i + 1; j < nU && first[j] == L; ++j) {
       acc += cf[j];
       if (last_row[j] != L) break;
     }
     y[L] += acc;
   }
-  if (i == 0 || last_row[i - 1] != F) {  // interval i is the first one holding row F
+  if (i == 0 || last_row[i - 1] != F) {  // unit i is the first one holding row F
     T acc = cf[i];
     if (L == F) {
-      for (int64_t j = i + 1; j < nI && (int)first[j] == F; ++j) {
+      for (int64_t j = i + 1; j < nU && first[j] == F; ++j) {
         acc += cf[j];
         if (last_row[j] != F) break;
       }

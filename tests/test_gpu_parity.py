@@ -92,6 +92,26 @@ def test_bro_ell_v1_kernels(lib, dev, kernel, ring_kb, dtype, monkeypatch):
             M.close()
 
 
+@pytest.mark.parametrize("upi", ["1", "2", "4"])
+@pytest.mark.parametrize("codec", [1, 0])
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_coo_work_units(lib, dev, upi, codec, dtype, monkeypatch):
+    """COO traversal split into 1, 2 or 4 work units per 1024-entry interval
+    (carries per unit, deterministic fix-up over units) gives the oracle's y,
+    including units entirely past nnz and rows spanning many units."""
+    monkeypatch.setenv("BRO_COO_UPI", upi)
+    cases = CASES + [("longrow", lambda: random_csr(40, 20000, 14, max_len=5, long_frac=0.2,
+                                                    long_len=5000)),
+                     ("tail", lambda: random_csr(300, 400, 15, max_len=4))]
+    for _, mk in cases:
+        A = mk()
+        for fmt in ("coo", "hyb"):
+            for V in (1, 4):
+                M, x, y = _run(lib, A, fmt, codec, dtype, dev, V=V)
+                _check_y(A, x, y, dtype)
+                M.close()
+
+
 def test_empty_matrix(lib, dev):
     A = Csr(0, 5, np.zeros(1, np.int64), np.zeros(0, np.int32), np.zeros(0), "empty")
     M = lib.BroMatrix(A, fmt="hyb", device=0)
