@@ -49,7 +49,7 @@ def parse_args():
     ap.add_argument("--workload", default="C5", choices=sorted(WORKLOADS))
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--vec-words", type=int, default=4)
+    ap.add_argument("--vec-words", type=int, default=0, help="0 = auto (fp64: 1, fp32: 4)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--flush-l2", action="store_true", help="write a 2xL2 buffer between steps")
@@ -358,7 +358,7 @@ def main():
                                                 3: "webbase-like 1,000,005 rows", 4: "random-block 2M rows, BAR-reordered",
                                                 5: "3D 27-point stencil 200^3"}[cfg],
             "format": bro_name, "m": A.m, "n": A.n, "nnz": A.nnz,
-            "vec_words": args.vec_words,
+            "vec_words": info["vec_words"],
             "l2": ("flushed (2x L2 write) before every step" if args.flush_l2 else
                    ("inputs larger than L2" if alg_bytes > 2 * L2_BYTES else "L2-resident (warm)")),
             "parallelism": f"row-block x{world}" + (" + NCCL allgather of y per step" if world > 1 else ""),
@@ -367,7 +367,7 @@ def main():
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
                      "peak_kind": peak_kind,
-                     "kernel": f"bro_ell_spmv_od<{'double' if dtype == np.float64 else 'float'},V={args.vec_words}>"
+                     "kernel": f"bro_ell_spmv_od<{'double' if dtype == np.float64 else 'float'},V={info['vec_words']}>"
                      if fmt == "ell" else "bro_ell_spmv + coo_spmv + coo_fixup",
                      "algorithmic_bytes_per_launch": alg_bytes, "kernel_ms": kern_ms,
                      "frac_of_8TBps_spec": achieved / 8000.0},

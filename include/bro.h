@@ -86,7 +86,9 @@ typedef struct {
   int32_t slice_h;   /* BRO-ELL slice height h. Must be 32 (one warp per slice). */
   int32_t sym_bits;  /* sym_len. Must be 32. */
   int32_t vec_words; /* V: 1, 2 or 4 symbols per lane chunk.  1 = the paper's multiplexing
-                        (comp_str_i[q*h + tid]); default 4 = 16-byte per-lane chunks (128-bit loads). */
+                        (comp_str_i[q*h + tid]); 4 = 16-byte per-lane chunks (128-bit loads);
+                        0 (default) = auto: 1 for BRO_FP64, 4 for BRO_FP32 (measured fastest;
+                        bro_info_t.vec_words reports the resolved value). */
   int32_t coo_T;     /* BRO-COO steps per interval (interval = 32*T entries). Must be 32. */
   int64_t hyb_K;     /* HYB dividing column; -1 = the "less than a third" rule. */
   int32_t codec;     /* 1 = BRO compressed formats; 0 = uncompressed ELL/COO/HYB baseline. */
@@ -139,7 +141,7 @@ typedef enum {
   BRO_PART_PELL_VALS = 13     /* value[K*pitch]  plain ELL values (codec 0) */
 } bro_part_t;
 
-/* Fill *opts with the defaults: h 32, sym 32, V 4, T 32, K auto, codec 1. */
+/* Fill *opts with the defaults: h 32, sym 32, V 0 (auto), T 32, K auto, codec 1. */
 void bro_opts_default(bro_opts_t* opts);
 
 /* Build an ELL-only matrix (BRO-ELL if opts->codec == 1, else ELLPACK with

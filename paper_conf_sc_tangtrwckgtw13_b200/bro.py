@@ -225,7 +225,7 @@ class BroMatrix:
     """Owns one libbro handle.  `fmt` in {"ell", "hyb", "coo"}; codec=1 gives
     BRO-ELL / BRO-HYB / BRO-COO, codec=0 the uncompressed baseline."""
 
-    def __init__(self, A, fmt="ell", codec=1, device=0, dtype=None, vec_words=4, hyb_K=-1, min_bits=0):
+    def __init__(self, A, fmt="ell", codec=1, device=0, dtype=None, vec_words=0, hyb_K=-1, min_bits=0):
         vals = A.vals if dtype is None else A.vals.astype(dtype)
         self.dtype = np.dtype(vals.dtype)
         self.m, self.n, self.fmt, self.device = A.m, A.n, fmt, device

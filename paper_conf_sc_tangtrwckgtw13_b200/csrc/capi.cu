@@ -23,7 +23,7 @@ bro_status_t fail(bro_status_t s, const std::string& msg) {
 
 constexpr int kCooThreads = 256;
 constexpr int kCooMaxUpi = 4;   // work units per COO interval (8 steps = 256 entries each at 4)
-constexpr int kCooUpi = 4;
+constexpr int kCooUpi = 2;
 constexpr int kPlainThreads = 256;
 
 struct DeviceGuard {
@@ -76,7 +76,8 @@ struct bro_matrix_s {
   void* d_xs = nullptr;
   void* d_ys = nullptr;
   int64_t device_bytes = 0;
-  uint32_t bulk_unit_max = 0;  // largest staged slice of the bulk BRO-ELL kernel (bytes)
+  uint32_t bulk_unit_max = 0;
+  int64_t ell_max_l = 0;       // longest BRO-ELL slice (columns)  // largest staged slice of the bulk BRO-ELL kernel (bytes)
   bro_info_t info{};
 };
 
@@ -203,6 +204,7 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
         A->s = A->ell.s;
         A->ell_words = (int64_t)A->ell.words.size();
         A->ell_slots = (int64_t)(A->ell.vals.size() / A->vsize);
+        A->ell_max_l = A->ell.max_l;
         for (int64_t t = 0; t < A->s; ++t)
           A->bulk_unit_max = std::max(A->bulk_unit_max,
               bro::dev::bulk_unit_bytes(A->ell.colptr[t], int(A->ell.colptr[t + 1] - A->ell.colptr[t]),
@@ -302,15 +304,18 @@ bro_status_t common_checks(bro_dtype_t dtype, const bro_opts_t* opts, bro_opts_t
   *out = nullptr;
   if (dtype != BRO_FP32 && dtype != BRO_FP64) return fail(BRO_ERR_ARG, "dtype must be BRO_FP32 or BRO_FP64");
   if (opts) *o = *opts; else bro_opts_default(o);
+  // vec_words 0 = auto: the layout measured fastest for the dtype on B200
+  // (fp64: V = 1, the paper's multiplexing; fp32: V = 4, 16-byte lane chunks)
+  if (o->vec_words == 0) o->vec_words = dtype == BRO_FP64 ? 1 : 4;
   return check_opts(*o);
 }
 
 // Persistent grid: as many resident blocks as the SMs hold (queried once per
 // instantiation), capped by the number of slices.
-template <typename T, int V, int kWarps, int kMinBlocks>
+template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34>
 void launch_bro_ell_od(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   using namespace bro::dev;
-  auto kern = bro_ell_spmv_od<T, V, kWarps, kMinBlocks>;
+  auto kern = bro_ell_spmv_od<T, V, kWarps, kMinBlocks, G, kRows>;
   static int resident = 0;
   if (resident == 0) {
     int per_sm = 0, sms = 0, dev = 0;
@@ -327,6 +332,7 @@ void launch_bro_ell_od(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
 
 constexpr int kEllWarps = 8;      // slices per block
 constexpr int kEllMinBlocks = 4;  // 32 resident warps per SM (64 registers)
+constexpr int kEllMinBlocksShort = 6;  // fp32: 48 resident warps per SM (40 registers), slices of <= 4 columns; fp64: 40 (48 registers)
 
 // Bulk-staged BRO-ELL (V = 1 only): per-warp ring of nslot slots, each
 // holding one whole slice.  Ring bytes per warp: BRO_RING_KB (tuning; default
@@ -380,8 +386,13 @@ bool launch_bro_ell_bulk(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
 
 template <typename T, int V>
 void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
-  if (V == 1 && env_int("BRO_ELL_KERNEL", 0) != 1 && launch_bro_ell_bulk<T>(A, x, y, st)) return;
-  launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks>(A, x, y, st);
+  // BRO_ELL_KERNEL=2 selects the bulk-staged kernel (V = 1 only; measured
+  // slower than the register-staged one on C3-C5)
+  if (V == 1 && env_int("BRO_ELL_KERNEL", 0) == 2 && launch_bro_ell_bulk<T>(A, x, y, st)) return;
+  if (A->ell_max_l <= 4 && env_int("BRO_ELL_SHORT", 1))
+    launch_bro_ell_od<T, V, kEllWarps, sizeof(T) == 8 ? kEllMinBlocksShort - 1 : kEllMinBlocksShort, 4, 6>(A, x, y, st);
+  else
+    launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks>(A, x, y, st);
 }
 
 template <typename T>
@@ -473,7 +484,7 @@ void bro_opts_default(bro_opts_t* o) {
   if (!o) return;
   o->slice_h = 32;
   o->sym_bits = 32;
-  o->vec_words = 4;
+  o->vec_words = 0;
   o->coo_T = 32;
   o->hyb_K = -1;
   o->codec = 1;

@@ -273,14 +273,17 @@ __device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __r
   win[nrows * 32 + lane] = 0u;
 }
 
-template <typename T, int V, int kWarps, int kMinBlocks>
+// G columns per group; kRows window rows per warp (34 holds any 32-column
+// block: <= 33 symbol rows + a zero guard row).  The short-slice instance
+// (G = 4, kRows = 6, 48 warps/SM) serves matrices whose slices all have
+// l <= 4 columns (<= 4 symbols per row): less shared memory and fewer
+// registers buy 1.5x the resident warps for the latency-bound short rows.
+template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
                 const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
                 const uint64_t* __restrict__ symptr, const T* __restrict__ vals,
                 const T* __restrict__ x, T* __restrict__ y) {
-  constexpr int G = 8;
-  constexpr int kRows = 34;
   struct Meta { uint64_t c0, q0; int l, S; };
   __shared__ uint32_t window[kWarps][kRows * 32];
   __shared__ uint2 colmeta[kWarps][32];  // per column of the block: {byte offset of its word row, r | (32-b) << 8}

@@ -92,7 +92,7 @@ class RowBlockSpmv:
     """This rank's block of A as a libbro handle plus the iteration buffers."""
 
     def __init__(self, A, rank: int, world: int, device, fmt="ell", codec=1, dtype=None,
-                 bounds=None, vec_words=4):
+                 bounds=None, vec_words=0):
         import torch
         from .bro import BroMatrix
         self.bounds = np.asarray(bounds if bounds is not None else choose_partition(A.row_ptr, world))

@@ -124,7 +124,8 @@ def test_hyb_split_and_parts_match_oracle_c3(lib):
         ep, ec, ev, cr, cc, cv = hyb.hyb_split(A.row_ptr, A.col, A.vals, K)
         assert info["nnz_ell"] == ec.size and info["nnz_coo"] == cc.size
         assert 0.6 < ec.size / A.nnz < 0.7  # webbase-1M: 64.2% in BRO-ELL (Table 4)
-        E = bro_ell.encode(ep, ec, ev, A.m, A.n, slices=[0, 1, 777, 31250])
+        assert info["vec_words"] == 1  # auto layout for fp64: the paper's multiplexing
+        E = bro_ell.encode(ep, ec, ev, A.m, A.n, V=1, slices=[0, 1, 777, 31250])
         words = lib.bro_export_encoded(h, "ell_words")
         assert np.array_equal(lib.bro_export_encoded(h, "ell_colptr"), E.colptr)
         assert np.array_equal(lib.bro_export_encoded(h, "ell_symptr"), E.symptr)
@@ -133,7 +134,7 @@ def test_hyb_split_and_parts_match_oracle_c3(lib):
             a, b = 32 * int(E.symptr[t]), 32 * int(E.symptr[t + 1])
             assert np.array_equal(words[a:b], E.words[a:b])
         # COO part: sampled intervals through the oracle encoder
-        C = bro_coo.encode(cr[:32 * 1024 * 3], cc[:32 * 1024 * 3], cv[:32 * 1024 * 3])
+        C = bro_coo.encode(cr[:32 * 1024 * 3], cc[:32 * 1024 * 3], cv[:32 * 1024 * 3], V=1)
         cw = lib.bro_export_encoded(h, "coo_words")
         sp = lib.bro_export_encoded(h, "coo_symptr")
         assert np.array_equal(sp[:C.symptr.size], C.symptr)
@@ -171,7 +172,8 @@ def test_c5_sampled_slices_match_oracle(lib):
         assert info["nnz"] == 598**3 and info["n_slices"] == 250000
         sample = [0, 1, 6249, 6250, 124999, 187500, 249999]
         sub = row_block(A, 0, A.m)
-        E = bro_ell.encode(sub.row_ptr, sub.col, sub.vals, A.m, A.n, slices=sample)
+        assert info["vec_words"] == 1
+        E = bro_ell.encode(sub.row_ptr, sub.col, sub.vals, A.m, A.n, V=1, slices=sample)
         assert np.array_equal(lib.bro_export_encoded(h, "ell_colptr"), E.colptr)
         assert np.array_equal(lib.bro_export_encoded(h, "ell_symptr"), E.symptr)
         words = lib.bro_export_encoded(h, "ell_words")
@@ -268,7 +270,7 @@ def test_forced_widths_bytes_match_oracle(lib, min_bits):
                  ("ell_words", "ell_bit_alloc", "ell_colptr", "ell_symptr", "ell_vals")}
     finally:
         lib.bro_destroy(h)
-    E = bro_ell.encode(A.row_ptr, A.col, A.vals, A.m, A.n, min_bits=min_bits)
+    E = bro_ell.encode(A.row_ptr, A.col, A.vals, A.m, A.n, V=1, min_bits=min_bits)  # auto V for fp64
     _assert_ell_equal(parts, E)
     assert bro_ell.decode(E) == [A.col[A.row_ptr[i]:A.row_ptr[i + 1]].tolist() for i in range(A.m)]
 
