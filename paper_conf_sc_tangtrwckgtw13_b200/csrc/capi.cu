@@ -312,10 +312,10 @@ bro_status_t common_checks(bro_dtype_t dtype, const bro_opts_t* opts, bro_opts_t
 
 // Persistent grid: as many resident blocks as the SMs hold (queried once per
 // instantiation), capped by the number of slices.
-template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34>
+template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34, bool kPf = false>
 void launch_bro_ell_od(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   using namespace bro::dev;
-  auto kern = bro_ell_spmv_od<T, V, kWarps, kMinBlocks, G, kRows>;
+  auto kern = bro_ell_spmv_od<T, V, kWarps, kMinBlocks, G, kRows, kPf>;
   static int resident = 0;
   if (resident == 0) {
     int per_sm = 0, sms = 0, dev = 0;
@@ -389,7 +389,14 @@ void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   // BRO_ELL_KERNEL=2 selects the bulk-staged kernel (V = 1 only; measured
   // slower than the register-staged one on C3-C5)
   if (V == 1 && env_int("BRO_ELL_KERNEL", 0) == 2 && launch_bro_ell_bulk<T>(A, x, y, st)) return;
-  if (A->ell_max_l <= 4 && env_int("BRO_ELL_SHORT", 1))
+  const int variant = env_int("BRO_ELL_VARIANT", 0);  // tuning sweeps only
+  if (variant == 1)
+    launch_bro_ell_od<T, V, kEllWarps, 5, 4, 34>(A, x, y, st);
+  else if (variant == 2)
+    launch_bro_ell_od<T, V, kEllWarps, 3, 8, 34>(A, x, y, st);
+  else if (variant == 3)
+    launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks, 8, 34, true>(A, x, y, st);
+  else if (A->ell_max_l <= 4 && env_int("BRO_ELL_SHORT", 1))
     launch_bro_ell_od<T, V, kEllWarps, sizeof(T) == 8 ? kEllMinBlocksShort - 1 : kEllMinBlocksShort, 4, 6>(A, x, y, st);
   else
     launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks>(A, x, y, st);
