@@ -229,12 +229,6 @@ __device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
   asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(p), "r"(bytes) : "memory");
 }
 
-__device__ __forceinline__ void cp_async4(void* smem_dst, const void* gsrc) {
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" :: "r"(smem_u32(smem_dst)), "l"(gsrc) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
-
 __device__ __forceinline__ void prefetch_l2_line(const void* p) {
   asm volatile("prefetch.global.L2 [%0];" :: "l"(p));
 }
@@ -304,9 +298,6 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
   const uint2* cm = colmeta[w];
   const char* win_lane = reinterpret_cast<const char*>(win + lane);
   const int64_t stride = int64_t(gridDim.x) * kWarps;
-  __shared__ uint32_t wpf[kWarps][kPf ? 16 : 1];  // prefetched widths (4-byte words of bit_alloc)
-  bool pre = false;
-  int pre_off = 0;
   int k32 = 0;
   for (int64_t t = int64_t(blockIdx.x) * kWarps + w; t < s; t += stride, k32 = (k32 + 1) & 31) {
     __syncwarp();
@@ -319,13 +310,15 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
       __syncwarp();
     }
     const Meta mt = metas[w][k32];
-    const bool have = pre;  // block 0 of this slice (widths + symbols) was prefetched
-    if constexpr (kPf) {
-      if (have) {
-        cp_async_wait_all();
-        __syncwarp();
+    if constexpr (kPf) {  // L2 prefetch of the warp's next slice (values, symbols, widths)
+      if (k32 < 31 && t + stride < s) {
+        const Meta nx = metas[w][k32 + 1];
+        const int vlines = (nx.l * int(sizeof(T)) + 3) / 4;  // 128-byte lines of 32*l values
+        const char* vb = reinterpret_cast<const char*>(vals + 32 * nx.c0);
+        for (int i = lane; i < vlines; i += 32) prefetch_l2_line(vb + 128 * i);
+        if (lane < nx.S) prefetch_l2_line(words + 32 * (nx.q0 + lane));
+        if (lane == 31) prefetch_l2_line(bit_alloc + nx.c0);
       }
-      pre = false;
     }
     const uint64_t c0 = mt.c0;
     const int l = mt.l;
@@ -339,15 +332,10 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
     int obase = 0;  // bit offset of the current block inside every row stream
     for (int jb = 0; jb < l; jb += 32) {
       const int nb = min(32, l - jb);
-      int b;
-      if (kPf && jb == 0 && have) {
-        b = lane < nb ? int(reinterpret_cast<const uint8_t*>(wpf[w])[pre_off + lane]) : 0;
-      } else {
-        b = lane < nb ? int(__ldg(ba + jb + lane)) : 0;
-        if (jb == 0) {  // first block starts at symbol 0: stage without waiting for the scan
-          __syncwarp();
-          stage_symbols<V>(win, wb, S, 0, min(S, kRows - 1), lane);
-        }
+      const int b = lane < nb ? int(__ldg(ba + jb + lane)) : 0;
+      if (jb == 0) {  // first block starts at symbol 0: stage without waiting for the scan
+        __syncwarp();
+        stage_symbols<V>(win, wb, S, 0, min(S, kRows - 1), lane);
       }
       int incl = b;  // inclusive scan of the widths over the block
 #pragma unroll
@@ -386,24 +374,6 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
 #pragma unroll
         for (int k = 0; k < G; ++k)
           if (ok[k]) xv[k] = ldg_x(x + cidx[k]);
-        if constexpr (kPf) {
-          // last decode of the slice done: stage block 0 of the warp's next
-          // slice (widths + symbol rows) with async copies, so that round
-          // trip overlaps this group's value / x loads
-          if (jb + g + G >= l && k32 < 31 && t + stride < s) {
-            const Meta nx = metas[w][k32 + 1];
-            __syncwarp();
-            const int nw = (int(nx.c0 & 3) + min(nx.l, 32) + 3) >> 2;
-            if (lane < nw) cp_async4(&wpf[w][lane], bit_alloc + (nx.c0 & ~uint64_t(3)) + 4 * lane);
-            const int nr = min(nx.S, kRows - 1);
-            const uint32_t* wbn = words + 32 * nx.q0;
-            for (int r = 0; r < nr; ++r) cp_async4(win + r * 32 + lane, wbn + place(lane, r, nx.S, V));
-            win[nr * 32 + lane] = 0u;
-            cp_async_commit();
-            pre = true;
-            pre_off = int(nx.c0 & 3);
-          }
-        }
 #pragma unroll
         for (int k = 0; k < G; ++k)
           if (ok[k]) sum = fma(v[k], xv[k], sum);  // padding slots (delta 0) are skipped, Alg. 1 line 17

@@ -95,22 +95,6 @@ def test_bro_ell_v1_kernels(lib, dev, kernel, ring_kb, dtype, monkeypatch):
             M.close()
 
 
-@pytest.mark.parametrize("variant", ["1", "2", "3"])
-@pytest.mark.parametrize("V", [1, 4])
-@pytest.mark.parametrize("dtype", [np.float64, np.float32])
-def test_bro_ell_tuning_variants(lib, dev, variant, V, dtype, monkeypatch):
-    """Every instance of the register-staged BRO-ELL kernel (G = 4 at 40
-    warps/SM, 80-register G = 8, next-slice cp.async staging of widths and
-    symbols) gives the oracle's y."""
-    monkeypatch.setenv("BRO_ELL_VARIANT", variant)
-    for _, mk in BULK_CASES:
-        A = mk()
-        for fmt in ("ell", "hyb"):
-            M, x, y = _run(lib, A, fmt, 1, dtype, dev, V=V)
-            _check_y(A, x, y, dtype)
-            M.close()
-
-
 @pytest.mark.parametrize("short", ["0", "1"])
 @pytest.mark.parametrize("V", [1, 2, 4])
 @pytest.mark.parametrize("dtype", [np.float64, np.float32])
