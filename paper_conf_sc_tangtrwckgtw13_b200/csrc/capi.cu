@@ -312,10 +312,10 @@ bro_status_t common_checks(bro_dtype_t dtype, const bro_opts_t* opts, bro_opts_t
 
 // Persistent grid: as many resident blocks as the SMs hold (queried once per
 // instantiation), capped by the number of slices.
-template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34, bool kPf = false>
+template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34>
 void launch_bro_ell_od(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   using namespace bro::dev;
-  auto kern = bro_ell_spmv_od<T, V, kWarps, kMinBlocks, G, kRows, kPf>;
+  auto kern = bro_ell_spmv_od<T, V, kWarps, kMinBlocks, G, kRows>;
   static int resident = 0;
   if (resident == 0) {
     int per_sm = 0, sms = 0, dev = 0;
@@ -394,8 +394,6 @@ void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
     launch_bro_ell_od<T, V, kEllWarps, 5, 4, 34>(A, x, y, st);
   else if (variant == 2)
     launch_bro_ell_od<T, V, kEllWarps, 3, 8, 34>(A, x, y, st);
-  else if (variant == 3)
-    launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks, 8, 34, true>(A, x, y, st);
   else if (A->ell_max_l <= 4 && env_int("BRO_ELL_SHORT", 1))
     launch_bro_ell_od<T, V, kEllWarps, sizeof(T) == 8 ? kEllMinBlocksShort - 1 : kEllMinBlocksShort, 4, 6>(A, x, y, st);
   else

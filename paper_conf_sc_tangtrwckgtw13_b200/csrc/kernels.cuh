@@ -282,7 +282,7 @@ __device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __r
 // (G = 4, kRows = 6, 48 warps/SM) serves matrices whose slices all have
 // l <= 4 columns (<= 4 symbols per row): less shared memory and fewer
 // registers buy 1.5x the resident warps for the latency-bound short rows.
-template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34, bool kPf = false>
+template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
                 const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
@@ -310,16 +310,6 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
       __syncwarp();
     }
     const Meta mt = metas[w][k32];
-    if constexpr (kPf) {  // L2 prefetch of the warp's next slice (values, symbols, widths)
-      if (k32 < 31 && t + stride < s) {
-        const Meta nx = metas[w][k32 + 1];
-        const int vlines = (nx.l * int(sizeof(T)) + 3) / 4;  // 128-byte lines of 32*l values
-        const char* vb = reinterpret_cast<const char*>(vals + 32 * nx.c0);
-        for (int i = lane; i < vlines; i += 32) prefetch_l2_line(vb + 128 * i);
-        if (lane < nx.S) prefetch_l2_line(words + 32 * (nx.q0 + lane));
-        if (lane == 31) prefetch_l2_line(bit_alloc + nx.c0);
-      }
-    }
     const uint64_t c0 = mt.c0;
     const int l = mt.l;
     const int S = mt.S;
