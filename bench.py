@@ -48,6 +48,8 @@ def parse_args():
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--workload", default="C5", choices=sorted(WORKLOADS))
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
+    ap.add_argument("--format", default=None, choices=["ell", "hyb", "coo"],
+                    help="override the workload's format (e.g. coo: standalone BRO-COO vs COO, Fig. 7)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--vec-words", type=int, default=0, help="0 = auto (fp64: 1, fp32: 4)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -246,6 +248,7 @@ def main():
     tdt = torch.float64 if dtype == np.float64 else torch.float32
     cfg, fmt = WORKLOADS[args.workload]
     A, fmt = load_workload(args.workload, dtype, P)
+    fmt = args.format or fmt
     x_host = make_x(A.n, cfg, dtype)
     bounds = choose_partition(A.row_ptr, world)
     stream = torch.cuda.current_stream(dev)
@@ -255,7 +258,7 @@ def main():
                        vec_words=args.vec_words)
     base = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=0, dtype=dtype, bounds=bounds)
     info, binfo = blk.mat.info, base.mat.info
-    launches = 1 if info["nnz_coo"] == 0 else 3  # ELL kernel (+ COO kernel + fix-up)
+    launches = (0 if fmt == "coo" else 1) + (2 if info["nnz_coo"] else 0)  # ELL kernel, COO kernel + fix-up
     flush_buf = torch.empty(2 * L2_BYTES // 4, dtype=torch.int32, device=dev) if args.flush_l2 else None
     flush = (lambda: flush_buf.fill_(1)) if args.flush_l2 else None
 
@@ -293,6 +296,20 @@ def main():
                                             stream, flush)))
     if world > 1:
         total_ms, base_ms = max_over_ranks([total_ms, base_ms], dev, args.dist_backend)
+
+    # --- launch latency: the same bro_spmv captured once in a CUDA graph and
+    # replayed (the CG-loop form; matters for the small, L2-resident C1/C2)
+    graph = None
+    if world == 1:
+        g = torch.cuda.CUDAGraph()
+        blk.spmv(x, stream)
+        torch.cuda.synchronize()
+        with torch.cuda.graph(g):
+            blk.spmv(x, None)
+        g_ms = time_steps(g.replay, min(args.steps, 500), 3, stream, flush)
+        graph = {"us_per_call": float(np.median(g_ms)) * 1e3,
+                 "p10_us": float(np.percentile(g_ms, 10)) * 1e3, "p90_us": float(np.percentile(g_ms, 90)) * 1e3,
+                 "gflops": 2.0 * A.nnz / (float(np.median(g_ms)) * 1e-3) / 1e9}
 
     # --- end to end through the C ABI with pinned host buffers (rank 0 / N=1 path)
     e2e = None
@@ -368,7 +385,8 @@ def main():
                      "frac": achieved / peak, "traffic": traffic,
                      "peak_kind": peak_kind,
                      "kernel": f"bro_ell_spmv_od<{'double' if dtype == np.float64 else 'float'},V={info['vec_words']}>"
-                     if fmt == "ell" else "bro_ell_spmv + coo_spmv + coo_fixup",
+                     if fmt == "ell" else ("coo_spmv + coo_fixup" if fmt == "coo" else
+                                           "bro_ell_spmv + coo_spmv + coo_fixup"),
                      "algorithmic_bytes_per_launch": alg_bytes, "kernel_ms": kern_ms,
                      "frac_of_8TBps_spec": achieved / 8000.0},
         "uncompressed": {"format": {"ell": "ELLPACK", "hyb": "HYB", "coo": "COO"}[fmt], "value": base_value,
@@ -376,6 +394,8 @@ def main():
                          "algorithmic_bytes": binfo["algorithmic_bytes"],
                          "achieved_GBps": binfo["algorithmic_bytes"] / (base_kern_ms * 1e-3) / 1e9,
                          "speedup_bro": value / base_value},
+        "step_ms_p10_p50_p90": [float(np.percentile(per_step, q)) for q in (10, 50, 90)],
+        "cuda_graph": graph,
         "gpu_launches": int(launches * args.steps),
         "clocks": ck,
         "cpu_baseline": cpu,
