@@ -202,7 +202,11 @@ bro_status_t bro_hyb_K(int64_t m, const int64_t* row_ptr, int64_t* K_out);
  * row length then by the bit-width signature of the row's deltas, O(nnz log m));
  * method 1 = Algorithm 2 greedy on Eqn. (1) with h = w = 32, alpha = sym_len = 32 and
  * Omega(c) = 128-byte line of x[c] for the dtype (O(m^2 k / h); m <= 65536,
- * else BRO_ERR_UNSUPPORTED).  Partitions hold 32 rows except the last. */
+ * else BRO_ERR_UNSUPPORTED);
+ * method 2 = Algorithm 2 with a candidate window (reading R24): line 11's
+ * argmin runs over the 64 non-full partitions nearest to the row's own partition
+ * floor(pos/32) in length-sorted order (O(m k W), any m; W >= v would equal method 1).
+ * Partitions hold 32 rows except the last. */
 bro_status_t bro_reorder_bar(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
                              bro_dtype_t dtype, int32_t method, int64_t* perm_out);
 

@@ -59,13 +59,29 @@ def phi(partitions, row_ptr, col, h=32, w=32, alpha=32, vsize=8):
         k = max((len(c) for c in rows_cols), default=0)
         dsum = sum(d_term(rows_cols, j) for j in range(k))
         csum = sum(c_term(rows_cols, j, vsize) for j in range(k))
-        total += (h // w) * (math.ceil(dsum / alpha) + csum)
+        total += h / w * (math.ceil(dsum / alpha) + csum)
     return total
 
 
-def algorithm2(row_ptr, col, m, h=32, alpha=32, vsize=8):
+def window_candidates(pos, sizes, cap, h, W):
+    """Reading R24 (method 2): the W non-full partitions nearest to the row's
+    own partition c = min(pos // h, v - 1) of the sorted sequence, ordered by
+    |p - c| then p."""
+    v = len(cap)
+    c = min(pos // h, v - 1)
+    free = [p for p in range(v) if sizes[p] < cap[p]]
+    free.sort(key=lambda p: (abs(p - c), p))
+    return free[:W]
+
+
+def algorithm2(row_ptr, col, m, h=32, alpha=32, vsize=8, window=None, w=None):
     """Algorithm 2, evaluating the full Phi_m of line 9 for every
-    candidate partition.  Returns the permutation S_1 ++ S_2 ++ ... ."""
+    candidate partition.  Returns the permutation S_1 ++ S_2 ++ ... .
+    window=W restricts line 11 to window_candidates (reading R24); None is
+    the paper's algorithm (every non-full partition).  w (warp size, w | h)
+    defaults to h: the factor h/w multiplies every partition's term alike and
+    cannot change line 11's argmin (reading R21)."""
+    w = h if w is None else w
     row_ptr = np.asarray(row_ptr, dtype=np.int64)
     if m == 0:
         return np.zeros(0, dtype=np.int64)
@@ -78,14 +94,20 @@ def algorithm2(row_ptr, col, m, h=32, alpha=32, vsize=8):
     for t in range(v):                                           # lines 3-6
         S[t].append(D[t * h])
         seeds.add(t * h)
-    rest = [D[p] for p in range(m) if p not in seeds]
-    for r in rest:                                               # line 7
-        costs = []
-        for mm in range(v):                                      # lines 8-10
+    for pos in range(m):                                         # line 7
+        if pos in seeds:
+            continue
+        r = D[pos]
+        if window is None:
+            cands = list(range(v))
+        else:
+            cands = window_candidates(pos, [len(St) for St in S], cap, h, window)
+        costs = {}
+        for mm in cands:                                         # lines 8-10
             trial = [S[t] + [r] if t == mm else S[t] for t in range(v)]
-            costs.append(phi(trial, row_ptr, col, h, 32, alpha, vsize))
+            costs[mm] = phi(trial, row_ptr, col, h, w, alpha, vsize)
         best = None
-        for p in range(v):                                       # line 11
+        for p in sorted(cands):                                  # line 11
             if len(S[p]) < cap[p] and (best is None or costs[p] < costs[best]):
                 best = p
         S[best].append(r)                                        # line 12

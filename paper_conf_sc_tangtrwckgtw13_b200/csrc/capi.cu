@@ -22,6 +22,7 @@ bro_status_t fail(bro_status_t s, const std::string& msg) {
 }
 
 constexpr int kCooThreads = 256;
+constexpr int kBarWindow = 64;  // candidate partitions of BAR method 2 (windowed Algorithm 2)
 constexpr int kCooMaxUpi = 4;   // work units per COO interval (8 steps = 256 entries each at 4)
 constexpr int kCooUpi = 2;
 constexpr int kPlainThreads = 256;
@@ -662,6 +663,11 @@ bro_status_t bro_reorder_bar(int64_t m, int64_t n, const int64_t* row_ptr, const
       bro::bar_signature_order(m, row_ptr, col_idx, perm_out);
       return BRO_OK;
     }
+    if (method == 2) {
+      bro::bar_window_order(m, row_ptr, col_idx, dtype == BRO_FP64 ? 8 : 4, env_int("BRO_BAR_WINDOW", kBarWindow),
+                            perm_out);
+      return BRO_OK;
+    }
     if (method == 1) {
       std::string err;
       if (!bro::bar_greedy_order(m, n, row_ptr, col_idx, dtype == BRO_FP64 ? 8 : 4, perm_out, &err))
@@ -671,7 +677,7 @@ bro_status_t bro_reorder_bar(int64_t m, int64_t n, const int64_t* row_ptr, const
   } catch (const std::bad_alloc&) {
     return fail(BRO_ERR_OOM, "host allocation failed");
   }
-  return fail(BRO_ERR_ARG, "method must be 0 or 1");
+  return fail(BRO_ERR_ARG, "method must be 0, 1 or 2");
 }
 
 const char* bro_status_str(bro_status_t s) {

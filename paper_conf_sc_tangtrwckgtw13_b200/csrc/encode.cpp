@@ -421,3 +421,131 @@ bool bar_greedy_order(int64_t m, int64_t n, const int64_t* row_ptr, const int32_
 }
 
 }  // namespace bro
+
+namespace bro {
+
+// Method 2: Algorithm 2 with a candidate window (reading R24), for
+// matrices too large for the O(m^2 k / h) exact greedy.  Lines 1-6 as in
+// method 1.  For the row at position pos of the sorted sequence D, line 11's
+// argmin runs only over the W non-full partitions nearest to the row's own
+// partition c = min(pos / h, v - 1) (nearest by |p - c|, equal distance ->
+// lower p); cost ties -> lowest p.  With W >= v every non-full partition is a
+// candidate and the result is exactly method 1.  Per partition: the column
+// widths d(S, j) (Eqn 2) and the distinct x lines of each column (Eqn 3, at
+// most h per column), grown to the partition's longest row.  Full partitions
+// are skipped with two path-compressed "next non-full" forests.
+bool bar_window_order(int64_t m, const int64_t* row_ptr, const int32_t* col, int vsize, int W,
+                      int64_t* perm) {
+  const int64_t h = kH;
+  if (m == 0) return true;
+  if (W < 1) W = 1;
+  const int64_t v = (m + h - 1) / h;
+  auto cap = [&](int64_t p) { return p < v - 1 ? h : m - (v - 1) * h; };
+  struct Part {
+    std::vector<uint8_t> d;      // d(S, j)
+    std::vector<uint8_t> nl;     // distinct lines in column j
+    std::vector<int32_t> lines;  // column j's lines at [32 j, 32 j + nl[j])
+    int64_t dsum = 0;
+    int size = 0;
+  };
+  std::vector<Part> P(v);
+  std::vector<std::vector<int64_t>> S(v);
+  std::vector<int> g;       // the current row's Gamma(delta_j)
+  std::vector<int32_t> ln;  // the current row's x lines
+  auto load_row = [&](int64_t i) {
+    const int64_t len = row_ptr[i + 1] - row_ptr[i];
+    g.resize(len);
+    ln.resize(len);
+    uint32_t prev = 0;
+    for (int64_t j = 0; j < len; ++j) {
+      const uint32_t c1 = uint32_t(col[row_ptr[i] + j]) + 1u;
+      g[j] = gamma_bits(c1 - prev);
+      prev = c1;
+      ln[j] = int32_t(int64_t(col[row_ptr[i] + j]) * vsize / 128);
+    }
+    return len;
+  };
+  auto has_line = [&](const Part& q, int64_t j, int32_t L) {
+    const int32_t* a = q.lines.data() + 32 * j;
+    for (int k = 0; k < q.nl[j]; ++k)
+      if (a[k] == L) return true;
+    return false;
+  };
+  auto insert = [&](int64_t p, int64_t i) {
+    const int64_t len = load_row(i);
+    Part& q = P[p];
+    if ((int64_t)q.d.size() < len) {
+      q.d.resize(len, 0);
+      q.nl.resize(len, 0);
+      q.lines.resize(32 * len, 0);
+    }
+    for (int64_t j = 0; j < len; ++j) {
+      if (g[j] > q.d[j]) { q.dsum += g[j] - q.d[j]; q.d[j] = (uint8_t)g[j]; }
+      if (!has_line(q, j, ln[j])) q.lines[32 * j + q.nl[j]++] = ln[j];
+    }
+    q.size++;
+    S[p].push_back(i);
+  };
+  // next non-full partition at or right of p (v if none) / at or left of p (-1 if none)
+  std::vector<int64_t> rpar(v + 1), lpar(v + 1);
+  std::iota(rpar.begin(), rpar.end(), 0);
+  std::iota(lpar.begin(), lpar.end(), 0);  // lpar index shifted by one: slot p + 1 <-> partition p
+  auto rfind = [&](int64_t p) {
+    int64_t r = p;
+    while (rpar[r] != r) r = rpar[r];
+    while (rpar[p] != r) { int64_t nx = rpar[p]; rpar[p] = r; p = nx; }
+    return r;
+  };
+  auto lfind = [&](int64_t p) {  // p in [-1, v)
+    int64_t s = p + 1, r = s;
+    while (lpar[r] != r) r = lpar[r];
+    while (lpar[s] != r) { int64_t nx = lpar[s]; lpar[s] = r; s = nx; }
+    return r - 1;
+  };
+  auto mark_full = [&](int64_t p) { rpar[p] = p + 1; lpar[p + 1] = p; };
+  // line 2
+  std::vector<int64_t> D(m);
+  std::iota(D.begin(), D.end(), 0);
+  std::stable_sort(D.begin(), D.end(), [&](int64_t a, int64_t b) {
+    return row_ptr[a + 1] - row_ptr[a] < row_ptr[b + 1] - row_ptr[b];
+  });
+  // lines 3-6
+  for (int64_t t = 0; t < v; ++t) {
+    insert(t, D[t * h]);
+    if (P[t].size >= cap(t)) mark_full(t);
+  }
+  const int64_t alpha = kSym;
+  std::vector<int64_t> cand;
+  for (int64_t pos = 0; pos < m; ++pos) {
+    if (pos % h == 0) continue;  // a seed
+    const int64_t i = D[pos];
+    const int64_t len = load_row(i);
+    const int64_t c = std::min(pos / h, v - 1);
+    cand.clear();
+    int64_t r = rfind(c), l = lfind(c - 1);
+    while ((int64_t)cand.size() < W && (l >= 0 || r < v)) {
+      if (l >= 0 && (r >= v || c - l <= r - c)) { cand.push_back(l); l = lfind(l - 1); }
+      else { cand.push_back(r); r = rfind(r + 1); }
+    }
+    int64_t best = -1, bestc = 0;
+    for (int64_t p : cand) {
+      const Part& q = P[p];
+      int64_t nd = q.dsum, dc = 0;
+      for (int64_t j = 0; j < len; ++j) {
+        const int dj = j < (int64_t)q.d.size() ? q.d[j] : 0;
+        if (g[j] > dj) nd += g[j] - dj;
+        if (j >= (int64_t)q.d.size() || !has_line(q, j, ln[j])) dc++;
+      }
+      const int64_t delta = (nd + alpha - 1) / alpha - (q.dsum + alpha - 1) / alpha + dc;
+      if (best < 0 || delta < bestc || (delta == bestc && p < best)) { best = p; bestc = delta; }
+    }
+    insert(best, i);
+    if (P[best].size >= cap(best)) mark_full(best);
+  }
+  int64_t k = 0;
+  for (int64_t p = 0; p < v; ++p)
+    for (int64_t i : S[p]) perm[k++] = i;
+  return true;
+}
+
+}  // namespace bro

@@ -287,3 +287,34 @@ def test_dense_band_eta_closed_form(lib):
         finally:
             lib.bro_destroy(h)
         assert info["eta_stream"] == pytest.approx(1 - b / 32)
+
+
+@pytest.mark.parametrize("seed,m", [(3, None), (4, 300)])
+def test_bar_window_matches_oracle(lib, seed, m, monkeypatch):
+    """Method 2 (Algorithm 2 with a candidate window, reading R24; window
+    forced to 8 through the library's tuning variable) == the oracle's
+    transcription with window=8; 10 partitions, so the window excludes some
+    (and h does not divide m in the second case)."""
+    monkeypatch.setenv("BRO_BAR_WINDOW", "8")
+    A = random_block(seed=seed, families=10, fam_rows=32)
+    if m is not None:
+        A = row_block(A, 0, m)
+    perm = lib.bro_reorder_bar(A.m, A.n, A.row_ptr, A.col, method=2)
+    assert np.array_equal(perm, bar.algorithm2(A.row_ptr, A.col, A.m, h=32, window=8))
+
+
+def test_bar_window_improves_eta_over_scrambled(lib):
+    """On scrambled random-block rows (C4's generator at 1/100 size) the
+    windowed greedy recovers compressibility: eta_stream of BRO-ELL rises."""
+    from gen import permute_rows
+    A = random_block(seed=11, families=625, fam_rows=32)
+    etas = {}
+    for name, method in (("scrambled", None), ("m0", 0), ("m2", 2)):
+        B = A if method is None else permute_rows(A, lib.bro_reorder_bar(A.m, A.n, A.row_ptr, A.col,
+                                                                          method=method))
+        h = lib.bro_create_ell(HOST, B.m, B.n, B.row_ptr, B.col, B.vals)
+        try:
+            etas[name] = lib.bro_get_info(h)["eta_stream"]
+        finally:
+            lib.bro_destroy(h)
+    assert etas["m2"] > etas["scrambled"] + 0.05, etas
