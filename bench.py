@@ -377,7 +377,7 @@ def main():
             "format": bro_name, "m": A.m, "n": A.n, "nnz": A.nnz,
             "vec_words": info["vec_words"],
             "l2": ("flushed (2x L2 write) before every step" if args.flush_l2 else
-                   ("inputs larger than L2" if alg_bytes > 2 * L2_BYTES else "L2-resident (warm)")),
+                   ("inputs larger than L2" if alg_bytes > L2_BYTES else "L2-resident (warm)")),
             "parallelism": f"row-block x{world}" + (" + NCCL allgather of y per step" if world > 1 else ""),
             "eta_stream": info["eta_stream"], "eta_total": info["eta_total"],
         },
