@@ -676,8 +676,16 @@ __device__ __forceinline__ void load8_s32(int* d, const int32_t* p) {
   d[4] = int(b.x); d[5] = int(b.y); d[6] = int(b.z); d[7] = int(b.w);
 }
 
+// delta of step t in a lane stream of b-bit fields staged as [row][lane]
+// (wl points at the lane's word of row 0); 0 when b = 0 (empty stream).
+__device__ __forceinline__ int coo_delta(const uint32_t* wl, int t, int b) {
+  const int o = t * b;
+  const uint32_t* p = wl + 32 * (o >> 5);
+  return int(shr_clamp(__funnelshift_l(p[32], p[0], uint32_t(o & 31)), uint32_t(32 - b)));
+}
+
 template <typename T, int V, bool kBro, int kThreads>
-__global__ void __launch_bounds__(kThreads)
+__global__ void __launch_bounds__(kThreads, 1024 / kThreads)
 coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restrict__ words,
          const uint32_t* __restrict__ base_row, const uint8_t* __restrict__ width,
          const uint64_t* __restrict__ symptr, const int32_t* __restrict__ rows,
@@ -686,6 +694,7 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restri
          int32_t* __restrict__ first_row, int32_t* __restrict__ last_row) {
   constexpr int TB = 8;
   __shared__ __align__(16) int32_t rowbuf[kThreads / 32][TB * 32];
+  __shared__ uint32_t cwin[kThreads / 32][kBro ? 33 * 32 : 1];  // lane word rows (+ zero guard row)
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
   // work unit = steps [ts, ts + T_steps / upi) of interval i (upi units per interval)
@@ -707,13 +716,21 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restri
   }
   int row = (int)base_row[i];
   int b = 0;
-  LaneStream<V> ls;
+  const uint32_t* wn = nullptr;
   if constexpr (kBro) {
+    // One width per interval, so the bit offset of step t is t*b in
+    // every lane stream: stage the words the unit needs (rows [0, q_hi]) in
+    // a per-warp [row][lane] window and extract each delta branch-free,
+    //   delta_t = funnelshift(w[q+1], w[q], o mod 32) >> (32 - b),  o = t*b.
     b = width[i];
     const uint64_t q0 = symptr[i];
-    ls.init(words + 32 * q0, int(symptr[i + 1] - q0), lane);
-    if (b)
-      for (int t = 0; t < ts; ++t) row += (int)ls.get(b, lane);  // rows of the steps before the unit
+    const int S = int(symptr[i + 1] - q0);
+    const int nrows = b ? min(S, (((ts + steps) * b - 1) >> 5) + 1) : 0;
+    uint32_t* wnw = cwin[w];
+    stage_symbols<V>(wnw, words + 32 * q0, S, 0, nrows, lane);
+    __syncwarp();
+    wn = wnw + lane;
+    for (int t = 0; t < ts; ++t) row += coo_delta(wn, t, b);  // rows of the steps before the unit
   }
   // row of the unit's first entry (element (ts, 0))
   int first = 0;
@@ -738,7 +755,7 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restri
     if constexpr (kBro) {
 #pragma unroll
       for (int k = 0; k < TB; ++k) {  // decode rows of steps t0..t0+7 for (t, lane)
-        if (b) row += (int)ls.get(b, lane);
+        row += coo_delta(wn, t0 + k, b);
         rb[k * 32 + lane] = row;
       }
       __syncwarp();
