@@ -685,7 +685,7 @@ __device__ __forceinline__ int coo_delta(const uint32_t* wl, int t, int b) {
 }
 
 template <typename T, int V, bool kBro, int kThreads>
-__global__ void __launch_bounds__(kThreads, 1024 / kThreads)
+__global__ void __launch_bounds__(kThreads)
 coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restrict__ words,
          const uint32_t* __restrict__ base_row, const uint8_t* __restrict__ width,
          const uint64_t* __restrict__ symptr, const int32_t* __restrict__ rows,
@@ -715,23 +715,8 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restri
     }
   }
   int row = (int)base_row[i];
-  int b = 0;
-  const uint32_t* wn = nullptr;
-  if constexpr (kBro) {
-    // One width per interval, so the bit offset of step t is t*b in
-    // every lane stream: stage the words the unit needs (rows [0, q_hi]) in
-    // a per-warp [row][lane] window and extract each delta branch-free,
-    //   delta_t = funnelshift(w[q+1], w[q], o mod 32) >> (32 - b),  o = t*b.
-    b = width[i];
-    const uint64_t q0 = symptr[i];
-    const int S = int(symptr[i + 1] - q0);
-    const int nrows = b ? min(S, (((ts + steps) * b - 1) >> 5) + 1) : 0;
-    uint32_t* wnw = cwin[w];
-    stage_symbols<V>(wnw, words + 32 * q0, S, 0, nrows, lane);
-    __syncwarp();
-    wn = wnw + lane;
-    for (int t = 0; t < ts; ++t) row += coo_delta(wn, t, b);  // rows of the steps before the unit
-  }
+  const int b = kBro ? int(width[i]) : 0;
+  const uint32_t* wn = cwin[w] + lane;
   // row of the unit's first entry (element (ts, 0))
   int first = 0;
   if constexpr (!kBro) first = rows[min(e0 + 32 * ts, nnz - 1)];
@@ -752,7 +737,37 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restri
     const int64_t el = eb + TB * lane;          // this lane's first entry (transposed)
     int r[TB], c[TB];
     T v[TB];
+    // col / vals (and plain rows) of the batch first: they do not depend on
+    // the row decode, so their round trip overlaps it
+    if (el + TB <= nnz) {
+      if constexpr (!kBro) load8_s32(r, rows + el);
+      load8_s32(c, col + el);
+      Vec8<T> vv;
+      vv.load(vals + el);
+#pragma unroll
+      for (int k = 0; k < TB; ++k) v[k] = vv.v[k];
+    } else {  // tail of the last interval: entries past nnz repeat the last row with value 0
+#pragma unroll
+      for (int k = 0; k < TB; ++k) {
+        const bool ok = el + k < nnz;
+        if constexpr (!kBro) r[k] = ld_stream_s32(rows + (ok ? el + k : nnz - 1));
+        c[k] = ok ? ld_stream_s32(col + el + k) : -1;
+        v[k] = ok ? ld_stream(vals + el + k) : T(0);
+      }
+    }
     if constexpr (kBro) {
+      if (t0 == ts) {
+        // One width per interval, so the bit offset of step t is t*b
+        // in every lane stream: stage the words the unit needs (rows
+        // [0, q_hi]) in a per-warp [row][lane] window and extract each delta
+        // branch-free: delta_t = funnelshift(w[q+1], w[q], o mod 32) >> (32 - b), o = t*b.
+        const uint64_t q0 = symptr[i];
+        const int S = int(symptr[i + 1] - q0);
+        const int nrows = b ? min(S, (((ts + steps) * b - 1) >> 5) + 1) : 0;
+        stage_symbols<V>(cwin[w], words + 32 * q0, S, 0, nrows, lane);
+        __syncwarp();
+        for (int t = 0; t < ts; ++t) row += coo_delta(wn, t, b);  // rows of the steps before the unit
+      }
 #pragma unroll
       for (int k = 0; k < TB; ++k) {  // decode rows of steps t0..t0+7 for (t, lane)
         row += coo_delta(wn, t0 + k, b);
@@ -769,22 +784,6 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restri
         first_pending = false;
       }
       __syncwarp();
-    }
-    if (el + TB <= nnz) {
-      if constexpr (!kBro) load8_s32(r, rows + el);
-      load8_s32(c, col + el);
-      Vec8<T> vv;
-      vv.load(vals + el);
-#pragma unroll
-      for (int k = 0; k < TB; ++k) v[k] = vv.v[k];
-    } else {  // tail of the last interval: entries past nnz repeat the last row with value 0
-#pragma unroll
-      for (int k = 0; k < TB; ++k) {
-        const bool ok = el + k < nnz;
-        if constexpr (!kBro) r[k] = ld_stream_s32(rows + (ok ? el + k : nnz - 1));
-        c[k] = ok ? ld_stream_s32(col + el + k) : -1;
-        v[k] = ok ? ld_stream(vals + el + k) : T(0);
-      }
     }
     T xv[TB];
 #pragma unroll
