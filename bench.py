@@ -6,8 +6,11 @@ BRO formats vs the in-repo uncompressed ELL/HYB kernels (BASELINE.json).
                   [--impl ours|reference] [--dtype f64|f32]
 
 A step is one pass of the hot path: one bro_spmv (BRO-ELL: one kernel; BRO-HYB:
-ELL kernel + COO kernel + fix-up) over the resident matrix; for N > 1 also the
-NCCL allgather of the y blocks (row-block iteration of a CG loop).  Default
+ELL kernel + COO kernel + fix-up) over the resident matrix.  For N > 1 a step
+is one row-block iteration x_(k+1) = A.x_k of a CG-style loop: every rank's
+SpMV plus the exchange that gives every rank all of x_(k+1) (--exchange:
+fused P2P scatter from the kernel epilogue, overlapped NCCL allgather, or
+SpMV-then-allgather; paper_conf_sc_tangtrwckgtw13_b200/dist.py).  Default
 workload: C5 (3D 27-point stencil on 200^3, 8M rows, 213.8M nnz, fp64,
 BRO-ELL) — the largest config, the one BASELINE.json runs at 1/2/4/8 GPUs.
 Its 2.0 GB working set exceeds the 126 MB L2, so no flush is needed between
@@ -55,6 +58,9 @@ def parse_args():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--flush-l2", action="store_true", help="write a 2xL2 buffer between steps")
+    ap.add_argument("--exchange", default="auto", choices=["auto", "allgather", "overlap", "p2p"],
+                    help="N>1 exchange of the row-block iteration (auto: p2p, else overlap, else allgather, "
+                         "each verified against allgather before timing)")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo only for functional checks of the N>1 path on one GPU")
     return ap.parse_args()
@@ -216,6 +222,50 @@ def run_reference(args):
            "e2e": {"value": val, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
 
+def build_row_block(A, rank, world, dev, fmt, dtype, bounds, args, x_host, stream):
+    """The BRO row block with the fastest exchange that reproduces the
+    allgather schedule on this box: p2p (fused scatter into symmetric memory),
+    else overlap, else allgather.  Every rank takes the same decision."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_tangtrwckgtw13_b200.dist import RowBlockSpmv
+    order = ["p2p", "overlap", "allgather"] if args.exchange == "auto" else [args.exchange]
+    notes = []
+    for mode in order:
+        blk, err = None, ""
+        try:
+            blk = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=1, dtype=dtype, bounds=bounds,
+                               vec_words=args.vec_words, exchange=mode)
+            if mode != "allgather":
+                res = []
+                for ex in (mode, "allgather"):
+                    blk.set_x(x_host)
+                    for _ in range(3):
+                        blk.step(stream, ex)
+                    blk.complete(stream)
+                    torch.cuda.synchronize()
+                    res.append(blk.X[blk.k % 2].clone())
+                a, b = res
+                if not (torch.isfinite(a).all() and torch.allclose(a, b, rtol=1e-9, atol=0.0)):
+                    err = "3-iteration result differs from the allgather schedule"
+        except Exception as e:  # noqa: BLE001 - any setup failure moves to the next mode
+            err = f"{type(e).__name__}: {e}"[:200]
+        ok = torch.tensor([0.0 if err else 1.0], dtype=torch.float64,
+                          device=dev if args.dist_backend == "nccl" else "cpu")
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+        if ok.item() == 1.0:
+            info = {"exchange": mode, "requested": args.exchange, "rejected": notes,
+                    "multicast": bool(blk.use_mc and blk.mc[0]),
+                    "overlap_split": list(getattr(blk, "split", (0, 0))) if mode == "overlap" else None}
+            return blk, info
+        notes.append({"mode": mode, "why": err or "failed on another rank"})
+        if blk is not None:
+            try:
+                blk.close()
+            except Exception:  # noqa: BLE001
+                pass
+    raise SystemExit(f"no exchange mode worked: {notes}")
+
 
 def main():
     args = parse_args()
@@ -254,26 +304,44 @@ def main():
     stream = torch.cuda.current_stream(dev)
     x = torch.from_numpy(x_host).to(dev)
 
-    blk = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=1, dtype=dtype, bounds=bounds,
-                       vec_words=args.vec_words)
-    base = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=0, dtype=dtype, bounds=bounds)
+    exch_info = None
+    if world > 1:
+        blk, exch_info = build_row_block(A, rank, world, dev, fmt, dtype, bounds, args, x_host, stream)
+        base = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=0, dtype=dtype, bounds=bounds,
+                            exchange=blk.exchange)
+        blk.set_x(x_host)
+        base.set_x(x_host)
+    else:
+        blk = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=1, dtype=dtype, bounds=bounds,
+                           vec_words=args.vec_words)
+        base = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=0, dtype=dtype, bounds=bounds)
     info, binfo = blk.mat.info, base.mat.info
     launches = (0 if fmt == "coo" else 1) + (2 if info["nnz_coo"] else 0)  # ELL kernel, COO kernel + fix-up
     flush_buf = torch.empty(2 * L2_BYTES // 4, dtype=torch.int32, device=dev) if args.flush_l2 else None
     flush = (lambda: flush_buf.fill_(1)) if args.flush_l2 else None
+    y1 = torch.empty(A.m, dtype=tdt, device=dev) if world == 1 else None
 
     if world > 1:
+        # x_{k+1} = A.x_k over the row blocks with the chosen exchange
         def step():
-            blk.step(x, stream)
+            blk.step(stream)
 
         def step_base():
-            base.step(x, stream)
+            base.step(stream)
+
+        def spmv_only():
+            blk.spmv(stream=stream)
+
+        def spmv_only_base():
+            base.spmv(stream=stream)
     else:
         def step():
-            blk.spmv(x, stream)
+            blk.mat.spmv(x, y1, stream)
 
         def step_base():
-            base.spmv(x, stream)
+            base.mat.spmv(x, y1, stream)
+
+        spmv_only, spmv_only_base = step, step_base
 
     # --- timed region (ours) with clock sampling
     clocks = ClockSampler(local) if rank == 0 else None
@@ -289,23 +357,30 @@ def main():
     ck = clocks.stop() if clocks else None
     total_ms = float(per_step.sum())
     # kernel-only duration (SpMV launch without the allgather) for the roofline
-    kern = time_steps(lambda: blk.spmv(x, stream), min(args.steps, 500), 3, stream, flush)
+    kern = time_steps(spmv_only, min(args.steps, 500), 3, stream, flush)
     kern_ms = float(np.mean(kern))
     base_ms = float(np.mean(time_steps(step_base, min(args.steps, 500), args.warmup, stream, flush)))
-    base_kern_ms = float(np.mean(time_steps(lambda: base.spmv(x, stream), min(args.steps, 500), 3,
-                                            stream, flush)))
+    base_kern_ms = float(np.mean(time_steps(spmv_only_base, min(args.steps, 500), 3, stream, flush)))
+    ag_ms = None
     if world > 1:
-        total_ms, base_ms = max_over_ranks([total_ms, base_ms], dev, args.dist_backend)
+        # the same iteration with the baseline schedule (SpMV, then allgather)
+        ag_ms = float(np.mean(time_steps(lambda: blk.step(stream, "allgather"), min(args.steps, 500),
+                                         args.warmup, stream, flush)))
+        total_ms, base_ms, kern_ms_max, ag_ms = max_over_ranks([total_ms, base_ms, kern_ms, ag_ms], dev,
+                                                                args.dist_backend)
+        exch_info.update({"allgather_ms_per_step": ag_ms, "spmv_only_ms_max_over_ranks": kern_ms_max,
+                          "spmv_only_gflops": 2.0 * A.nnz / (kern_ms_max * 1e-3) / 1e9,
+                          "speedup_vs_allgather": ag_ms / (total_ms / args.steps)})
 
     # --- launch latency: the same bro_spmv captured once in a CUDA graph and
     # replayed (the CG-loop form; matters for the small, L2-resident C1/C2)
     graph = None
     if world == 1:
         g = torch.cuda.CUDAGraph()
-        blk.spmv(x, stream)
+        blk.mat.spmv(x, y1, stream)
         torch.cuda.synchronize()
         with torch.cuda.graph(g):
-            blk.spmv(x, None)
+            blk.mat.spmv(x, y1, None)
         g_ms = time_steps(g.replay, min(args.steps, 500), 3, stream, flush)
         graph = {"us_per_call": float(np.median(g_ms)) * 1e3,
                  "p10_us": float(np.percentile(g_ms, 10)) * 1e3, "p90_us": float(np.percentile(g_ms, 90)) * 1e3,
@@ -314,7 +389,8 @@ def main():
     # --- end to end through the C ABI with pinned host buffers (rank 0 / N=1 path)
     e2e = None
     if not args.no_e2e:
-        xh = torch.from_numpy(x_host).pin_memory()
+        from paper_conf_sc_tangtrwckgtw13_b200.dist import global_to_padded
+        xh = torch.from_numpy(global_to_padded(x_host, bounds) if world > 1 else x_host).pin_memory()
         yh = torch.empty(blk.mat.m, dtype=tdt).pin_memory()
         xh_np, yh_np = xh.numpy(), yh.numpy()
         P.bro_spmv_host(blk.mat.h, xh_np, yh_np, stream.cuda_stream)  # warm
@@ -332,7 +408,7 @@ def main():
             (e2e_ms,) = max_over_ranks([e2e_ms], dev, args.dist_backend)
         isz = np.dtype(dtype).itemsize
         e2e = {"value": 2.0 * A.nnz / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s",
-               "h2d_bytes_per_step": int(A.n * isz), "d2h_bytes_per_step": int(blk.mat.m * isz),
+               "h2d_bytes_per_step": int(blk.mat.n * isz), "d2h_bytes_per_step": int(blk.mat.m * isz),
                "ms_per_step": e2e_ms,
                "path": "bro_spmv_host: pinned x H2D + bro_spmv + y D2H + stream sync, per rank"}
 
@@ -378,7 +454,8 @@ def main():
             "vec_words": info["vec_words"],
             "l2": ("flushed (2x L2 write) before every step" if args.flush_l2 else
                    ("inputs larger than L2" if alg_bytes > L2_BYTES else "L2-resident (warm)")),
-            "parallelism": f"row-block x{world}" + (" + NCCL allgather of y per step" if world > 1 else ""),
+            "parallelism": f"row-block x{world}" + (f" + {exch_info['exchange']} exchange of y per step (x_(k+1) = A.x_k)"
+                                                    if world > 1 else ""),
             "eta_stream": info["eta_stream"], "eta_total": info["eta_total"],
         },
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
@@ -396,6 +473,7 @@ def main():
                          "speedup_bro": value / base_value},
         "step_ms_p10_p50_p90": [float(np.percentile(per_step, q)) for q in (10, 50, 90)],
         "cuda_graph": graph,
+        "exchange": exch_info,
         "gpu_launches": int(launches * args.steps),
         "clocks": ck,
         "cpu_baseline": cpu,

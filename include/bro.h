@@ -168,6 +168,31 @@ bro_status_t bro_create_hyb(int device, bro_dtype_t dtype, int64_t m, int64_t n,
  * Launch errors are returned; device faults surface at the next sync. */
 bro_status_t bro_spmv(bro_matrix_t A, const void* x_dev, void* y_dev, bro_stream_t stream);
 
+/* Maximum number of y destinations of bro_spmv_scatter. */
+#define BRO_MAX_DST 8
+
+/* y = A.x stored into several destinations at once: the fused exchange of
+ * the row-block iteration (BASELINE.json north_star: "x replicated via an
+ * allgather per iteration, as in a CG loop").
+ *   y_dsts  HOST array of n_dst (1..BRO_MAX_DST) DEVICE pointers, each to m
+ *           values of the handle's dtype.  y_dsts[0] is the local y on the
+ *           handle's device; the others may be any addresses that device can
+ *           store to — typically this rank's block inside every peer GPU's
+ *           x replica, peer-mapped through symmetric memory over NVLink.
+ *           The array is read during the call only.
+ *   y_mc    NULL, or an NVLS multicast address (m values) bound to every
+ *           replica including y_dsts[0]'s memory: stores then go once
+ *           through multimem.st and the switch fans them out.
+ * For ELL-only handles (BRO-ELL, ELLPACK) the kernel's epilogue stores every
+ * destination (no separate copy); handles with a COO part (COO, HYB) finish
+ * y in y_dsts[0] and then replicate it (the COO part adds into y).
+ * Asynchronous on `stream`; completion on a PEER is not signalled: the
+ * caller orders readers after a cross-GPU barrier.  x must not alias any
+ * destination.  Errors: BRO_ERR_ARG (n_dst out of range, NULL or aliasing
+ * pointers), BRO_ERR_UNSUPPORTED (host-only handle), BRO_ERR_CUDA. */
+bro_status_t bro_spmv_scatter(bro_matrix_t A, const void* x_dev, void* const* y_dsts, int32_t n_dst,
+                              void* y_mc, bro_stream_t stream);
+
 /* End-to-end y = A.x with HOST vectors: copies x (n values) host->device,
  * runs bro_spmv, copies y (m values) device->host and synchronizes `stream`.
  * Pinned host memory gives full PCIe bandwidth; pageable memory works. */

@@ -2,8 +2,9 @@
 
 Hot path: y = A.x over BRO-ELL / BRO-COO / BRO-HYB with the index streams
 decoded inside sm_100a kernels (csrc/kernels.cuh) behind the C ABI of
-include/bro.h.  `dist` adds the row-block multi-GPU iteration (NCCL allgather
-of y into the replicated x).
+include/bro.h.  `dist` adds the row-block multi-GPU iteration x_{k+1} = A.x_k
+(allgather, overlapped allgather, or the fused P2P scatter of y into every
+rank's x replica).
 """
 from .bro import (  # noqa: F401
     BroError,
@@ -22,6 +23,8 @@ from .bro import (  # noqa: F401
     bro_reorder_bar,
     bro_spmv,
     bro_spmv_host,
+    bro_spmv_scatter,
+    BRO_MAX_DST,
     bro_status_str,
     bro_version,
     BRO_DEVICE_HOST_ONLY,

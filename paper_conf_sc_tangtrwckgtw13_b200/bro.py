@@ -12,7 +12,10 @@ import os
 
 import numpy as np
 
-_LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libbro.so")
+# BRO_LIB names an alternative in-tree build (A/B timing of two kernel
+# versions in one session); default libbro.so
+_LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)),
+                         os.path.basename(os.environ.get("BRO_LIB", "") or "libbro.so"))
 if not os.path.exists(_LIB_PATH):
     raise ImportError(f"libbro.so not built ({_LIB_PATH}); run __graft_entry__.build() "
                       "or python -m paper_conf_sc_tangtrwckgtw13_b200._build")
@@ -64,6 +67,7 @@ _sig = {
                                  C.POINTER(bro_opts_t), C.POINTER(_H)]),
     "bro_spmv": (C.c_int, [_H, _P, _P, _P]),
     "bro_spmv_host": (C.c_int, [_H, _P, _P, _P]),
+    "bro_spmv_scatter": (C.c_int, [_H, _P, C.POINTER(C.c_void_p), C.c_int32, _P, _P]),
     "bro_destroy": (C.c_int, [_H]),
     "bro_get_info": (C.c_int, [_H, C.POINTER(bro_info_t)]),
     "bro_export_encoded": (C.c_int, [_H, C.c_int32, _P, C.POINTER(C.c_size_t)]),
@@ -153,6 +157,18 @@ def bro_create_coo(device, m, n, row_idx, col_idx, vals, opts=None) -> int:
 
 def bro_spmv(h: int, x_dev_ptr: int, y_dev_ptr: int, stream_ptr: int = 0):
     _check(_lib.bro_spmv(h, x_dev_ptr, y_dev_ptr, stream_ptr or None), "bro_spmv")
+
+
+BRO_MAX_DST = 8
+
+
+def bro_spmv_scatter(h: int, x_dev_ptr: int, y_dst_ptrs, y_mc_ptr: int = 0, stream_ptr: int = 0):
+    """y stored into every device address of y_dst_ptrs (first = local y), or
+    through the multicast address y_mc_ptr (include/bro.h)."""
+    n = len(y_dst_ptrs)
+    arr = (C.c_void_p * max(n, 1))(*[int(p) for p in y_dst_ptrs])
+    _check(_lib.bro_spmv_scatter(h, x_dev_ptr, arr, n, y_mc_ptr or None, stream_ptr or None),
+           "bro_spmv_scatter")
 
 
 def bro_spmv_host(h: int, x: np.ndarray, y: np.ndarray, stream_ptr: int = 0):
@@ -253,6 +269,17 @@ class BroMatrix:
             stream = torch.cuda.current_stream(x.device)
         bro_spmv(self.h, x.data_ptr(), y.data_ptr(), stream.cuda_stream)
         return y
+
+    def spmv_scatter(self, x, y_dst_ptrs, y_mc_ptr=0, stream=None):
+        """y = A.x stored into every device address of y_dst_ptrs (each m
+        values; the first is the local y) — the fused exchange of dist.py."""
+        import torch
+        tdt = torch.float64 if self.dtype == np.float64 else torch.float32
+        if not (x.is_cuda and x.dtype == tdt and x.is_contiguous() and x.numel() == self.n):
+            raise ValueError("x must be a contiguous CUDA tensor of the matrix dtype and length n")
+        if stream is None:
+            stream = torch.cuda.current_stream(x.device)
+        bro_spmv_scatter(self.h, x.data_ptr(), y_dst_ptrs, y_mc_ptr, stream.cuda_stream)
 
     def spmv_host(self, x: np.ndarray, y: np.ndarray = None, stream=None):
         if y is None:

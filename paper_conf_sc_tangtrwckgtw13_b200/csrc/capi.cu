@@ -7,6 +7,7 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <type_traits>
 
 #include "../../include/bro.h"
 #include "encode.hpp"
@@ -313,10 +314,10 @@ bro_status_t common_checks(bro_dtype_t dtype, const bro_opts_t* opts, bro_opts_t
 
 // Persistent grid: as many resident blocks as the SMs hold (queried once per
 // instantiation), capped by the number of slices.
-template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34>
-void launch_bro_ell_od(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+template <typename T, int V, int kWarps, int kMinBlocks, int G, int kRows, bool kMulti>
+void launch_bro_ell_od_k(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cudaStream_t st) {
   using namespace bro::dev;
-  auto kern = bro_ell_spmv_od<T, V, kWarps, kMinBlocks, G, kRows>;
+  auto kern = bro_ell_spmv_od<T, V, kWarps, kMinBlocks, G, kRows, kMulti>;
   static int resident = 0;
   if (resident == 0) {
     int per_sm = 0, sms = 0, dev = 0;
@@ -329,6 +330,13 @@ void launch_bro_ell_od(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
   const unsigned grid = (unsigned)std::min<int64_t>(need, resident);
   kern<<<grid, kWarps * 32, 0, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr,
                                      (const T*)A->d_ell_vals, x, y);
+}
+
+// single-destination instance unless the call scatters (bro_spmv_scatter)
+template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34>
+void launch_bro_ell_od(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cudaStream_t st) {
+  if (y.n > 1 || y.mc != nullptr) launch_bro_ell_od_k<T, V, kWarps, kMinBlocks, G, kRows, true>(A, x, y, st);
+  else launch_bro_ell_od_k<T, V, kWarps, kMinBlocks, G, kRows, false>(A, x, y, st);
 }
 
 constexpr int kEllWarps = 8;      // slices per block
@@ -350,7 +358,7 @@ int env_int(const char* name, int dflt) {
 }
 
 template <typename T, int G>
-bool launch_bro_ell_bulk_g(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+bool launch_bro_ell_bulk_g(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cudaStream_t st) {
   using namespace bro::dev;
   using L = BulkSmem<kBulkWarps>;
   const int unit = int((A->bulk_unit_max + 127) / 128 * 128);
@@ -380,16 +388,17 @@ bool launch_bro_ell_bulk_g(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
 }
 
 template <typename T>
-bool launch_bro_ell_bulk(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+bool launch_bro_ell_bulk(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cudaStream_t st) {
   if (env_int("BRO_BULK_G", kBulkG) == 16) return launch_bro_ell_bulk_g<T, 16>(A, x, y, st);
   return launch_bro_ell_bulk_g<T, 32>(A, x, y, st);
 }
 
 template <typename T, int V>
-void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+void launch_bro_ell(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cudaStream_t st) {
   // BRO_ELL_KERNEL=2 selects the bulk-staged kernel (V = 1 only; measured
   // slower than the register-staged one on C3-C5)
-  if (V == 1 && env_int("BRO_ELL_KERNEL", 0) == 2 && launch_bro_ell_bulk<T>(A, x, y, st)) return;
+  if (V == 1 && y.n == 1 && y.mc == nullptr && env_int("BRO_ELL_KERNEL", 0) == 2 && launch_bro_ell_bulk<T>(A, x, y, st))
+    return;
   const int variant = env_int("BRO_ELL_VARIANT", 0);  // tuning sweeps only
   if (variant == 1)
     launch_bro_ell_od<T, V, kEllWarps, 5, 4, 34>(A, x, y, st);
@@ -402,20 +411,39 @@ void launch_bro_ell(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
 }
 
 template <typename T>
-bro_status_t launch_spmv(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
+bro::dev::YOut<T> make_yout(T* y) {
+  bro::dev::YOut<T> o{};
+  o.p[0] = y;
+  o.n = 1;
+  return o;
+}
+
+// y = A.x stored into every destination of yo (yo.p[0] = the local y on A's
+// device).  ELL-only handles store all destinations from the ELL kernel's
+// epilogue (fused exchange); handles with a COO part finish y locally and
+// then replicate it (the COO part and the fix-up add into y).
+template <typename T>
+bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& yo, cudaStream_t st) {
   using namespace bro::dev;
   const int V = A->opts.vec_words;
+  T* y = yo.p[0];
+  const bool fused = !(A->has_coo && A->nI > 0);
+  const YOut<T> ye = fused ? yo : make_yout(y);
   if (A->has_ell) {
     if (A->opts.codec) {
       if (A->s > 0) {
-        if (V == 4) launch_bro_ell<T, 4>(A, x, y, st);
-        else if (V == 2) launch_bro_ell<T, 2>(A, x, y, st);
-        else launch_bro_ell<T, 1>(A, x, y, st);
+        if (V == 4) launch_bro_ell<T, 4>(A, x, ye, st);
+        else if (V == 2) launch_bro_ell<T, 2>(A, x, ye, st);
+        else launch_bro_ell<T, 1>(A, x, ye, st);
       }
     } else if (A->m > 0) {
       dim3 grid((unsigned)((A->m + kPlainThreads - 1) / kPlainThreads));
-      ell_spmv<T, kPlainThreads><<<grid, kPlainThreads, 0, st>>>(A->m, A->K, A->pitch, A->d_pell_col,
-                                                                  (const T*)A->d_ell_vals, x, y);
+      if (ye.n > 1 || ye.mc != nullptr)
+        ell_spmv<T, kPlainThreads, true><<<grid, kPlainThreads, 0, st>>>(A->m, A->K, A->pitch, A->d_pell_col,
+                                                                        (const T*)A->d_ell_vals, x, ye);
+      else
+        ell_spmv<T, kPlainThreads, false><<<grid, kPlainThreads, 0, st>>>(A->m, A->K, A->pitch, A->d_pell_col,
+                                                                         (const T*)A->d_ell_vals, x, ye);
     }
   } else if (A->m > 0) {
     cudaMemsetAsync(y, 0, size_t(A->m) * sizeof(T), st);
@@ -442,6 +470,10 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, T* y, cudaStream_t st) {
     dim3 g2((unsigned)((nU + 255) / 256));
     coo_fixup<T><<<g2, 256, 0, st>>>(nU, A->d_first_row, A->d_last_row, (const T*)A->d_cf,
                                      (const T*)A->d_cl, y);
+  }
+  if (!fused && A->m > 0 && (yo.n > 1 || yo.mc != nullptr)) {
+    const unsigned g3 = (unsigned)std::min<int64_t>((A->m + 255) / 256, 148 * 8);
+    replicate_y<T><<<g3, 256, 0, st>>>(A->m, yo);
   }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("kernel launch: ") + cudaGetErrorString(e));
@@ -549,8 +581,34 @@ bro_status_t bro_spmv(bro_matrix_t A, const void* x, void* y, bro_stream_t strea
   if (x == y && A->m > 0) return fail(BRO_ERR_ARG, "x and y must not alias");
   DeviceGuard g(A->device);
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-  if (A->dtype == BRO_FP64) return launch_spmv<double>(A, (const double*)x, (double*)y, st);
-  return launch_spmv<float>(A, (const float*)x, (float*)y, st);
+  if (A->dtype == BRO_FP64) return launch_spmv<double>(A, (const double*)x, make_yout((double*)y), st);
+  return launch_spmv<float>(A, (const float*)x, make_yout((float*)y), st);
+}
+
+bro_status_t bro_spmv_scatter(bro_matrix_t A, const void* x, void* const* y_dsts, int32_t n_dst,
+                              void* y_mc, bro_stream_t stream) {
+  if (!A) return fail(BRO_ERR_ARG, "matrix is NULL");
+  if (A->host_only) return fail(BRO_ERR_UNSUPPORTED, "host-only handle: no device copy (there is no CPU SpMV path)");
+  if (!y_dsts || n_dst < 1 || n_dst > bro::dev::kMaxDst)
+    return fail(BRO_ERR_ARG, "y_dsts must hold 1.." + std::to_string(bro::dev::kMaxDst) + " pointers");
+  if (!x && A->n > 0) return fail(BRO_ERR_ARG, "x is NULL");
+  for (int i = 0; i < n_dst; ++i) {
+    if (!y_dsts[i] && A->m > 0) return fail(BRO_ERR_ARG, "y_dsts[" + std::to_string(i) + "] is NULL");
+    if (y_dsts[i] == x && A->m > 0) return fail(BRO_ERR_ARG, "x and a y destination must not alias");
+  }
+  if (y_mc && y_mc == x && A->m > 0) return fail(BRO_ERR_ARG, "x and the multicast y must not alias");
+  DeviceGuard g(A->device);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  auto run = [&](auto* tag) {
+    using T = std::remove_pointer_t<decltype(tag)>;
+    bro::dev::YOut<T> o{};
+    for (int i = 0; i < n_dst; ++i) o.p[i] = static_cast<T*>(y_dsts[i]);
+    o.n = n_dst;
+    o.mc = static_cast<T*>(y_mc);
+    return launch_spmv<T>(A, static_cast<const T*>(x), o, st);
+  };
+  if (A->dtype == BRO_FP64) return run((double*)nullptr);
+  return run((float*)nullptr);
 }
 
 bro_status_t bro_spmv_host(bro_matrix_t A, const void* x_host, void* y_host, bro_stream_t stream) {

@@ -94,6 +94,47 @@ __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
 
+// ------------------------------------------------------------------ y destinations
+// Where an ELL kernel stores y[row].  n = 1 is plain SpMV.  n > 1 is the
+// fused exchange of the row-block iteration: the same
+// value is also stored into the x replica of every peer GPU (P2P stores
+// through NVLink, p[i] = peer-mapped symmetric-memory pointers), so the
+// allgather of y overlaps the SpMV row by row instead of following it.
+// mc != nullptr: one multimem.st to an NVLS multicast address writes every
+// bound replica (the local one included) through the NVSwitch, and p[] is
+// unused.  Indices are static (unrolled) so the table stays in the
+// kernel-parameter bank.
+constexpr int kMaxDst = 8;
+template <typename T>
+struct YOut {
+  T* p[kMaxDst];
+  T* mc;
+  int n;
+};
+
+__device__ __forceinline__ void multimem_st(double* a, double v) {
+  asm volatile("multimem.st.relaxed.sys.global.f64 [%0], %1;" :: "l"(a), "d"(v) : "memory");
+}
+__device__ __forceinline__ void multimem_st(float* a, float v) {
+  asm volatile("multimem.st.relaxed.sys.global.f32 [%0], %1;" :: "l"(a), "f"(v) : "memory");
+}
+
+template <bool kMulti, typename T>
+__device__ __forceinline__ void store_y(const YOut<T>& o, int64_t row, T v) {
+  if constexpr (!kMulti) {  // plain SpMV: one store, no destination table
+    o.p[0][row] = v;
+    return;
+  }
+  if (o.mc != nullptr) {
+    multimem_st(o.mc + row, v);
+    return;
+  }
+  o.p[0][row] = v;
+#pragma unroll
+  for (int i = 1; i < kMaxDst; ++i)
+    if (i < o.n) o.p[i][row] = v;
+}
+
 // shl with the PTX clamp (shift >= 32 gives 0)
 __device__ __forceinline__ uint32_t shl_clamp(uint32_t v, uint32_t s) {
   uint32_t r;
@@ -282,12 +323,12 @@ __device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __r
 // (G = 4, kRows = 6, 48 warps/SM) serves matrices whose slices all have
 // l <= 4 columns (<= 4 symbols per row): less shared memory and fewer
 // registers buy 1.5x the resident warps for the latency-bound short rows.
-template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34>
+template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34, bool kMulti = false>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
                 const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
                 const uint64_t* __restrict__ symptr, const T* __restrict__ vals,
-                const T* __restrict__ x, T* __restrict__ y) {
+                const T* __restrict__ x, const YOut<T> y) {
   struct Meta { uint64_t c0, q0; int l, S; };
   __shared__ uint32_t window[kWarps][kRows * 32];
   __shared__ uint2 colmeta[kWarps][32];  // per column of the block: {byte offset of its word row, r | (32-b) << 8}
@@ -371,7 +412,7 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
       obase += tot;
     }
     const int64_t row = 32 * t + lane;
-    if (row < m) y[row] = sum;
+    if (row < m) store_y<kMulti>(y, row, sum);
   }
 }
 
@@ -443,7 +484,7 @@ __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_spmv_bulk(int64_t m, int64_t s, const uint32_t* __restrict__ words,
                   const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
                   const uint64_t* __restrict__ symptr, const T* __restrict__ vals,
-                  const T* __restrict__ x, T* __restrict__ y, int nslot, int slot_bytes) {
+                  const T* __restrict__ x, const YOut<T> y, int nslot, int slot_bytes) {
   using L = BulkSmem<kWarps>;
   constexpr int VV = Chunk<T>::N;
   extern __shared__ __align__(128) uint8_t smem[];
@@ -576,7 +617,7 @@ bro_ell_spmv_bulk(int64_t m, int64_t s, const uint32_t* __restrict__ words,
       __syncwarp();
     }
     const int64_t row = 32 * (t0 + int64_t(k) * stride) + lane;
-    if (row < m) y[row] = sum;
+    if (row < m) store_y<false>(y, row, sum);
     if (++slot == nslot) { slot = 0; phase ^= 1; }
   }
 }
@@ -604,10 +645,10 @@ __global__ void bro_ell_decode(int64_t s, const uint32_t* __restrict__ words,
 }
 
 // ------------------------------------------------------------------ plain ELLPACK
-template <typename T, int kThreads>
+template <typename T, int kThreads, bool kMulti = false>
 __global__ void __launch_bounds__(kThreads)
 ell_spmv(int64_t m, int64_t K, int64_t pitch, const int32_t* __restrict__ col,
-         const T* __restrict__ vals, const T* __restrict__ x, T* __restrict__ y) {
+         const T* __restrict__ vals, const T* __restrict__ x, const YOut<T> y) {
   constexpr int G = 8;
   const int64_t row = int64_t(blockIdx.x) * kThreads + threadIdx.x;
   if (row >= m) return;
@@ -632,7 +673,7 @@ ell_spmv(int64_t m, int64_t K, int64_t pitch, const int32_t* __restrict__ col,
     const T v = ld_stream(vals + j * pitch + row);
     if (c >= 0) sum = fma(v, ldg_x(x + c), sum);
   }
-  y[row] = sum;
+  store_y<kMulti>(y, row, sum);
 }
 
 __global__ void ell_decode(int64_t m, int64_t K, int64_t pitch, const int32_t* __restrict__ col,
@@ -843,6 +884,27 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restri
       carry_last[u] = T(0);
     } else {
       carry_last[u] = carry;
+    }
+  }
+}
+
+// Exchange of a finished y for formats whose last kernel is not an ELL
+// kernel (COO / HYB: the COO part and the fix-up add into y after the ELL
+// part stored it, so only the final values may leave the GPU): copy the
+// local y (o.p[0]) into the other destinations o.p[1..n-1], or once through
+// the multicast address; m * sizeof(T) bytes per peer.
+template <typename T>
+__global__ void replicate_y(int64_t m, const YOut<T> o) {
+  const T* __restrict__ src = o.p[0];
+  const int64_t stride = int64_t(gridDim.x) * blockDim.x;
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < m; i += stride) {
+    const T v = src[i];
+    if (o.mc != nullptr) {
+      multimem_st(o.mc + i, v);
+    } else {
+#pragma unroll
+      for (int k = 1; k < kMaxDst; ++k)
+        if (k < o.n) o.p[k][i] = v;
     }
   }
 }
