@@ -460,12 +460,14 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
                                          (const T*)A->d_coo_vals, x, y, (T*)A->d_cf, (T*)A->d_cl,
                                          A->d_first_row, A->d_last_row);
     };
+    // BRO_COO_MINB=4: 64-register instances (32 resident warps/SM; tuning sweeps)
+    const bool minb4 = env_int("BRO_COO_MINB", 0) == 4;
     if (A->opts.codec) {
-      if (V == 4) args(coo_spmv<T, 4, true, kCooThreads>);
+      if (V == 4) minb4 ? args(coo_spmv<T, 4, true, kCooThreads, 4>) : args(coo_spmv<T, 4, true, kCooThreads>);
       else if (V == 2) args(coo_spmv<T, 2, true, kCooThreads>);
-      else args(coo_spmv<T, 1, true, kCooThreads>);
+      else minb4 ? args(coo_spmv<T, 1, true, kCooThreads, 4>) : args(coo_spmv<T, 1, true, kCooThreads>);
     } else {
-      args(coo_spmv<T, 4, false, kCooThreads>);
+      minb4 ? args(coo_spmv<T, 4, false, kCooThreads, 4>) : args(coo_spmv<T, 4, false, kCooThreads>);
     }
     dim3 g2((unsigned)((nU + 255) / 256));
     coo_fixup<T><<<g2, 256, 0, st>>>(nU, A->d_first_row, A->d_last_row, (const T*)A->d_cf,

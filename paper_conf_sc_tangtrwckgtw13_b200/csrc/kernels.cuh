@@ -725,8 +725,8 @@ __device__ __forceinline__ int coo_delta(const uint32_t* wl, int t, int b) {
   return int(shr_clamp(__funnelshift_l(p[32], p[0], uint32_t(o & 31)), uint32_t(32 - b)));
 }
 
-template <typename T, int V, bool kBro, int kThreads>
-__global__ void __launch_bounds__(kThreads)
+template <typename T, int V, bool kBro, int kThreads, int kMinBlocks = 1>
+__global__ void __launch_bounds__(kThreads, kMinBlocks)
 coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restrict__ words,
          const uint32_t* __restrict__ base_row, const uint8_t* __restrict__ width,
          const uint64_t* __restrict__ symptr, const int32_t* __restrict__ rows,
