@@ -79,6 +79,7 @@ struct bro_matrix_s {
   void* d_ys = nullptr;
   int64_t device_bytes = 0;
   uint32_t bulk_unit_max = 0;
+  int64_t ell_max_S = 0;       // most 32-bit symbols in one BRO-ELL row stream
   int64_t ell_max_l = 0;       // longest BRO-ELL slice (columns)  // largest staged slice of the bulk BRO-ELL kernel (bytes)
   bro_info_t info{};
 };
@@ -207,6 +208,8 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
         A->ell_words = (int64_t)A->ell.words.size();
         A->ell_slots = (int64_t)(A->ell.vals.size() / A->vsize);
         A->ell_max_l = A->ell.max_l;
+        for (int64_t t = 0; t < A->s; ++t)
+          A->ell_max_S = std::max<int64_t>(A->ell_max_S, int64_t(A->ell.symptr[t + 1] - A->ell.symptr[t]));
         for (int64_t t = 0; t < A->s; ++t)
           A->bulk_unit_max = std::max(A->bulk_unit_max,
               bro::dev::bulk_unit_bytes(A->ell.colptr[t], int(A->ell.colptr[t + 1] - A->ell.colptr[t]),
@@ -393,6 +396,31 @@ bool launch_bro_ell_bulk(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
   return launch_bro_ell_bulk_g<T, 32>(A, x, y, st);
 }
 
+// Few slices (fewer than the 32 warps/SM of the general instance can hold,
+// e.g. C2: 1,951 slices of up to 81 columns): every warp is resident anyway,
+// so spend registers on more columns in flight per warp instead: G = 16 at
+// 16 warps/SM for fp64 (127 registers), G = 32 at 8 warps/SM for fp32 (128
+// registers) — measured best on C2 (profiles/r01/s3/few_slices.txt: fp64
+// 22.5 -> 18.5 us, fp32 20.5 -> 16.4 us).  BRO_ELL_FEW_G = 0 disables.
+template <typename T>
+constexpr int kEllFewG = sizeof(T) == 8 ? 16 : 32;
+// Window rows of the small-window instance: every row stream fits in
+// kEllSmallRows - 1 symbols (C5: S <= 7), so the per-warp symbol window
+// shrinks from 34 rows (4.3 KB) to 10 (1.3 KB): 12 KB less shared memory per
+// block, which the SM gives back to L1 for the x gather.
+constexpr int kEllSmallRows = 10;
+inline int64_t few_slices(bro_matrix_s* A) {
+  static int64_t sms = 0;
+  if (sms == 0) {
+    int n = 0, dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    sms = std::max(1, n);
+  }
+  (void)A;
+  return sms * kEllWarps * kEllMinBlocks;
+}
+
 template <typename T, int V>
 void launch_bro_ell(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cudaStream_t st) {
   // BRO_ELL_KERNEL=2 selects the bulk-staged kernel (V = 1 only; measured
@@ -404,10 +432,79 @@ void launch_bro_ell(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cud
     launch_bro_ell_od<T, V, kEllWarps, 5, 4, 34>(A, x, y, st);
   else if (variant == 2)
     launch_bro_ell_od<T, V, kEllWarps, 3, 8, 34>(A, x, y, st);
+  else if (variant == 3)  // 16 columns in flight per warp (few, long slices: C2)
+    launch_bro_ell_od<T, V, kEllWarps, 2, 16, 34>(A, x, y, st);
+  else if (variant == 4)
+    launch_bro_ell_od<T, V, 4, 4, 16, 34>(A, x, y, st);
+  else if (variant == 5)
+    launch_bro_ell_od<T, V, 4, 2, 32, 34>(A, x, y, st);
   else if (A->ell_max_l <= 4 && env_int("BRO_ELL_SHORT", 1))
     launch_bro_ell_od<T, V, kEllWarps, sizeof(T) == 8 ? kEllMinBlocksShort - 1 : kEllMinBlocksShort, 4, 6>(A, x, y, st);
+  else if (A->s < few_slices(A) && env_int("BRO_ELL_FEW_G", kEllFewG<T>) == 32)
+    launch_bro_ell_od<T, V, 4, 2, 32, 34>(A, x, y, st);
+  else if (A->s < few_slices(A) && env_int("BRO_ELL_FEW_G", kEllFewG<T>) == 16)
+    launch_bro_ell_od<T, V, kEllWarps, 2, 16, 34>(A, x, y, st);
+  else if (A->ell_max_S < kEllSmallRows && env_int("BRO_ELL_SMALLWIN", 1))
+    launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks, 8, kEllSmallRows>(A, x, y, st);
   else
     launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks>(A, x, y, st);
+}
+
+// Persistent pipelined COO kernel: kCooPipeWarps warps per block, as many
+// blocks as are resident; one work unit per warp (contiguous intervals).
+// Register budget: MB = 2 (<= 128 registers, 16 warps/SM) or 3 (<= 80, 24
+// warps/SM); BRO_COO_PIPE_MINB selects (tuning), default kCooPipeMinBlocks.
+constexpr int kCooPipeWarps = 8;
+constexpr int kCooPipeMinBlocks = 2;
+
+template <typename T, int V, bool kBro, int MB>
+int64_t coo_pipe_resident() {
+  static int64_t resident = 0;
+  if (resident == 0) {
+    int per_sm = 0, sms = 0, dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+        &per_sm, bro::dev::coo_spmv_pipe<T, V, kBro, kCooPipeWarps, MB>, kCooPipeWarps * 32, 0);
+    resident = int64_t(std::max(1, per_sm)) * std::max(1, sms) * kCooPipeWarps;
+  }
+  return resident;
+}
+
+template <typename T, int MB>
+int64_t coo_pipe_warps_mb(bro_matrix_s* A, int V) {
+  if (!A->opts.codec) return coo_pipe_resident<T, 4, false, MB>();
+  return V == 4 ? coo_pipe_resident<T, 4, true, MB>() : coo_pipe_resident<T, 1, true, MB>();
+}
+
+template <typename T>
+int64_t coo_pipe_warps(bro_matrix_s* A, int V) {
+  return env_int("BRO_COO_PIPE_MINB", kCooPipeMinBlocks) == 3 ? coo_pipe_warps_mb<T, 3>(A, V)
+                                                               : coo_pipe_warps_mb<T, 2>(A, V);
+}
+
+template <typename T, int MB>
+int64_t launch_coo_pipe_mb(bro_matrix_s* A, int V, const T* x, T* y, cudaStream_t st) {
+  using namespace bro::dev;
+  const int64_t nW = std::max<int64_t>(
+      kCooPipeWarps, std::min(coo_pipe_warps_mb<T, MB>(A, V), A->nI) / kCooPipeWarps * kCooPipeWarps);
+  const unsigned grid = (unsigned)(nW / kCooPipeWarps);
+  auto go = [&](auto kern) {
+    kern<<<grid, kCooPipeWarps * 32, 0, st>>>(A->nnz_coo, A->nI, A->d_coo_words, A->d_coo_base, A->d_coo_width,
+                                              A->d_coo_symptr, A->d_coo_row, A->d_coo_col, (const T*)A->d_coo_vals,
+                                              x, y, (T*)A->d_cf, (T*)A->d_cl, A->d_first_row, A->d_last_row);
+  };
+  if (!A->opts.codec) go(coo_spmv_pipe<T, 4, false, kCooPipeWarps, MB>);
+  else if (V == 4) go(coo_spmv_pipe<T, 4, true, kCooPipeWarps, MB>);
+  else go(coo_spmv_pipe<T, 1, true, kCooPipeWarps, MB>);
+  return nW;
+}
+
+// returns the number of work units (warps) for the fix-up
+template <typename T>
+int64_t launch_coo_pipe(bro_matrix_s* A, int V, const T* x, T* y, cudaStream_t st) {
+  return env_int("BRO_COO_PIPE_MINB", kCooPipeMinBlocks) == 3 ? launch_coo_pipe_mb<T, 3>(A, V, x, y, st)
+                                                               : launch_coo_pipe_mb<T, 2>(A, V, x, y, st);
 }
 
 template <typename T>
@@ -450,10 +547,20 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
   }
   if (A->has_coo && A->nI > 0) {
     const int warps = kCooThreads / 32;
-    const int upi = std::max(1, std::min(kCooMaxUpi, env_int("BRO_COO_UPI", kCooUpi)));
-    const int64_t nU = A->nI * upi;
+    int upi = std::max(1, std::min(kCooMaxUpi, env_int("BRO_COO_UPI", kCooUpi)));
+    int64_t nU = A->nI * upi;
+    // BRO_COO_KERNEL: 1 (default) per-unit kernel; 2 persistent pipelined
+    // kernel (opt-in: measured no faster); 0 auto =
+    // pipelined when there are at least as many intervals as resident warps
+    const int ck = env_int("BRO_COO_KERNEL", 1);
+    const int64_t pipe_w = (V == 2 || ck == 1) ? 0 : coo_pipe_warps<T>(A, V);
+    if (pipe_w > 0 && A->nI >= kCooPipeWarps && (ck == 2 || (ck == 0 && A->nI >= pipe_w))) {
+      nU = launch_coo_pipe<T>(A, V, x, y, st);
+      upi = 0;
+    }
     dim3 grid((unsigned)((nU + warps - 1) / warps));
     const int T_ = A->opts.coo_T;
+    if (upi > 0) {
     auto args = [&](auto kern) {
       kern<<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, upi, A->d_coo_words, A->d_coo_base,
                                          A->d_coo_width, A->d_coo_symptr, A->d_coo_row, A->d_coo_col,
@@ -468,6 +575,7 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
       else minb4 ? args(coo_spmv<T, 1, true, kCooThreads, 4>) : args(coo_spmv<T, 1, true, kCooThreads>);
     } else {
       minb4 ? args(coo_spmv<T, 4, false, kCooThreads, 4>) : args(coo_spmv<T, 4, false, kCooThreads>);
+    }
     }
     dim3 g2((unsigned)((nU + 255) / 256));
     coo_fixup<T><<<g2, 256, 0, st>>>(nU, A->d_first_row, A->d_last_row, (const T*)A->d_cf,

@@ -24,6 +24,7 @@
 #pragma once
 #include <cstdint>
 #include <cuda_runtime.h>
+#include <type_traits>
 
 namespace bro {
 namespace dev {
@@ -725,7 +726,67 @@ __device__ __forceinline__ int coo_delta(const uint32_t* wl, int t, int b) {
   return int(shr_clamp(__funnelshift_l(p[32], p[0], uint32_t(o & 31)), uint32_t(32 - b)));
 }
 
-template <typename T, int V, bool kBro, int kThreads, int kMinBlocks = 1>
+// One transposed batch of 8*32 entries (lane owns entries 8*lane .. 8*lane+7,
+// rows r[] non-decreasing across the batch): gathers x, reduces each lane's
+// entries sequentially and links segments across lanes with one warp
+// segmented scan; complete segments go to emit(row, partial), the batch's
+// trailing partial is carried (crow, carry) into the next batch.
+template <typename T, typename Emit>
+__device__ __forceinline__ void coo_segments(const int* r, const int* c, const T* v, const T* __restrict__ x,
+                                             int lane, int& crow, T& carry, Emit&& emit) {
+  constexpr int TB = 8;
+  T xv[TB];
+#pragma unroll
+  for (int k = 0; k < TB; ++k) xv[k] = c[k] >= 0 ? ldg_x(x + c[k]) : T(0);
+  // sequential pass over the lane's 8 entries
+  const int f = r[0];
+  T A = T(0), cur = T(0);
+  bool one = true;
+  int cr = f;
+#pragma unroll
+  for (int k = 0; k < TB; ++k) {
+    const T p = v[k] * xv[k];
+    if (r[k] != cr) {           // the segment of row cr ends inside this lane
+      if (one) { A = cur; one = false; }
+      else emit(cr, cur);       // interior segment: complete, row unique to this lane
+      cr = r[k];
+      cur = p;
+    } else {
+      cur += p;
+    }
+  }
+  if (one) A = cur;
+  const int L = cr;             // trailing segment: row L, partial cur
+  // carry-in from earlier lanes (or earlier batches for lane 0)
+  const int Lprev = __shfl_up_sync(0xffffffffu, L, 1);
+  const bool link = lane == 0 ? (crow == f) : (Lprev == f);
+  // C_out(l) = B_l + [one_l && link_l] * C_out(l-1): segmented scan
+  T co = cur;
+  bool open = one && link;      // this lane's partial continues an earlier one
+  if (lane == 0 && open) co += carry;
+#pragma unroll
+  for (int off = 1; off < 32; off <<= 1) {
+    const T o = __shfl_up_sync(0xffffffffu, co, off);
+    const int op = __shfl_up_sync(0xffffffffu, int(open), off);
+    if (lane >= off && open) co += o;
+    if (lane >= off) open = open && op;
+  }
+  // C_in = C_out(l-1) if linked; lane 0 takes the batch carry
+  T cin = __shfl_up_sync(0xffffffffu, co, 1);
+  if (lane == 0) cin = carry;
+  if (!link) cin = T(0);
+  if (lane == 0 && !link && crow != f) {
+    // the carried row ended before this batch
+    emit(crow, carry);
+  }
+  if (!one) emit(f, A + cin);   // first segment complete inside this lane
+  const int fnext = __shfl_down_sync(0xffffffffu, f, 1);
+  if (lane < 31 && fnext != L) emit(L, co);  // trailing segment complete at this lane
+  carry = __shfl_sync(0xffffffffu, co, 31);
+  crow = __shfl_sync(0xffffffffu, L, 31);
+}
+
+template <typename T, int V, bool kBro, int kThreads, int kMinBlocks = 0>
 __global__ void __launch_bounds__(kThreads, kMinBlocks)
 coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restrict__ words,
          const uint32_t* __restrict__ base_row, const uint8_t* __restrict__ width,
@@ -826,55 +887,181 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restri
       }
       __syncwarp();
     }
-    T xv[TB];
+    coo_segments<T>(r, c, v, x, lane, crow, carry, emit);
+  }
+  if (lane == 0) {
+    first_row[u] = first;
+    last_row[u] = crow;
+    if (crow == first) {
+      carry_first[u] = carry;
+      carry_last[u] = T(0);
+    } else {
+      carry_last[u] = carry;
+    }
+  }
+}
+
+// ------------------------------------------------------------------ (BRO-)COO, persistent pipeline
+// Same entry order, decode and segment logic as coo_spmv, but a persistent
+// warp walks a CONTIGUOUS range of whole intervals batch by batch (8 steps =
+// 256 entries) with a one-batch software pipeline: while batch k is decoded,
+// gathered and reduced, batch k+1's col / vals (rows for plain COO) are
+// already in flight into registers and its row-stream words are copied into
+// the other half of a double-buffered per-warp window by cp.async (no
+// registers).  A batch at step t0 of an interval with width b needs word rows
+// (t0*b)>>5 .. ((t0+8)*b-1)>>5 only (<= 9 rows, S = b words per lane for
+// T = 32), so staging is per batch and never skips.  Interval metadata
+// (base row, width, first word) of the warp's next 32 intervals is fetched
+// lane-parallel into shared memory.  One work unit (carry pair) per warp:
+// rows continue across the warp's intervals, so the fix-up sees nW units.
+__device__ __forceinline__ void cp_async4(uint32_t* dst, const uint32_t* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" :: "r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" :: "n"(N) : "memory"); }
+
+constexpr int kCooPipeRows = 10;  // window rows per batch buffer (<= 9 used)
+
+template <typename T, int V, bool kBro, int kWarps, int kMinBlocks>
+__global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
+coo_spmv_pipe(int64_t nnz, int64_t nI, const uint32_t* __restrict__ words,
+              const uint32_t* __restrict__ base_row, const uint8_t* __restrict__ width,
+              const uint64_t* __restrict__ symptr, const int32_t* __restrict__ rows,
+              const int32_t* __restrict__ col, const T* __restrict__ vals, const T* __restrict__ x,
+              T* __restrict__ y, T* __restrict__ carry_first, T* __restrict__ carry_last,
+              int32_t* __restrict__ first_row, int32_t* __restrict__ last_row) {
+  constexpr int TB = 8;          // steps per batch
+  constexpr int BPI = 32 / TB;   // batches per interval (T = 32)
+  struct IMeta { uint64_t q0; uint32_t base; int b; };
+  __shared__ __align__(16) int32_t rowbuf[kWarps][TB * 32];
+  __shared__ uint32_t cwin[kWarps][kBro ? 2 * kCooPipeRows * 32 : 1];
+  __shared__ IMeta metas[kWarps][kBro ? 32 : 1];
+  const int lane = threadIdx.x & 31;
+  const int w = threadIdx.x >> 5;
+  const int64_t nW = int64_t(gridDim.x) * kWarps;
+  const int64_t u = int64_t(blockIdx.x) * kWarps + w;  // this warp = one work unit
+  const int64_t iA = u * nI / nW, iB = (u + 1) * nI / nW;
+  const int64_t nbat = (iB - iA) * BPI;
+  int32_t* rb = rowbuf[w];
+  if (nbat == 0) {  // (launcher keeps nW <= nI; kept for safety) an empty unit
+    if (lane == 0) { first_row[u] = -1; last_row[u] = -1; carry_first[u] = T(0); carry_last[u] = T(0); }
+    return;
+  }
+  // metadata of intervals [i0, i0 + 32) of this warp into shared memory
+  auto fetch_meta = [&](int64_t i0) {
+    __syncwarp();
+    const int64_t il = i0 + lane;
+    if (kBro && il < iB) metas[w][kBro ? lane : 0] = IMeta{symptr[il], base_row[il], int(width[il])};
+    __syncwarp();
+  };
+  // cp.async the word rows of batch (interval i, step t0) into buffer buf
+  auto stage = [&](int64_t i, int t0, int buf) {
+    if constexpr (kBro) {
+      const IMeta mt = metas[w][(i - iA) & 31];
+      const int b = mt.b;
+      if (b == 0) return;
+      const int S = b;  // T = 32 steps of b bits = b words per lane
+      const int qa = (t0 * b) >> 5, qb = ((t0 + TB) * b - 1) >> 5;
+      const uint32_t* wb = words + 32 * mt.q0;
+      uint32_t* dst = cwin[w] + buf * kCooPipeRows * 32 + lane;
+      for (int q = qa; q <= qb; ++q) cp_async4(dst + 32 * (q - qa), wb + place(lane, q, S, V));
+    }
+  };
+  auto load_batch = [&](int64_t i, int t0, int* r, int* c, T* v) {
+    const int64_t el = i * 1024 + 32 * t0 + TB * lane;  // transposed: lane's 8 consecutive entries
+    if (el + TB <= nnz) {
+      if constexpr (!kBro) load8_s32(r, rows + el);
+      load8_s32(c, col + el);
+      Vec8<T> vv;
+      vv.load(vals + el);
 #pragma unroll
-    for (int k = 0; k < TB; ++k) xv[k] = c[k] >= 0 ? ldg_x(x + c[k]) : T(0);
-    // sequential pass over the lane's 8 entries
-    const int f = r[0];
-    T A = T(0), cur = T(0);
-    bool one = true;
-    int cr = f;
+      for (int k = 0; k < TB; ++k) v[k] = vv.v[k];
+    } else {  // tail of the last interval: entries past nnz repeat the last row with value 0
 #pragma unroll
-    for (int k = 0; k < TB; ++k) {
-      const T p = v[k] * xv[k];
-      if (r[k] != cr) {           // the segment of row cr ends inside this lane
-        if (one) { A = cur; one = false; }
-        else emit(cr, cur);       // interior segment: complete, row unique to this lane
-        cr = r[k];
-        cur = p;
-      } else {
-        cur += p;
+      for (int k = 0; k < TB; ++k) {
+        const bool ok = el + k < nnz;
+        if constexpr (!kBro) r[k] = ld_stream_s32(rows + (ok ? el + k : nnz - 1));
+        c[k] = ok ? ld_stream_s32(col + el + k) : -1;
+        v[k] = ok ? ld_stream(vals + el + k) : T(0);
       }
     }
-    if (one) A = cur;
-    const int L = cr;             // trailing segment: row L, partial cur
-    // carry-in from earlier lanes (or earlier batches for lane 0)
-    const int Lprev = __shfl_up_sync(0xffffffffu, L, 1);
-    const bool link = lane == 0 ? (crow == f) : (Lprev == f);
-    // C_out(l) = B_l + [one_l && link_l] * C_out(l-1): segmented scan
-    T co = cur;
-    bool open = one && link;      // this lane's partial continues an earlier one
-    if (lane == 0 && open) co += carry;
+  };
+
+  if constexpr (kBro) fetch_meta(iA);
+  int r[TB], c[TB];
+  T v[TB];
+  stage(iA, 0, 0);
+  cp_async_commit();
+  load_batch(iA, 0, r, c, v);
+  int row = 0, b = 0;
+  int first = 0;
+  bool first_pending = true;
+  T carry = T(0);
+  int crow = 0;
+  auto emit = [&](int rr, T val) {
+    if (rr == first) carry_first[u] = val;
+    else atomicAdd(y + rr, val);
+  };
+  for (int64_t k = 0; k < nbat; ++k) {
+    const int64_t i = iA + k / BPI;
+    const int t0 = int(k % BPI) * TB;
+    if constexpr (kBro) {
+      if (t0 == 0) {
+        const IMeta mt = metas[w][(i - iA) & 31];
+        row = int(mt.base);
+        b = mt.b;
+      }
+    }
+    // issue batch k+1: words (cp.async) and col / vals (registers)
+    int rn[TB], cn[TB];
+    T vn[TB];
+    const bool has_next = k + 1 < nbat;
+    if (has_next) {
+      const int64_t i1 = iA + (k + 1) / BPI;
+      const int t1 = int((k + 1) % BPI) * TB;
+      if constexpr (kBro) {
+        if (t1 == 0 && ((i1 - iA) & 31) == 0) fetch_meta(i1);  // every 32 intervals (current one in registers)
+      }
+      stage(i1, t1, int((k + 1) & 1));
+      cp_async_commit();
+      load_batch(i1, t1, rn, cn, vn);
+      cp_async_wait<1>();
+    } else {
+      cp_async_wait<0>();
+    }
+    __syncwarp();
+    if constexpr (kBro) {
+      const uint32_t* wl = cwin[w] + int(k & 1) * kCooPipeRows * 32 + lane;
+      const int obase = (t0 * b) & ~31;  // bit offset of the window's first row
 #pragma unroll
-    for (int off = 1; off < 32; off <<= 1) {
-      const T o = __shfl_up_sync(0xffffffffu, co, off);
-      const int op = __shfl_up_sync(0xffffffffu, int(open), off);
-      if (lane >= off && open) co += o;
-      if (lane >= off) open = open && op;
+      for (int s = 0; s < TB; ++s) {
+        const int o = (t0 + s) * b - obase;
+        const uint32_t* pw = wl + 32 * (o >> 5);
+        row += int(shr_clamp(__funnelshift_l(pw[32], pw[0], uint32_t(o & 31)), uint32_t(32 - b)));
+        rb[s * 32 + lane] = row;
+      }
+      __syncwarp();
+      const int4 ra = *reinterpret_cast<const int4*>(rb + TB * lane);
+      const int4 rc = *reinterpret_cast<const int4*>(rb + TB * lane + 4);
+      r[0] = ra.x; r[1] = ra.y; r[2] = ra.z; r[3] = ra.w;
+      r[4] = rc.x; r[5] = rc.y; r[6] = rc.z; r[7] = rc.w;
+      __syncwarp();
     }
-    // C_in = C_out(l-1) if linked; lane 0 takes the batch carry
-    T cin = __shfl_up_sync(0xffffffffu, co, 1);
-    if (lane == 0) cin = carry;
-    if (!link) cin = T(0);
-    if (lane == 0 && !link && crow != f) {
-      // the carried row ended before this batch
-      emit(crow, carry);
+    if (first_pending) {
+      first = __shfl_sync(0xffffffffu, r[0], 0);
+      crow = first;
+      first_pending = false;
     }
-    if (!one) emit(f, A + cin);   // first segment complete inside this lane
-    const int fnext = __shfl_down_sync(0xffffffffu, f, 1);
-    if (lane < 31 && fnext != L) emit(L, co);  // trailing segment complete at this lane
-    carry = __shfl_sync(0xffffffffu, co, 31);
-    crow = __shfl_sync(0xffffffffu, L, 31);
+    coo_segments<T>(r, c, v, x, lane, crow, carry, emit);
+    if (has_next) {
+#pragma unroll
+      for (int q = 0; q < TB; ++q) {
+        c[q] = cn[q];
+        v[q] = vn[q];
+        if constexpr (!kBro) r[q] = rn[q];
+      }
+    }
   }
   if (lane == 0) {
     first_row[u] = first;

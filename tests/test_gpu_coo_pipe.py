@@ -1,0 +1,91 @@
+"""GPU: the persistent pipelined (BRO-)COO kernel (coo_spmv_pipe) against the
+oracle on cases that span many intervals, a ragged last interval, rows that
+cross intervals and warps, and long rows (-m gpu).  BRO_COO_KERNEL=2 forces
+it wherever there are >= 8 intervals; BRO_COO_PIPE_MINB picks the register
+budget (2: 16 warps/SM, 3: 24 warps/SM)."""
+import os
+
+import numpy as np
+import pytest
+
+from gen import make_config, make_x, random_csr
+from oracle import spmv
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+TOL = {np.float64: 1e-12, np.float32: 1e-5}
+
+
+@pytest.fixture(scope="module")
+def dev():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    return torch.device("cuda:0")
+
+
+@pytest.fixture
+def pipe_env():
+    old = {k: os.environ.get(k) for k in ("BRO_COO_KERNEL", "BRO_COO_PIPE_MINB")}
+    yield
+    for k, v in old.items():
+        if v is None:
+            os.environ.pop(k, None)
+        else:
+            os.environ[k] = v
+
+
+CASES = [
+    # ~ 9.5 intervals of COO entries, ragged tail, short rows
+    ("short", lambda: random_csr(4000, 5000, 21, max_len=5, empty_frac=0.2)),
+    # long rows crossing many intervals and warps
+    ("long", lambda: random_csr(3000, 9000, 22, max_len=12, long_frac=0.05, long_len=4000)),
+    # one row of 40,000 entries (every interval one row, width 0)
+    ("one_row", lambda: random_csr(1, 60000, 23, max_len=0, long_frac=1.0, long_len=40000)),
+    ("c1", lambda: make_config(1)),
+]
+
+
+@pytest.mark.parametrize("name,mk", CASES, ids=[c[0] for c in CASES])
+@pytest.mark.parametrize("fmt", ["coo", "hyb"])
+@pytest.mark.parametrize("codec", [1, 0])
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+@pytest.mark.parametrize("minb", ["2", "3"])
+def test_coo_pipe_vs_oracle(lib, dev, pipe_env, name, mk, fmt, codec, dtype, minb):
+    A = mk()
+    os.environ["BRO_COO_KERNEL"] = "2"
+    os.environ["BRO_COO_PIPE_MINB"] = minb
+    for V in ((1, 4) if codec else (4,)):
+        M = lib.BroMatrix(A, fmt=fmt, codec=codec, device=0, dtype=dtype, vec_words=V)
+        if M.info["n_intervals"] < 8:
+            M.close()
+            pytest.skip("fewer than 8 intervals: the per-unit kernel runs")
+        x = make_x(A.n, 9, dtype)
+        y = M.spmv(torch.from_numpy(x).to(dev))
+        torch.cuda.synchronize()
+        y_ref, S = spmv.csr_spmv(A.row_ptr, A.col, A.vals.astype(dtype), x)
+        ok, err = spmv.within_tolerance(y.cpu().numpy(), y_ref, S, TOL[dtype])
+        bad = np.nonzero(~ok)[0]
+        assert ok.all(), f"V={V}: {bad.size} rows out of tolerance, first {bad[:5]} err {err[bad[:5]]}"
+        # deterministic: a second call gives the same bits
+        y2 = M.spmv(torch.from_numpy(x).to(dev))
+        torch.cuda.synchronize()
+        assert torch.equal(y, y2)
+        M.close()
+
+
+def test_coo_pipe_config4_sampled(lib, dev, pipe_env):
+    """C4 (the config BRO_COO_KERNEL=0's auto choice sends to the pipelined
+    kernel) on 3,000 sampled rows, both dtypes."""
+    import bench
+    os.environ["BRO_COO_KERNEL"] = "0"
+    for dtype in (np.float64, np.float32):
+        A, _ = bench.load_workload("C4", dtype, lib)
+        M = lib.BroMatrix(A, fmt="hyb", codec=1, device=0, dtype=dtype)
+        x = make_x(A.n, 4, dtype)
+        y = M.spmv(torch.from_numpy(x).to(dev)).cpu().numpy()
+        rows = np.random.default_rng(5).integers(0, A.m, 3000)
+        yr, S = spmv.csr_spmv_rows(A.row_ptr, A.col, A.vals.astype(dtype), x, rows)
+        ok, _ = spmv.within_tolerance(y[rows], yr, S, TOL[dtype])
+        assert ok.all()
+        M.close()
