@@ -404,11 +404,13 @@ bool launch_bro_ell_bulk(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
 // 22.5 -> 18.5 us, fp32 20.5 -> 16.4 us).  BRO_ELL_FEW_G = 0 disables.
 template <typename T>
 constexpr int kEllFewG = sizeof(T) == 8 ? 16 : 32;
-// Window rows of the small-window instance: every row stream fits in
-// kEllSmallRows - 1 symbols (C5: S <= 7), so the per-warp symbol window
-// shrinks from 34 rows (4.3 KB) to 10 (1.3 KB): 12 KB less shared memory per
-// block, which the SM gives back to L1 for the x gather.
+// Window rows of the small-window instances: every row stream fits in
+// kRows - 1 symbols (C5: S <= 7), so the per-warp symbol window shrinks from
+// 34 rows (4.3 KB) to 10 (1.3 KB) or 18: up to 24 KB less shared memory per
+// block, which the SM gives back to L1 for the x gather (C5 fp64 349 -> 345
+// us, profiles/r01/s3/smallwin.txt).
 constexpr int kEllSmallRows = 10;
+constexpr int kEllMidRows = 18;  // S <= 17
 inline int64_t few_slices(bro_matrix_s* A) {
   static int64_t sms = 0;
   if (sms == 0) {
@@ -446,6 +448,8 @@ void launch_bro_ell(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cud
     launch_bro_ell_od<T, V, kEllWarps, 2, 16, 34>(A, x, y, st);
   else if (A->ell_max_S < kEllSmallRows && env_int("BRO_ELL_SMALLWIN", 1))
     launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks, 8, kEllSmallRows>(A, x, y, st);
+  else if (A->ell_max_S < kEllMidRows && env_int("BRO_ELL_SMALLWIN", 1))
+    launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks, 8, kEllMidRows>(A, x, y, st);
   else
     launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks>(A, x, y, st);
 }
