@@ -317,10 +317,10 @@ bro_status_t common_checks(bro_dtype_t dtype, const bro_opts_t* opts, bro_opts_t
 
 // Persistent grid: as many resident blocks as the SMs hold (queried once per
 // instantiation), capped by the number of slices.
-template <typename T, int V, int kWarps, int kMinBlocks, int G, int kRows, bool kMulti>
+template <typename T, int V, int kWarps, int kMinBlocks, int G, int kRows, bool kMulti, int kPf = 0>
 void launch_bro_ell_od_k(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cudaStream_t st) {
   using namespace bro::dev;
-  auto kern = bro_ell_spmv_od<T, V, kWarps, kMinBlocks, G, kRows, kMulti>;
+  auto kern = bro_ell_spmv_od<T, V, kWarps, kMinBlocks, G, kRows, kMulti, kPf>;
   static int resident = 0;
   if (resident == 0) {
     int per_sm = 0, sms = 0, dev = 0;
@@ -336,10 +336,10 @@ void launch_bro_ell_od_k(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
 }
 
 // single-destination instance unless the call scatters (bro_spmv_scatter)
-template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34>
+template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34, int kPf = 0>
 void launch_bro_ell_od(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cudaStream_t st) {
-  if (y.n > 1 || y.mc != nullptr) launch_bro_ell_od_k<T, V, kWarps, kMinBlocks, G, kRows, true>(A, x, y, st);
-  else launch_bro_ell_od_k<T, V, kWarps, kMinBlocks, G, kRows, false>(A, x, y, st);
+  if (y.n > 1 || y.mc != nullptr) launch_bro_ell_od_k<T, V, kWarps, kMinBlocks, G, kRows, true, kPf>(A, x, y, st);
+  else launch_bro_ell_od_k<T, V, kWarps, kMinBlocks, G, kRows, false, kPf>(A, x, y, st);
 }
 
 constexpr int kEllWarps = 8;      // slices per block
@@ -446,6 +446,10 @@ void launch_bro_ell(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cud
     launch_bro_ell_od<T, V, 4, 2, 32, 34>(A, x, y, st);
   else if (A->s < few_slices(A) && env_int("BRO_ELL_FEW_G", kEllFewG<T>) == 16)
     launch_bro_ell_od<T, V, kEllWarps, 2, 16, 34>(A, x, y, st);
+  else if (A->ell_max_S < kEllSmallRows && env_int("BRO_ELL_SMALLWIN", 1) && env_int("BRO_ELL_CPV", 0) == 1)
+    launch_bro_ell_od<T, V, 4, 8, 8, kEllSmallRows, 1>(A, x, y, st);
+  else if (A->ell_max_S < kEllSmallRows && env_int("BRO_ELL_SMALLWIN", 1) && env_int("BRO_ELL_CPV", 0) == 2)
+    launch_bro_ell_od<T, V, 4, 6, 8, kEllSmallRows, 2>(A, x, y, st);
   else if (A->ell_max_S < kEllSmallRows && env_int("BRO_ELL_SMALLWIN", 1))
     launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks, 8, kEllSmallRows>(A, x, y, st);
   else if (A->ell_max_S < kEllMidRows && env_int("BRO_ELL_SMALLWIN", 1))

@@ -136,6 +136,14 @@ __device__ __forceinline__ void store_y(const YOut<T>& o, int64_t row, T v) {
     if (i < o.n) o.p[i][row] = v;
 }
 
+// cp.async (LDGSTS) helpers
+__device__ __forceinline__ void cp_async4(uint32_t* dst, const uint32_t* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" :: "r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" :: "n"(N) : "memory"); }
+
 // shl with the PTX clamp (shift >= 32 gives 0)
 __device__ __forceinline__ uint32_t shl_clamp(uint32_t v, uint32_t s) {
   uint32_t r;
@@ -324,13 +332,43 @@ __device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __r
 // (G = 4, kRows = 6, 48 warps/SM) serves matrices whose slices all have
 // l <= 4 columns (<= 4 symbols per row): less shared memory and fewer
 // registers buy 1.5x the resident warps for the latency-bound short rows.
-template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34, bool kMulti = false>
+//
+// kPf > 0: values move by cp.async (LDGSTS, no registers while in flight)
+// into a per-warp ring of kPf + 1 group slots laid out exactly like the
+// global chunks; groups 0 .. kPf-1 of a slice are issued before its widths
+// and symbols are staged, so the value stream overlaps that round trip, and
+// group g + kPf is issued while group g is decoded.
+template <typename T, int G>
+__device__ __forceinline__ void cp_async_group_vals(T* slot, const T* vs, int j, int l, int lfull, int lane) {
+  constexpr int VV = Chunk<T>::N;
+#pragma unroll
+  for (int u = 0; u < G / VV; ++u) {
+    const int jj = j + u * VV;
+    T* d = slot + u * 32 * VV + lane * VV;
+    if (jj + VV <= lfull) {
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(smem_u32(d)), "l"(vs + 32 * jj + lane * VV)
+                   : "memory");
+    } else if (jj < l) {
+      const int tw = l - lfull;  // tail slots per lane (< VV), contiguous per lane
+#pragma unroll
+      for (int k = 0; k < VV; ++k)
+        if (jj + k < l)
+          asm volatile("cp.async.ca.shared.global [%0], [%1], %2;"
+                       :: "r"(smem_u32(d + k)), "l"(vs + 32 * lfull + lane * tw + (jj + k - lfull)), "n"(sizeof(T))
+                       : "memory");
+    }
+  }
+}
+
+template <typename T, int V, int kWarps, int kMinBlocks, int G = 8, int kRows = 34, bool kMulti = false, int kPf = 0>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
                 const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
                 const uint64_t* __restrict__ symptr, const T* __restrict__ vals,
                 const T* __restrict__ x, const YOut<T> y) {
   struct Meta { uint64_t c0, q0; int l, S; };
+  constexpr int kNV = kPf + 1;
+  __shared__ __align__(16) T vring[kPf ? kWarps : 1][kPf ? kNV * G * 32 : 1];
   __shared__ uint32_t window[kWarps][kRows * 32];
   __shared__ uint2 colmeta[kWarps][32];  // per column of the block: {byte offset of its word row, r | (32-b) << 8}
   __shared__ Meta metas[kWarps][32];     // metadata of this warp's next 32 slices
@@ -362,6 +400,13 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
     T sum = T(0);
     int col = -1;
     int obase = 0;  // bit offset of the current block inside every row stream
+    if constexpr (kPf > 0) {  // first groups' values in flight before the staging round trip
+#pragma unroll
+      for (int p = 0; p < kPf; ++p) {
+        if (p * G < l) cp_async_group_vals<T, G>(vring[w] + (p % kNV) * G * 32, vs, p * G, l, lfull, lane);
+        cp_async_commit();
+      }
+    }
     for (int jb = 0; jb < l; jb += 32) {
       const int nb = min(32, l - jb);
       const int b = lane < nb ? int(__ldg(ba + jb + lane)) : 0;
@@ -389,7 +434,26 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
       __syncwarp();
       for (int g = 0; g < nb; g += G) {
         T v[G];
-        load_vals<T, G>(v, vs, jb + g, l, lfull, lane);
+        if constexpr (kPf > 0) {
+          const int gi = (jb + g) / G;  // group index within the slice
+          const int jn = jb + g + kPf * G;
+          if (jn < l) cp_async_group_vals<T, G>(vring[w] + ((gi + kPf) % kNV) * G * 32, vs, jn, l, lfull, lane);
+          cp_async_commit();
+          cp_async_wait<kPf>();
+          const T* sl = vring[w] + (gi % kNV) * G * 32 + lane * Chunk<T>::N;
+#pragma unroll
+          for (int u = 0; u < G / Chunk<T>::N; ++u) {
+            if constexpr (sizeof(T) == 8) {
+              const double2 c2 = *reinterpret_cast<const double2*>(sl + u * 32 * Chunk<T>::N);
+              v[2 * u] = c2.x; v[2 * u + 1] = c2.y;
+            } else {
+              const float4 c4 = *reinterpret_cast<const float4*>(sl + u * 32 * Chunk<T>::N);
+              v[4 * u] = c4.x; v[4 * u + 1] = c4.y; v[4 * u + 2] = c4.z; v[4 * u + 3] = c4.w;
+            }
+          }
+        } else {
+          load_vals<T, G>(v, vs, jb + g, l, lfull, lane);
+        }
         int cidx[G];
         bool ok[G];
 #pragma unroll
@@ -914,12 +978,6 @@ coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restri
 // (base row, width, first word) of the warp's next 32 intervals is fetched
 // lane-parallel into shared memory.  One work unit (carry pair) per warp:
 // rows continue across the warp's intervals, so the fix-up sees nW units.
-__device__ __forceinline__ void cp_async4(uint32_t* dst, const uint32_t* src) {
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" :: "r"(smem_u32(dst)), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" :: "n"(N) : "memory"); }
 
 constexpr int kCooPipeRows = 10;  // window rows per batch buffer (<= 9 used)
 

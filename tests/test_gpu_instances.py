@@ -1,8 +1,10 @@
-"""GPU: the persistent pipelined (BRO-)COO kernel (coo_spmv_pipe) against the
-oracle on cases that span many intervals, a ragged last interval, rows that
-cross intervals and warps, and long rows (-m gpu).  BRO_COO_KERNEL=2 forces
-it wherever there are >= 8 intervals; BRO_COO_PIPE_MINB picks the register
-budget (2: 16 warps/SM, 3: 24 warps/SM)."""
+"""GPU: kernel instances chosen by size or by tuning variables, against the
+oracle (-m gpu): the persistent pipelined (BRO-)COO kernel (coo_spmv_pipe;
+BRO_COO_KERNEL=2 forces it wherever there are >= 8 intervals,
+BRO_COO_PIPE_MINB picks 16 or 24 warps/SM) on cases spanning many intervals,
+a ragged last interval, rows crossing intervals and warps, and long rows; and
+the general BRO-ELL instances a large matrix can take (window rows, cp.async
+value ring)."""
 import os
 
 import numpy as np
@@ -89,3 +91,37 @@ def test_coo_pipe_config4_sampled(lib, dev, pipe_env):
         ok, _ = spmv.within_tolerance(y[rows], yr, S, TOL[dtype])
         assert ok.all()
         M.close()
+
+
+@pytest.fixture
+def ell_env():
+    keys = ("BRO_ELL_CPV", "BRO_ELL_SMALLWIN", "BRO_ELL_FEW_G")
+    old = {k: os.environ.get(k) for k in keys}
+    yield
+    for k, v in old.items():
+        if v is None:
+            os.environ.pop(k, None)
+        else:
+            os.environ[k] = v
+
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+@pytest.mark.parametrize("env", ["BRO_ELL_SMALLWIN=0", "BRO_ELL_SMALLWIN=1", "BRO_ELL_CPV=1", "BRO_ELL_CPV=2"])
+def test_bro_ell_instances_stencil(lib, dev, ell_env, dtype, env):
+    """The general BRO-ELL instances a large matrix can take (34-row window,
+    10-row small window, cp.async value ring with 1 or 2 groups ahead) on a
+    27-point stencil big enough to fill the GPU (6,750 slices, S <= 7),
+    every row against the oracle."""
+    from gen.matrices import stencil_27pt
+    A = stencil_27pt(60)
+    k, v = env.split("=")
+    os.environ[k] = v
+    M = lib.BroMatrix(A, fmt="ell", codec=1, device=0, dtype=dtype)
+    assert M.info["n_slices"] >= 148 * 32
+    x = make_x(A.n, 6, dtype)
+    y = M.spmv(torch.from_numpy(x).to(dev))
+    torch.cuda.synchronize()
+    y_ref, S = spmv.csr_spmv(A.row_ptr, A.col, A.vals.astype(dtype), x)
+    ok, err = spmv.within_tolerance(y.cpu().numpy(), y_ref, S, TOL[dtype])
+    assert ok.all(), f"{np.count_nonzero(~ok)} rows out of tolerance"
+    M.close()
