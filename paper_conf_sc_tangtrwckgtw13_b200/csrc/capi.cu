@@ -396,6 +396,30 @@ bool launch_bro_ell_bulk(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
   return launch_bro_ell_bulk_g<T, 32>(A, x, y, st);
 }
 
+// Tiny slices (every slice <= 4 columns): register-resident decode, kSl
+// slices interleaved per warp iteration.  Default (BRO_ELL_TINY = 1, one
+// slice per iteration at 40-48 warps/SM): C3's ELL part, BRO-HYB f64 42.0 ->
+// 35.9 us (profiles/r01/s3/tiny.txt); 2 = two slices interleaved (slower:
+// 40.0 us); 0 = the short-slice instance of the offset-decode kernel.
+template <typename T, int V, int kMinBlocks, int kSl>
+void launch_bro_ell_tiny(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cudaStream_t st) {
+  using namespace bro::dev;
+  constexpr int kW = 8;
+  auto kern = bro_ell_spmv_tiny<T, V, kW, kMinBlocks, kSl>;
+  static int resident = 0;
+  if (resident == 0) {
+    int per_sm = 0, sms = 0, dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kW * 32, 0);
+    resident = std::max(1, per_sm) * std::max(1, sms);
+  }
+  const int64_t need = (A->s + kW * kSl - 1) / (kW * kSl);
+  const unsigned grid = (unsigned)std::min<int64_t>(need, resident);
+  kern<<<grid, kW * 32, 0, st>>>(A->m, A->s, A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr,
+                                 (const T*)A->d_ell_vals, x, y);
+}
+
 // Few slices (fewer than the 32 warps/SM of the general instance can hold,
 // e.g. C2: 1,951 slices of up to 81 columns): every warp is resident anyway,
 // so spend registers on more columns in flight per warp instead: G = 16 at
@@ -440,6 +464,10 @@ void launch_bro_ell(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cud
     launch_bro_ell_od<T, V, 4, 4, 16, 34>(A, x, y, st);
   else if (variant == 5)
     launch_bro_ell_od<T, V, 4, 2, 32, 34>(A, x, y, st);
+  else if (A->ell_max_l <= 4 && y.n == 1 && y.mc == nullptr && env_int("BRO_ELL_TINY", 1) == 1)
+    launch_bro_ell_tiny<T, V, sizeof(T) == 8 ? 5 : 6, 1>(A, x, y, st);
+  else if (A->ell_max_l <= 4 && y.n == 1 && y.mc == nullptr && env_int("BRO_ELL_TINY", 1) == 2)
+    launch_bro_ell_tiny<T, V, sizeof(T) == 8 ? 3 : 4, 2>(A, x, y, st);
   else if (A->ell_max_l <= 4 && env_int("BRO_ELL_SHORT", 1))
     launch_bro_ell_od<T, V, kEllWarps, sizeof(T) == 8 ? kEllMinBlocksShort - 1 : kEllMinBlocksShort, 4, 6>(A, x, y, st);
   else if (A->s < few_slices(A) && env_int("BRO_ELL_FEW_G", kEllFewG<T>) == 32)

@@ -481,6 +481,96 @@ bro_ell_spmv_od(int64_t m, int64_t s, const uint32_t* __restrict__ words,
   }
 }
 
+// ------------------------------------------------------------------ BRO-ELL, tiny slices
+// Every slice has l <= 4 columns (e.g. the ELL part of C3's BRO-HYB, K = 2),
+// so a row stream has S <= 4 symbols (<= 4 fields of <= 32 bits): each lane
+// keeps its <= 4 words in registers — no shared-memory window, no width
+// scan, no column records.  Per slice one round trip fetches the widths
+// (broadcast), the lane's words and its values together, then one fetches
+// the x gathers; kSl slices are processed interleaved per warp iteration so
+// their round trips overlap.  Field j starts at the warp-uniform offset
+// o_j = b_0 + ... + b_{j-1}, so q = o_j / 32 selects the word pair uniformly.
+template <typename T, int V, int kWarps, int kMinBlocks, int kSl>
+__global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
+bro_ell_spmv_tiny(int64_t m, int64_t s, const uint32_t* __restrict__ words,
+                  const uint8_t* __restrict__ bit_alloc, const uint64_t* __restrict__ colptr,
+                  const uint64_t* __restrict__ symptr, const T* __restrict__ vals,
+                  const T* __restrict__ x, const YOut<T> y) {
+  struct Meta { uint64_t c0, q0; int l, S; };
+  __shared__ Meta metas[kWarps][32];  // metadata of this warp's next 32 slices
+  const int lane = threadIdx.x & 31;
+  const int w = threadIdx.x >> 5;
+  const int64_t stride = int64_t(gridDim.x) * kWarps;
+  int k32 = 0;
+  for (int64_t t0 = int64_t(blockIdx.x) * kWarps + w; t0 < s; t0 += kSl * stride) {
+    int l[kSl], S[kSl];
+    uint32_t wd[kSl][5];
+    T v[kSl][4];
+    int bw[kSl][4];
+    bool live[kSl];
+#pragma unroll
+    for (int u = 0; u < kSl; ++u) {
+      const int64_t t = t0 + u * stride;
+      live[u] = t < s;
+      if (k32 == 0) {  // one round trip fetches the metadata of the next 32 slices
+        __syncwarp();
+        const int64_t tl = t + lane * stride;
+        if (tl < s) {
+          const uint64_t c0l = __ldg(colptr + tl), q0l = __ldg(symptr + tl);
+          metas[w][lane] = Meta{c0l, q0l, int(__ldg(colptr + tl + 1) - c0l), int(__ldg(symptr + tl + 1) - q0l)};
+        }
+        __syncwarp();
+      }
+      const Meta mt = metas[w][k32];
+      k32 = (k32 + 1) & 31;
+      l[u] = live[u] ? mt.l : 0;
+      S[u] = live[u] ? mt.S : 0;
+      const uint32_t* wb = words + 32 * mt.q0;
+      const uint8_t* ba = bit_alloc + mt.c0;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) bw[u][j] = j < l[u] ? int(__ldg(ba + j)) : 0;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) wd[u][q] = q < S[u] ? __ldg(wb + place(lane, q, S[u], V)) : 0u;
+      wd[u][4] = 0u;
+      const int lfull = (l[u] / Chunk<T>::N) * Chunk<T>::N;
+      if (l[u] > 0) load_group_vals<T, 4>(v[u], vals + 32 * mt.c0, 0, l[u], lfull, lane);
+    }
+    int cidx[kSl][4];
+    bool ok[kSl][4];
+#pragma unroll
+    for (int u = 0; u < kSl; ++u) {
+      int col = -1, o = 0;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int b = bw[u][j];
+        const int q = o >> 5;
+        const uint32_t hi = q == 0 ? wd[u][0] : q == 1 ? wd[u][1] : q == 2 ? wd[u][2] : wd[u][3];
+        const uint32_t lo = q == 0 ? wd[u][1] : q == 1 ? wd[u][2] : q == 2 ? wd[u][3] : wd[u][4];
+        const uint32_t d = shr_clamp(__funnelshift_l(lo, hi, uint32_t(o & 31)), uint32_t(32 - b));
+        col += int(d);
+        cidx[u][j] = col;
+        ok[u][j] = d != 0u;  // padding (and j >= l: b = 0) is skipped, Alg. 1 line 17
+        o += b;
+      }
+    }
+    T xv[kSl][4];
+#pragma unroll
+    for (int u = 0; u < kSl; ++u)
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        if (ok[u][j]) xv[u][j] = ldg_x(x + cidx[u][j]);
+#pragma unroll
+    for (int u = 0; u < kSl; ++u) {
+      T sum = T(0);
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        if (ok[u][j]) sum = fma(v[u][j], xv[u][j], sum);
+      const int64_t row = 32 * (t0 + u * stride) + lane;
+      if (live[u] && row < m) store_y<false>(y, row, sum);
+    }
+  }
+}
+
 // ------------------------------------------------------------------ BRO-ELL, bulk-staged
 // Same offset decode, but every byte of a slice (its values, its symbol
 // stream in the paper's V = 1 multiplexing comp_str[q*h + tid], and
@@ -1158,6 +1248,41 @@ __global__ void replicate_y(int64_t m, const YOut<T> o) {
 // fixed summation order = unit order).  first[u] / last[u] = rows of the
 // unit's first and last entries; cf = partial of the first row (the whole
 // unit if first == last), cl = partial of the last row.
+// acc += cf[j] for the units j = i+1, i+2, ... that continue row R (first[j]
+// == R), stopping after the first of them that ends on another row.  Units
+// are read 8 at a time, so a row spanning up to 9 units costs one round trip
+// instead of one per unit; the additions stay in unit order.
+template <typename T>
+__device__ __forceinline__ T chain_sum(int64_t i, int64_t nU, int R, T acc, const int32_t* __restrict__ first,
+                                       const int32_t* __restrict__ last_row, const T* __restrict__ cf) {
+  constexpr int B = 8;
+  for (int64_t j0 = i + 1; j0 < nU; j0 += B) {
+    int fj[B], lj[B];
+    T cj[B];
+#pragma unroll
+    for (int k = 0; k < B; ++k) {
+      const bool in = j0 + k < nU;
+      fj[k] = in ? first[j0 + k] : -1;
+      lj[k] = in ? last_row[j0 + k] : -1;
+      cj[k] = in ? cf[j0 + k] : T(0);
+    }
+    bool done = false;
+#pragma unroll
+    for (int k = 0; k < B; ++k) {
+      if (!done) {
+        if (fj[k] != R) {
+          done = true;
+        } else {
+          acc += cj[k];
+          done = lj[k] != R;
+        }
+      }
+    }
+    if (done) break;
+  }
+  return acc;
+}
+
 template <typename T>
 __global__ void coo_fixup(int64_t nU, const int32_t* __restrict__ first,
                           const int32_t* __restrict__ last_row, const T* __restrict__ cf,
@@ -1166,24 +1291,10 @@ __global__ void coo_fixup(int64_t nU, const int32_t* __restrict__ first,
   if (i >= nU) return;
   const int F = first[i];
   const int L = last_row[i];
-  if (L != F) {  // unit i is the first one holding row L
-    T acc = cl[i];
-    for (int64_t j = i + 1; j < nU && first[j] == L; ++j) {
-      acc += cf[j];
-      if (last_row[j] != L) break;
-    }
-    y[L] += acc;
-  }
-  if (i == 0 || last_row[i - 1] != F) {  // unit i is the first one holding row F
-    T acc = cf[i];
-    if (L == F) {
-      for (int64_t j = i + 1; j < nU && first[j] == F; ++j) {
-        acc += cf[j];
-        if (last_row[j] != F) break;
-      }
-    }
-    y[F] += acc;
-  }
+  if (L != F)  // unit i is the first one holding row L
+    y[L] += chain_sum<T>(i, nU, L, cl[i], first, last_row, cf);
+  if (i == 0 || last_row[i - 1] != F)  // unit i is the first one holding row F
+    y[F] += L == F ? chain_sum<T>(i, nU, F, cf[i], first, last_row, cf) : cf[i];
 }
 
 template <int V>

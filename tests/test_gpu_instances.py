@@ -95,7 +95,7 @@ def test_coo_pipe_config4_sampled(lib, dev, pipe_env):
 
 @pytest.fixture
 def ell_env():
-    keys = ("BRO_ELL_CPV", "BRO_ELL_SMALLWIN", "BRO_ELL_FEW_G")
+    keys = ("BRO_ELL_CPV", "BRO_ELL_SMALLWIN", "BRO_ELL_FEW_G", "BRO_ELL_TINY")
     old = {k: os.environ.get(k) for k in keys}
     yield
     for k, v in old.items():
@@ -125,3 +125,34 @@ def test_bro_ell_instances_stencil(lib, dev, ell_env, dtype, env):
     ok, err = spmv.within_tolerance(y.cpu().numpy(), y_ref, S, TOL[dtype])
     assert ok.all(), f"{np.count_nonzero(~ok)} rows out of tolerance"
     M.close()
+
+
+TINY_CASES = [
+    ("short", lambda: random_csr(20000, 30000, 31, max_len=4, empty_frac=0.2)),
+    ("wide", lambda: random_csr(9000, 2**31 - 1, 32, max_len=4, wide_cols=True)),
+    ("ragged_m", lambda: random_csr(7777, 5000, 33, max_len=3, empty_frac=0.5)),
+]
+
+
+@pytest.mark.parametrize("name,mk", TINY_CASES, ids=[c[0] for c in TINY_CASES])
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+@pytest.mark.parametrize("tiny", ["1", "2"])
+def test_bro_ell_tiny_slices(lib, dev, ell_env, name, mk, dtype, tiny):
+    """The register-resident tiny-slice BRO-ELL kernel (every slice <= 4
+    columns; BRO_ELL_TINY = 1: one slice per warp iteration, 2: two
+    interleaved) for V = 1, 2, 4, including 31-bit first deltas, empty rows and
+    m not a multiple of 32; every row against the oracle."""
+    A = mk()
+    os.environ["BRO_ELL_TINY"] = tiny
+    x = make_x(A.n, 7, dtype)
+    y_ref, S = spmv.csr_spmv(A.row_ptr, A.col, A.vals.astype(dtype), x)
+    xd = torch.from_numpy(x).to(dev)
+    for V in (1, 2, 4):
+        M = lib.BroMatrix(A, fmt="ell", codec=1, device=0, dtype=dtype, vec_words=V)
+        assert M.info["K"] <= 4
+        y = M.spmv(xd)
+        torch.cuda.synchronize()
+        ok, err = spmv.within_tolerance(y.cpu().numpy(), y_ref, S, TOL[dtype])
+        assert ok.all(), f"V={V}: {np.count_nonzero(~ok)} rows out of tolerance"
+        M.close()
+    os.environ.pop("BRO_ELL_TINY", None)
