@@ -584,6 +584,8 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
   if (A->has_coo && A->nI > 0) {
     const int warps = kCooThreads / 32;
     int upi = std::max(1, std::min(kCooMaxUpi, env_int("BRO_COO_UPI", kCooUpi)));
+    const int upi_log2 = upi >= 4 ? 2 : upi >= 2 ? 1 : 0;
+    upi = 1 << upi_log2;
     int64_t nU = A->nI * upi;
     // BRO_COO_KERNEL: 1 (default) per-unit kernel; 2 persistent pipelined
     // kernel (opt-in: measured no faster); 0 auto =
@@ -598,10 +600,10 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
     const int T_ = A->opts.coo_T;
     if (upi > 0) {
     auto args = [&](auto kern) {
-      kern<<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, upi, A->d_coo_words, A->d_coo_base,
+      kern<<<grid, kCooThreads, 0, st>>>(A->nnz_coo, A->nI, T_, upi_log2, A->d_coo_words, A->d_coo_base,
                                          A->d_coo_width, A->d_coo_symptr, A->d_coo_row, A->d_coo_col,
                                          (const T*)A->d_coo_vals, x, y, (T*)A->d_cf, (T*)A->d_cl,
-                                         A->d_first_row, A->d_last_row);
+                                         A->d_first_row, A->d_last_row, env_int("BRO_COO_L2PF", 0));
     };
     // BRO_COO_MINB=4: 64-register instances (32 resident warps/SM; tuning sweeps)
     const bool minb4 = env_int("BRO_COO_MINB", 0) == 4;

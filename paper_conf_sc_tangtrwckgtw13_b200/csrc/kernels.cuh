@@ -942,26 +942,30 @@ __device__ __forceinline__ void coo_segments(const int* r, const int* c, const T
 
 template <typename T, int V, bool kBro, int kThreads, int kMinBlocks = 0>
 __global__ void __launch_bounds__(kThreads, kMinBlocks)
-coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi, const uint32_t* __restrict__ words,
+coo_spmv(int64_t nnz, int64_t nI, int T_steps, int upi_log2, const uint32_t* __restrict__ words,
          const uint32_t* __restrict__ base_row, const uint8_t* __restrict__ width,
          const uint64_t* __restrict__ symptr, const int32_t* __restrict__ rows,
          const int32_t* __restrict__ col, const T* __restrict__ vals, const T* __restrict__ x,
          T* __restrict__ y, T* __restrict__ carry_first, T* __restrict__ carry_last,
-         int32_t* __restrict__ first_row, int32_t* __restrict__ last_row) {
+         int32_t* __restrict__ first_row, int32_t* __restrict__ last_row, int l2_prefetch) {
   constexpr int TB = 8;
   __shared__ __align__(16) int32_t rowbuf[kThreads / 32][TB * 32];
   __shared__ uint32_t cwin[kThreads / 32][kBro ? 33 * 32 : 1];  // lane word rows (+ zero guard row)
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
-  // work unit = steps [ts, ts + T_steps / upi) of interval i (upi units per interval)
+  // work unit = steps [ts, ts + T_steps / upi) of interval i (upi = 2^upi_log2
+  // units per interval; shifts, not 64-bit divisions)
   const int64_t u = int64_t(blockIdx.x) * (kThreads / 32) + w;
-  const int64_t i = u / upi;
+  const int64_t i = u >> upi_log2;
   if (i >= nI) return;
-  const int steps = T_steps / upi;
-  const int ts = int(u - i * upi) * steps;
+  const int steps = T_steps >> upi_log2;
+  const int ts = int(u & ((int64_t(1) << upi_log2) - 1)) * steps;
   int32_t* rb = rowbuf[w];
   const int64_t e0 = i * 32 * T_steps;
-  if (lane == 0) {  // L2 prefetch (TMA engine) of the unit's batches after the first one
+  // optional L2 prefetch (TMA engine) of the unit's batches after the first
+  // one (BRO_COO_L2PF=1): measured slower, C4 BRO-HYB f64 115.2 vs 111.2 us
+  // (profiles/r01/s3/coo_l2pf.txt), so off by default
+  if (l2_prefetch && lane == 0) {
     const int64_t p0 = e0 + 32 * (ts + TB);
     const int64_t p1 = min(e0 + 32 * int64_t(ts + steps), nnz) & ~int64_t(3);
     if (p1 > p0) {
