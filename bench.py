@@ -186,9 +186,10 @@ def time_steps(fn, steps, warmup, stream, flush=None):
 
 
 def read_ceiling(dev, gib=2, reps=5):
-    """Practical read-only HBM ceiling on this box: best-of-N
-    torch.sum over a 2 GiB fp32 buffer, CUDA events (context for the
-    roofline, whose denominator stays the driver-measured copy bandwidth)."""
+    """A read-only streaming kernel on this box: best-of-N
+    torch.sum over a 2 GiB fp32 buffer, CUDA events.  Context only — the
+    roofline's denominator stays the driver-measured copy bandwidth, and the
+    in-repo ELLPACK kernel streams faster than this library reduction."""
     import torch
     buf = torch.ones(gib * 2**30 // 4, dtype=torch.float32, device=dev)
     best = None
@@ -494,7 +495,8 @@ def main():
                                            "bro_ell_spmv + coo_spmv + coo_fixup"),
                      "algorithmic_bytes_per_launch": alg_bytes, "kernel_ms": kern_ms,
                      "frac_of_8TBps_spec": achieved / 8000.0,
-                     "read_ceiling_GBps": rc, "frac_of_read_ceiling": achieved / rc if rc else None},
+                     "read_stream_GBps": rc, "read_stream_how": "torch.sum over 2 GiB fp32 (a library "
+                     "reduction, context only: the in-repo ELLPACK streams faster)" if rc else None},
         "uncompressed": {"format": {"ell": "ELLPACK", "hyb": "HYB", "coo": "COO"}[fmt], "value": base_value,
                          "unit": "GFLOP/s", "kernel_ms": base_kern_ms,
                          "algorithmic_bytes": binfo["algorithmic_bytes"],
