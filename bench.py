@@ -102,18 +102,22 @@ class ClockSampler:
 
     def start(self):
         import tempfile
-        self.path = tempfile.mktemp(suffix=".csv")
+        fd, self.path = tempfile.mkstemp(suffix=".csv")
+        self._out = os.fdopen(fd, "w")
         q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active")
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}", "--format=csv,noheader,nounits",
-                 "-lms", "50"], stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+                 "-lms", "50"], stdout=self._out, stderr=subprocess.DEVNULL)
             time.sleep(0.4)
         except (OSError, FileNotFoundError):
             self.proc = None
 
     def stop(self):
         if self.proc is None:
+            if self.path:
+                self._out.close()
+                os.unlink(self.path)
             return None
         time.sleep(0.1)
         self.proc.terminate()
@@ -121,6 +125,7 @@ class ClockSampler:
             self.proc.wait(timeout=5)
         except subprocess.TimeoutExpired:
             self.proc.kill()
+        self._out.close()
         rows = []
         with open(self.path) as f:
             for line in f:
@@ -346,7 +351,15 @@ def main():
                            vec_words=args.vec_words)
         base = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=0, dtype=dtype, bounds=bounds)
     info, binfo = blk.mat.info, base.mat.info
-    launches = (0 if fmt == "coo" else 1) + (2 if info["nnz_coo"] else 0)  # ELL kernel, COO kernel + fix-up
+    # our kernels per step: ELL kernel, COO kernel + fix-up; the overlap
+    # exchange runs one SpMV per row part (interior / head / tail); a
+    # HYB/COO handle scattering to peers adds its replicate kernel
+    per_spmv = (0 if fmt == "coo" else 1) + (2 if info["nnz_coo"] else 0)
+    launches = per_spmv
+    if world > 1 and blk.exchange == "overlap":
+        launches = sum((0 if fmt == "coo" else 1) + (2 if p.info["nnz_coo"] else 0) for _, _, p in blk.parts)
+    elif world > 1 and blk.exchange == "p2p" and info["nnz_coo"]:
+        launches = per_spmv + 1
     flush_buf = torch.empty(2 * L2_BYTES // 4, dtype=torch.int32, device=dev) if args.flush_l2 else None
     flush = (lambda: flush_buf.fill_(1)) if args.flush_l2 else None
     y1 = torch.empty(A.m, dtype=tdt, device=dev) if world == 1 else None
