@@ -195,7 +195,13 @@ bro_status_t bro_spmv_scatter(bro_matrix_t A, const void* x_dev, void* const* y_
 
 /* End-to-end y = A.x with HOST vectors: copies x (n values) host->device,
  * runs bro_spmv, copies y (m values) device->host and synchronizes `stream`.
- * Pinned host memory gives full PCIe bandwidth; pageable memory works. */
+ * Pinned host memory gives full PCIe bandwidth; pageable memory works.
+ * ELL-only handles (BRO-ELL, ELLPACK) pipeline the three steps: x goes up in
+ * pieces on an internal stream, each block of rows runs on `stream` as soon
+ * as the pieces covering its columns have arrived, and its y goes down on a
+ * second internal stream while later blocks compute (environment variable
+ * BRO_E2E_CHUNKS = pieces, default 8; 1 = serial).  The result is identical
+ * to bro_spmv's.  Returns after all of it has completed. */
 bro_status_t bro_spmv_host(bro_matrix_t A, const void* x_host, void* y_host, bro_stream_t stream);
 
 /* Release the handle and all of its memory.  NULL is accepted. */

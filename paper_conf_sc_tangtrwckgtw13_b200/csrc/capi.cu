@@ -3,6 +3,7 @@
 
 #include <algorithm>
 #include <chrono>
+#include <climits>
 #include <cstdlib>
 #include <cstring>
 #include <new>
@@ -23,6 +24,7 @@ bro_status_t fail(bro_status_t s, const std::string& msg) {
 }
 
 constexpr int kCooThreads = 256;
+constexpr int kE2eChunks = 8;  // pieces of the pipelined bro_spmv_host
 constexpr int kBarWindow = 64;  // candidate partitions of BAR method 2 (windowed Algorithm 2)
 constexpr int kCooMaxUpi = 4;   // work units per COO interval (8 steps = 256 entries each at 4)
 constexpr int kCooUpi = 2;
@@ -79,6 +81,11 @@ struct bro_matrix_s {
   void* d_ys = nullptr;
   int64_t device_bytes = 0;
   uint32_t bulk_unit_max = 0;
+  // end-to-end pipeline of ELL-only handles (bro_spmv_host): column range of
+  // every 32-row block, side streams and events (created on first use)
+  std::vector<int32_t> blk_cmin, blk_cmax;
+  cudaStream_t e2e_h2d = nullptr, e2e_d2h = nullptr;
+  std::vector<cudaEvent_t> e2e_ev;
   int64_t ell_max_S = 0;       // most 32-bit symbols in one BRO-ELL row stream
   int64_t ell_max_l = 0;       // longest BRO-ELL slice (columns)  // largest staged slice of the bulk BRO-ELL kernel (bytes)
   bro_info_t info{};
@@ -115,6 +122,9 @@ void free_device(bro_matrix_s* A) {
                 A->d_coo_col, A->d_coo_vals, A->d_cf, A->d_cl, A->d_last_row, A->d_first_row, A->d_xs, A->d_ys};
   for (void* p : ps)
     if (p) cudaFree(p);
+  for (cudaEvent_t e : A->e2e_ev) cudaEventDestroy(e);
+  if (A->e2e_h2d) cudaStreamDestroy(A->e2e_h2d);
+  if (A->e2e_d2h) cudaStreamDestroy(A->e2e_d2h);
 }
 
 bro_status_t check_opts(const bro_opts_t& o) {
@@ -240,6 +250,19 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
         bro::build_plain_coo(A->nnz_coo, cr.data(), cc.data(), cv.data(), A->vsize, o.coo_T, A->coo);
       A->nI = A->coo.nI;
       A->coo_words = (int64_t)A->coo.words.size();
+    }
+    // column range of every 32-row block (ELL-only handles): which part of x
+    // a block of rows needs, for the pipelined bro_spmv_host
+    if (A->has_ell && !A->has_coo) {
+      const int64_t nb = (m + 31) / 32;
+      A->blk_cmin.assign(nb, INT32_MAX);
+      A->blk_cmax.assign(nb, -1);
+      for (int64_t i = 0; i < m; ++i) {
+        if (row_ptr[i + 1] == row_ptr[i]) continue;
+        const int64_t bi = i / 32;
+        A->blk_cmin[bi] = std::min(A->blk_cmin[bi], col[row_ptr[i]]);
+        A->blk_cmax[bi] = std::max(A->blk_cmax[bi], col[row_ptr[i + 1] - 1]);
+      }
     }
   } catch (const std::bad_alloc&) {
     delete A;
@@ -664,6 +687,101 @@ PartView part_view(bro_matrix_s* A, int32_t part) {
 
 }  // namespace
 
+namespace {
+
+// y = A.x over 32-row blocks [b0, b1) only: the ELL arrays are addressed
+// through the block range (slice metadata / plain ELL rows offset by b0, y
+// offset by 32*b0), the kernels are unchanged.  ELL-only handles.
+template <typename T>
+bro_status_t launch_spmv_blocks(bro_matrix_s* A, const T* x, T* y, int64_t b0, int64_t b1, cudaStream_t st) {
+  const int64_t m0 = A->m, s0 = A->s;
+  uint64_t* const cp0 = A->d_colptr;
+  uint64_t* const sp0 = A->d_symptr;
+  int32_t* const pc0 = A->d_pell_col;
+  void* const pv0 = A->d_ell_vals;
+  A->m = std::min(m0, 32 * b1) - 32 * b0;
+  if (A->opts.codec) {
+    A->s = b1 - b0;
+    A->d_colptr = cp0 + b0;
+    A->d_symptr = sp0 + b0;
+  } else {
+    A->d_pell_col = pc0 + 32 * b0;
+    A->d_ell_vals = static_cast<char*>(pv0) + size_t(32 * b0) * A->vsize;
+  }
+  const bro_status_t r = launch_spmv<T>(A, x, make_yout(y + 32 * b0), st);
+  A->m = m0; A->s = s0; A->d_colptr = cp0; A->d_symptr = sp0; A->d_pell_col = pc0; A->d_ell_vals = pv0;
+  return r;
+}
+
+// Pipelined end-to-end SpMV of an ELL-only handle: x goes up in K pieces on
+// one stream, each block of rows runs as soon as the pieces covering its
+// columns (blk_cmin/blk_cmax) have arrived, and its y goes down on a third
+// stream while later blocks compute — H2D, compute and D2H overlap (PCIe is
+// full duplex).  Same kernels and per-row arithmetic as bro_spmv.
+bro_status_t spmv_host_pipelined(bro_matrix_s* A, const void* x_host, void* y_host, cudaStream_t st, int K) {
+  const int64_t nb = (A->m + 31) / 32;
+  const size_t vs = size_t(A->vsize);
+  cudaError_t e = cudaSuccess;
+  if (!A->e2e_h2d) {
+    if ((e = cudaStreamCreateWithFlags(&A->e2e_h2d, cudaStreamNonBlocking)) != cudaSuccess ||
+        (e = cudaStreamCreateWithFlags(&A->e2e_d2h, cudaStreamNonBlocking)) != cudaSuccess)
+      return fail(BRO_ERR_CUDA, std::string("stream create: ") + cudaGetErrorString(e));
+  }
+  while ((int)A->e2e_ev.size() < 2 * K + 1) {
+    cudaEvent_t ev;
+    if ((e = cudaEventCreateWithFlags(&ev, cudaEventDisableTiming)) != cudaSuccess)
+      return fail(BRO_ERR_CUDA, std::string("event create: ") + cudaGetErrorString(e));
+    A->e2e_ev.push_back(ev);
+  }
+  cudaEvent_t* evx = A->e2e_ev.data();
+  cudaEvent_t* evy = evx + K;
+  cudaEvent_t start = evx[2 * K];
+  auto xa = [&](int i) { return A->n * i / K; };
+  // the side streams start after earlier work on the caller's stream
+  cudaEventRecord(start, st);
+  cudaStreamWaitEvent(A->e2e_h2d, start, 0);
+  cudaStreamWaitEvent(A->e2e_d2h, start, 0);
+  for (int i = 0; i < K; ++i) {
+    const int64_t a = xa(i), b = xa(i + 1);
+    if (b > a)
+      e = cudaMemcpyAsync(static_cast<char*>(A->d_xs) + a * vs, static_cast<const char*>(x_host) + a * vs,
+                          size_t(b - a) * vs, cudaMemcpyHostToDevice, A->e2e_h2d);
+    if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("H2D x: ") + cudaGetErrorString(e));
+    cudaEventRecord(evx[i], A->e2e_h2d);
+  }
+  for (int c = 0; c < K; ++c) {
+    const int64_t b0 = nb * c / K, b1 = nb * (c + 1) / K;
+    if (b1 <= b0) {
+      cudaEventRecord(evy[c], st);
+      continue;
+    }
+    int32_t hi = -1;
+    for (int64_t bi = b0; bi < b1; ++bi) hi = std::max(hi, A->blk_cmax[bi]);
+    // wait for the piece holding column hi (pieces arrive in order)
+    int p = K - 1;
+    if (hi < 0) p = -1;
+    else
+      while (p > 0 && xa(p) > hi) --p;
+    if (p >= 0) cudaStreamWaitEvent(st, evx[p], 0);
+    bro_status_t r = A->dtype == BRO_FP64
+        ? launch_spmv_blocks<double>(A, (const double*)A->d_xs, (double*)A->d_ys, b0, b1, st)
+        : launch_spmv_blocks<float>(A, (const float*)A->d_xs, (float*)A->d_ys, b0, b1, st);
+    if (r != BRO_OK) return r;
+    cudaEventRecord(evy[c], st);
+    cudaStreamWaitEvent(A->e2e_d2h, evy[c], 0);
+    const int64_t r0 = 32 * b0, r1 = std::min(A->m, 32 * b1);
+    e = cudaMemcpyAsync(static_cast<char*>(y_host) + r0 * vs, static_cast<const char*>(A->d_ys) + r0 * vs,
+                        size_t(r1 - r0) * vs, cudaMemcpyDeviceToHost, A->e2e_d2h);
+    if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("D2H y: ") + cudaGetErrorString(e));
+  }
+  if ((e = cudaStreamSynchronize(A->e2e_d2h)) != cudaSuccess || (e = cudaStreamSynchronize(st)) != cudaSuccess ||
+      (e = cudaStreamSynchronize(A->e2e_h2d)) != cudaSuccess)
+    return fail(BRO_ERR_CUDA, std::string("sync: ") + cudaGetErrorString(e));
+  return BRO_OK;
+}
+
+}  // namespace
+
 extern "C" {
 
 void bro_opts_default(bro_opts_t* o) {
@@ -770,6 +888,10 @@ bro_status_t bro_spmv_host(bro_matrix_t A, const void* x_host, void* y_host, bro
   if (!A->d_xs && xb) s = dev_upload(A, &A->d_xs, nullptr, xb);
   if (s == BRO_OK && !A->d_ys && yb) s = dev_upload(A, &A->d_ys, nullptr, yb);
   if (s != BRO_OK) return s;
+  // ELL-only handles: pipelined copies and compute (BRO_E2E_CHUNKS pieces, 1 = serial)
+  const int K = std::max(1, std::min(64, env_int("BRO_E2E_CHUNKS", kE2eChunks)));
+  if (K > 1 && A->has_ell && !A->has_coo && int64_t(A->blk_cmax.size()) >= K && A->n > 0)
+    return spmv_host_pipelined(A, x_host, y_host, st, K);
   cudaError_t e = xb ? cudaMemcpyAsync(A->d_xs, x_host, xb, cudaMemcpyHostToDevice, st) : cudaSuccess;
   if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("H2D x: ") + cudaGetErrorString(e));
   s = bro_spmv(A, A->d_xs, A->d_ys, stream);

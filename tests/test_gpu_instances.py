@@ -156,3 +156,42 @@ def test_bro_ell_tiny_slices(lib, dev, ell_env, name, mk, dtype, tiny):
         assert ok.all(), f"V={V}: {np.count_nonzero(~ok)} rows out of tolerance"
         M.close()
     os.environ.pop("BRO_ELL_TINY", None)
+
+
+@pytest.fixture
+def e2e_env():
+    old = os.environ.get("BRO_E2E_CHUNKS")
+    yield
+    if old is None:
+        os.environ.pop("BRO_E2E_CHUNKS", None)
+    else:
+        os.environ["BRO_E2E_CHUNKS"] = old
+
+
+E2E_CASES = [
+    ("c1", lambda: make_config(1)),
+    ("banded_ragged", lambda: random_csr(10007, 10007, 41, max_len=30, empty_frac=0.1)),
+    ("wide", lambda: random_csr(3000, 50000, 42, max_len=8, wide_cols=True)),
+    ("empty_rows", lambda: random_csr(2000, 2000, 43, max_len=0)),
+]
+
+
+@pytest.mark.parametrize("name,mk", E2E_CASES, ids=[c[0] for c in E2E_CASES])
+@pytest.mark.parametrize("codec", [1, 0])
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_spmv_host_pipelined(lib, dev, e2e_env, name, mk, codec, dtype):
+    """bro_spmv_host of an ELL-only handle pipelines x pieces, row blocks and
+    y pieces over three streams; every chunking gives exactly bro_spmv's y
+    (same kernels, same per-row arithmetic)."""
+    A = mk()
+    x = make_x(A.n, 8, dtype)
+    M = lib.BroMatrix(A, fmt="ell", codec=codec, device=0, dtype=dtype)
+    y_dev = M.spmv(torch.from_numpy(x).to(dev)).cpu().numpy()
+    xh = torch.from_numpy(x).pin_memory().numpy()
+    for K in ("1", "2", "8", "64"):
+        os.environ["BRO_E2E_CHUNKS"] = K
+        yh = torch.empty(A.m, dtype=torch.float64 if dtype == np.float64 else torch.float32).pin_memory().numpy()
+        yh[:] = np.nan
+        M.spmv_host(xh, yh)
+        assert np.array_equal(yh, y_dev), f"K={K}"
+    M.close()
