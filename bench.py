@@ -453,7 +453,8 @@ def main():
         e2e = {"value": 2.0 * A.nnz / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s",
                "h2d_bytes_per_step": int(blk.mat.n * isz), "d2h_bytes_per_step": int(blk.mat.m * isz),
                "ms_per_step": e2e_ms,
-               "path": "bro_spmv_host: pinned x H2D + bro_spmv + y D2H + stream sync, per rank"}
+               "path": "bro_spmv_host: pinned x H2D + bro_spmv + y D2H + stream sync, per rank "
+                       "(ELL-only handles pipeline the three over streams in 8 pieces)"}
 
     if rank != 0:
         if world > 1:
