@@ -196,7 +196,8 @@ bro_status_t bro_spmv_scatter(bro_matrix_t A, const void* x_dev, void* const* y_
 /* End-to-end y = A.x with HOST vectors: copies x (n values) host->device,
  * runs bro_spmv, copies y (m values) device->host and synchronizes `stream`.
  * Pinned host memory gives full PCIe bandwidth; pageable memory works.
- * ELL-only handles (BRO-ELL, ELLPACK) pipeline the three steps: x goes up in
+ * ELL-only handles (BRO-ELL, ELLPACK) with x of at least 4 MB pipeline the
+ * three steps: x goes up in
  * pieces on an internal stream, each block of rows runs on `stream` as soon
  * as the pieces covering its columns have arrived, and its y goes down on a
  * second internal stream while later blocks compute (environment variable

@@ -25,6 +25,9 @@ bro_status_t fail(bro_status_t s, const std::string& msg) {
 
 constexpr int kCooThreads = 256;
 constexpr int kE2eChunks = 8;  // pieces of the pipelined bro_spmv_host
+// below this x size the pieces' launch and event overheads exceed the copy
+// time they hide (C1/C2 e2e: 1.3 -> 0.5 and 63 -> 57 GFLOP/s when pipelined)
+constexpr size_t kE2eMinBytes = size_t(4) << 20;
 constexpr int kBarWindow = 64;  // candidate partitions of BAR method 2 (windowed Algorithm 2)
 constexpr int kCooMaxUpi = 4;   // work units per COO interval (8 steps = 256 entries each at 4)
 constexpr int kCooUpi = 2;
@@ -890,7 +893,8 @@ bro_status_t bro_spmv_host(bro_matrix_t A, const void* x_host, void* y_host, bro
   if (s != BRO_OK) return s;
   // ELL-only handles: pipelined copies and compute (BRO_E2E_CHUNKS pieces, 1 = serial)
   const int K = std::max(1, std::min(64, env_int("BRO_E2E_CHUNKS", kE2eChunks)));
-  if (K > 1 && A->has_ell && !A->has_coo && int64_t(A->blk_cmax.size()) >= K && A->n > 0)
+  const size_t min_bytes = size_t(std::max(0, env_int("BRO_E2E_MIN_KB", int(kE2eMinBytes >> 10)))) << 10;
+  if (K > 1 && A->has_ell && !A->has_coo && int64_t(A->blk_cmax.size()) >= K && xb >= min_bytes && xb > 0)
     return spmv_host_pipelined(A, x_host, y_host, st, K);
   cudaError_t e = xb ? cudaMemcpyAsync(A->d_xs, x_host, xb, cudaMemcpyHostToDevice, st) : cudaSuccess;
   if (e != cudaSuccess) return fail(BRO_ERR_CUDA, std::string("H2D x: ") + cudaGetErrorString(e));

@@ -160,12 +160,15 @@ def test_bro_ell_tiny_slices(lib, dev, ell_env, name, mk, dtype, tiny):
 
 @pytest.fixture
 def e2e_env():
-    old = os.environ.get("BRO_E2E_CHUNKS")
+    keys = ("BRO_E2E_CHUNKS", "BRO_E2E_MIN_KB")
+    old = {k: os.environ.get(k) for k in keys}
+    os.environ["BRO_E2E_MIN_KB"] = "0"  # pipeline these small cases too
     yield
-    if old is None:
-        os.environ.pop("BRO_E2E_CHUNKS", None)
-    else:
-        os.environ["BRO_E2E_CHUNKS"] = old
+    for k, v in old.items():
+        if v is None:
+            os.environ.pop(k, None)
+        else:
+            os.environ[k] = v
 
 
 E2E_CASES = [
