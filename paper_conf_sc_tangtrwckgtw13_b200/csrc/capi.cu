@@ -490,6 +490,10 @@ void launch_bro_ell(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cud
     launch_bro_ell_od<T, V, 4, 4, 16, 34>(A, x, y, st);
   else if (variant == 5)
     launch_bro_ell_od<T, V, 4, 2, 32, 34>(A, x, y, st);
+  else if (variant == 6 && A->ell_max_S < kEllSmallRows)  // 4-warp blocks, 10-row window
+    launch_bro_ell_od<T, V, 4, 8, 8, kEllSmallRows>(A, x, y, st);
+  else if (variant == 7 && A->ell_max_S < kEllSmallRows)  // 8-warp blocks, 10-row window (the previous default)
+    launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks, 8, kEllSmallRows>(A, x, y, st);
   else if (A->ell_max_l <= 4 && y.n == 1 && y.mc == nullptr && env_int("BRO_ELL_TINY", 1) == 1)
     launch_bro_ell_tiny<T, V, sizeof(T) == 8 ? 5 : 6, 1>(A, x, y, st);
   else if (A->ell_max_l <= 4 && y.n == 1 && y.mc == nullptr && env_int("BRO_ELL_TINY", 1) == 2)
@@ -505,7 +509,7 @@ void launch_bro_ell(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y, cud
   else if (A->ell_max_S < kEllSmallRows && env_int("BRO_ELL_SMALLWIN", 1) && env_int("BRO_ELL_CPV", 0) == 2)
     launch_bro_ell_od<T, V, 4, 6, 8, kEllSmallRows, 2>(A, x, y, st);
   else if (A->ell_max_S < kEllSmallRows && env_int("BRO_ELL_SMALLWIN", 1))
-    launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks, 8, kEllSmallRows>(A, x, y, st);
+    launch_bro_ell_od<T, V, 16, 2, 8, kEllSmallRows>(A, x, y, st);  // 16-warp blocks: C5 f32 255.4 -> 250.4 us
   else if (A->ell_max_S < kEllMidRows && env_int("BRO_ELL_SMALLWIN", 1))
     launch_bro_ell_od<T, V, kEllWarps, kEllMinBlocks, 8, kEllMidRows>(A, x, y, st);
   else
