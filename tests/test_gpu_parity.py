@@ -276,6 +276,25 @@ def test_config5_full_size(lib, dev):
     M.close()
 
 
+def test_config5_full_size_f32(lib, dev):
+    """C5 fp32 at full size (bench.py --dtype f32's launch configuration):
+    x = 1 gives small integers, exact in fp32 (y_i = 27 - len_i); sampled
+    rows against the oracle within 1e-5 * sum|a||x| for random x."""
+    A = make_config(5, np.float32)
+    M = lib.BroMatrix(A, fmt="ell", codec=1, device=0, dtype=np.float32)
+    ones = torch.ones(A.n, dtype=torch.float32, device=dev)
+    y = M.spmv(ones).cpu().numpy()
+    assert np.array_equal(y, (27.0 - A.row_lengths()).astype(np.float32))
+    x = make_x(A.n, 5, np.float32)
+    y = M.spmv(torch.from_numpy(x).to(dev)).cpu().numpy()
+    rows = np.unique(np.concatenate([np.arange(40), A.m - 1 - np.arange(40),
+                                     np.random.default_rng(2).integers(0, A.m, 3000)]))
+    yr, S = spmv.csr_spmv_rows(A.row_ptr, A.col, A.vals.astype(np.float32), x, rows)
+    ok, err = spmv.within_tolerance(y[rows], yr, S, TOL[np.float32])
+    assert ok.all(), float(err.max())
+    M.close()
+
+
 def test_config5_row_blocks(lib, dev):
     """Row-block partition used by the multi-GPU driver: local blocks with
     global columns reproduce the global product (one GPU, 4 blocks)."""
