@@ -268,6 +268,23 @@ def build_row_block(A, rank, world, dev, fmt, dtype, bounds, args, x_host, strea
     notes = []
     for mode in order:
         blk, err = None, ""
+        if mode == "p2p":
+            # every rank agrees on the preconditions before any rank enters the
+            # collective symmetric-memory rendezvous (an asymmetric failure
+            # inside it would leave the other ranks waiting)
+            pre = 0.0
+            try:
+                idx = torch.device(dev).index or 0
+                pre = float(torch.cuda.device_count() >= world and all(
+                    torch.cuda.can_device_access_peer(idx, p) for p in range(world) if p != idx))
+            except Exception:  # noqa: BLE001
+                pre = 0.0
+            ok_pre = torch.tensor([pre], dtype=torch.float64,
+                                  device=dev if args.dist_backend == "nccl" else "cpu")
+            dist.all_reduce(ok_pre, op=dist.ReduceOp.MIN)
+            if ok_pre.item() != 1.0:
+                notes.append({"mode": mode, "why": "no peer access between every pair of ranks' GPUs"})
+                continue
         try:
             blk = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=1, dtype=dtype, bounds=bounds,
                                vec_words=args.vec_words, exchange=mode)
