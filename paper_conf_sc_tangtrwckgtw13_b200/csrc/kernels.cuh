@@ -32,6 +32,15 @@ namespace dev {
 constexpr int kWarp = 32;
 
 // ------------------------------------------------------------------ loads
+// BRO_L2_PF: L2 prefetch-size qualifier of the streamed loads.  Measured
+// (profiles/r01/s4/ab_l2_256B.txt, A/B in one session): neutral for every
+// BRO kernel (C5 f64 343.1 vs 343.8 us, f32 250.4 vs 250.3, C4 111.7 vs
+// 111.7, C2 18.5 vs 18.5) and up to 3% faster for the uncompressed ELLPACK
+// baseline (C2 27.9 -> 27.0 us), so it is on for both: the speedups are
+// quoted against the faster baseline.  -DBRO_L2_PF='""' turns it off.
+#ifndef BRO_L2_PF
+#define BRO_L2_PF ".L2::256B"
+#endif
 // Streamed arrays (values, symbols, COO col/row) are read with non-volatile
 // inline asm ld.global.nc.L1::no_allocate.  The compiler treats these as pure
 // and may issue a guarded load (cond ? ld(p) : 0, or the full-chunk path of
@@ -45,28 +54,28 @@ constexpr int kStreamPad = 16384;
 
 __device__ __forceinline__ uint4 ld_stream_u4(const uint32_t* p) {
   uint4 r;
-  asm("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+  asm("ld.global.nc.L1::no_allocate" BRO_L2_PF ".v4.u32 {%0,%1,%2,%3}, [%4];"
       : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
   return r;
 }
 __device__ __forceinline__ uint32_t ld_stream_u32(const uint32_t* p) {
   uint32_t r;
-  asm("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+  asm("ld.global.nc.L1::no_allocate" BRO_L2_PF ".u32 %0, [%1];" : "=r"(r) : "l"(p));
   return r;
 }
 __device__ __forceinline__ int32_t ld_stream_s32(const int32_t* p) {
   int32_t r;
-  asm("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(r) : "l"(p));
+  asm("ld.global.nc.L1::no_allocate" BRO_L2_PF ".s32 %0, [%1];" : "=r"(r) : "l"(p));
   return r;
 }
 __device__ __forceinline__ double ld_stream(const double* p) {
   double r;
-  asm("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(r) : "l"(p));
+  asm("ld.global.nc.L1::no_allocate" BRO_L2_PF ".f64 %0, [%1];" : "=d"(r) : "l"(p));
   return r;
 }
 __device__ __forceinline__ float ld_stream(const float* p) {
   float r;
-  asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(r) : "l"(p));
+  asm("ld.global.nc.L1::no_allocate" BRO_L2_PF ".f32 %0, [%1];" : "=f"(r) : "l"(p));
   return r;
 }
 
@@ -76,14 +85,14 @@ template <> struct Chunk<double> {
   double v[2];
   static constexpr int N = 2;
   __device__ __forceinline__ void load(const double* p) {
-    asm("ld.global.nc.L1::no_allocate.v2.f64 {%0,%1}, [%2];" : "=d"(v[0]), "=d"(v[1]) : "l"(p));
+    asm("ld.global.nc.L1::no_allocate" BRO_L2_PF ".v2.f64 {%0,%1}, [%2];" : "=d"(v[0]), "=d"(v[1]) : "l"(p));
   }
 };
 template <> struct Chunk<float> {
   float v[4];
   static constexpr int N = 4;
   __device__ __forceinline__ void load(const float* p) {
-    asm("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+    asm("ld.global.nc.L1::no_allocate" BRO_L2_PF ".v4.f32 {%0,%1,%2,%3}, [%4];"
         : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]) : "l"(p));
   }
 };
