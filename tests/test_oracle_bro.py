@@ -172,14 +172,69 @@ def coo_rows_strategy(draw):
 
 
 @settings(max_examples=40, deadline=None, suppress_health_check=[HealthCheck.too_slow])
-@given(rows=coo_rows_strategy(), T=st.sampled_from([1, 4, 32]), V=st.sampled_from([1, 4]))
+@given(rows=coo_rows_strategy(), T=st.sampled_from([1, 8, 16, 32]), V=st.sampled_from([1, 4]))
 def test_bro_coo_roundtrip_fuzz(rows, T, V):
     rows = rows[rows < 2**31 - 1]
-    cols = np.zeros(rows.size, dtype=np.int32)
-    C = bro_coo.encode(rows, cols, np.zeros(rows.size), T=T, V=V)
+    cols = np.arange(rows.size, dtype=np.int32)
+    vals = np.arange(rows.size, dtype=np.float64) + 0.5
+    C = bro_coo.encode(rows, cols, vals, T=T, V=V)
     assert np.array_equal(bro_coo.decode_rows(C), rows)
+    assert np.array_equal(bro_coo.unarrange(C.col, rows.size, T, 4), cols)
+    assert np.array_equal(bro_coo.unarrange(C.vals, rows.size, T, 2), vals)
+    I = 32 * T
     for i in range(C.n_intervals):
-        assert int(C.width[i]) <= 32
+        # one width per interval = Gamma of the largest consecutive
+        # difference of the sorted rows inside the interval (brute force)
+        seg = rows[i * I:(i + 1) * I]
+        dmax = int(np.max(np.diff(seg))) if seg.size > 1 else 0
+        assert int(C.width[i]) == dmax.bit_length() <= 32
+        assert int(C.base_row[i]) == int(seg[0])
+
+
+def test_bro_coo_hand_example_T1():
+    """One interval of 32 entries, T = 1 (lane l holds entry l): rows
+    0 x10, 1 x10, 5 x12.  Deltas in entry order: 1 at entry 10, 4 at entry
+    20, else 0 -> one width b = Gamma(4) = 3; each lane stream is
+    3 bits MSB first padded to a 32-bit symbol: lane 10 = 001 -> 0x20000000,
+    lane 20 = 100 -> 0x80000000, every other lane 0 (worked by hand)."""
+    rows = np.array([0] * 10 + [1] * 10 + [5] * 12)
+    C = bro_coo.encode(rows, np.zeros(32, np.int32), np.zeros(32), T=1, V=1)
+    assert C.width.tolist() == [3] and C.base_row.tolist() == [0]
+    assert C.symptr.tolist() == [0, 1]
+    want = [0] * 32
+    want[10], want[20] = 0x20000000, 0x80000000
+    assert C.words.tolist() == want
+    assert np.array_equal(bro_coo.decode_rows(C), rows)
+
+
+def test_bro_coo_hand_example_T2_lane_contiguous():
+    """T = 2, 64 entries, row(e) = e // 3 (worked by hand): lane l holds
+    entries 2l and 2l+1 (consecutive), deltas are 1 where e % 3 == 0
+    (e > 0), width 1; lane stream = [delta(2l), delta(2l+1)] MSB first:
+    lane 0 (e 0,1) 00 -> 0; lane 1 (e 2,3) 01 -> 0x40000000; lane 3
+    (e 6,7) 10 -> 0x80000000; lane 4 (e 8,9) 01 -> 0x40000000; lane 2
+    (e 4,5) 00 -> 0.  col/vals are stored lane-contiguously: with 4-entry
+    chunks, lane l's 2 entries sit at 2l, 2l+1 (place() tail of a 2-slot
+    lane stream), so col equals COO order here."""
+    rows = np.arange(64) // 3
+    cols = np.arange(64, dtype=np.int32) * 7
+    C = bro_coo.encode(rows, cols, np.ones(64), T=2, V=1)
+    assert C.width.tolist() == [1]
+    assert C.words[:5].tolist() == [0, 0x40000000, 0, 0x80000000, 0x40000000]
+    assert np.array_equal(C.col, cols)
+    assert np.array_equal(bro_coo.decode_rows(C), rows)
+
+
+def test_bro_coo_values_chunked_like_bro_ell():
+    """T = 8, fp64: lane l's 8 values are 4 chunks of 2 (16 bytes); chunk c
+    of all 32 lanes is one contiguous 512-byte row: entry (l, t) at
+    64*(t//2) + 2*l + t%2 (BRO-ELL's value multiplexing, P:L116)."""
+    N = 256
+    vals = np.arange(N, dtype=np.float64)
+    C = bro_coo.encode(np.zeros(N, np.int64), np.zeros(N, np.int32), vals, T=8, V=4)
+    for lane in (0, 1, 31):
+        for t in range(8):
+            assert C.vals[64 * (t // 2) + 2 * lane + t % 2] == 8 * lane + t
 
 
 def test_bro_coo_single_row_interval_has_zero_width():
@@ -190,11 +245,35 @@ def test_bro_coo_single_row_interval_has_zero_width():
     assert np.array_equal(bro_coo.decode_rows(C), rows)
 
 
-def test_bro_coo_spmv_equals_csr():
+def test_bro_coo_tail_interval_padding():
+    """A ragged last interval: slots past the end hold col 0 / value 0, the
+    plain baseline repeats the last row there."""
+    rows = np.sort(np.random.default_rng(5).integers(0, 90, 300))
+    C = bro_coo.encode(rows, np.arange(300, dtype=np.int32), np.ones(300), T=8)
+    assert C.col.size == 2 * 256 and C.vals.size == 512
+    assert np.count_nonzero(C.vals) == 300
+    pr = bro_coo.plain_rows(rows, T=8)
+    assert np.array_equal(bro_coo.unarrange(pr, 300, 8, 4), rows)
+    assert np.count_nonzero(pr == rows[-1]) >= 512 - 300
+
+
+@pytest.mark.parametrize("T", [8, 32])
+def test_bro_coo_spmv_equals_csr(T):
     A = random_csr(400, 900, 3, max_len=30, empty_frac=0.3, long_frac=0.02, long_len=700)
     rows, cols, vals = _coo(A)
     x = np.random.default_rng(0).uniform(-1, 1, A.n)
-    C = bro_coo.encode(rows, cols, vals)
+    C = bro_coo.encode(rows, cols, vals, T=T)
     y = bro_coo.spmv_accumulate(C, x, np.zeros(A.m))
     yr, S = spmv.csr_spmv(A.row_ptr, A.col, A.vals, x)
     assert np.all(np.abs(y - np.array(yr, np.float64)) <= 1e-13 * np.array(S, np.float64) + 1e-300)
+
+
+@pytest.mark.parametrize("T", [1, 8, 32])
+@pytest.mark.parametrize("seed", range(3))
+def test_bro_coo_interval_shapes_match_encoder(T, seed):
+    rows = np.sort(np.random.default_rng(seed).integers(0, 5000 * (seed + 1), 3000 + 77 * seed))
+    C = bro_coo.encode(rows, np.zeros(rows.size, np.int32), np.zeros(rows.size), T=T)
+    base, width, S = bro_coo.interval_shapes(rows, T)
+    assert base.tolist() == C.base_row.tolist()
+    assert width.tolist() == C.width.tolist()
+    assert S.tolist() == np.diff(C.symptr.astype(np.int64)).tolist()
