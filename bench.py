@@ -55,6 +55,9 @@ def parse_args():
                     help="override the workload's format (e.g. coo: standalone BRO-COO vs COO, Fig. 7)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--vec-words", type=int, default=0, help="0 = auto (fp64: 1, fp32: 4)")
+    ap.add_argument("--slice-h", type=int, default=0, help="BRO-ELL slice height: 0 = auto, 32, 64")
+    ap.add_argument("--coo-T", type=int, default=0, help="BRO-COO entries per lane: 0 = auto, 8, 16, 32")
+    ap.add_argument("--ell-kernel", type=int, default=0, help="BRO-ELL instance: 0 = auto, 1..5 (A/B only)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--flush-l2", action="store_true", help="write a 2xL2 buffer between steps")
@@ -257,6 +260,11 @@ def run_reference(args):
            "e2e": {"value": val, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
 
+def layout_opts(args):
+    """BroMatrix layout options of the BRO handle (0 = the library's auto choice)."""
+    return {"slice_h": args.slice_h, "coo_T": args.coo_T, "ell_kernel": args.ell_kernel}
+
+
 def build_row_block(A, rank, world, dev, fmt, dtype, bounds, args, x_host, stream):
     """The BRO row block with the fastest exchange that reproduces the
     allgather schedule on this box: p2p (fused scatter into symmetric memory),
@@ -287,7 +295,7 @@ def build_row_block(A, rank, world, dev, fmt, dtype, bounds, args, x_host, strea
                 continue
         try:
             blk = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=1, dtype=dtype, bounds=bounds,
-                               vec_words=args.vec_words, exchange=mode)
+                               vec_words=args.vec_words, exchange=mode, **layout_opts(args))
             if mode != "allgather":
                 res = []
                 for ex in (mode, "allgather"):
@@ -298,7 +306,11 @@ def build_row_block(A, rank, world, dev, fmt, dtype, bounds, args, x_host, strea
                     torch.cuda.synchronize()
                     res.append(blk.X[blk.k % 2].clone())
                 a, b = res
-                if not (torch.isfinite(a).all() and torch.allclose(a, b, rtol=1e-9, atol=0.0)):
+                # the modes split rows differently (overlap: three handles), so
+                # summation orders differ: compare at the dtype's bound, not bitwise
+                rtol = 1e-12 if dtype == np.float64 else 1e-5
+                scale = torch.maximum(a.abs(), b.abs()).max().clamp_min(1e-300)
+                if not (torch.isfinite(a).all() and ((a - b).abs() <= 10 * rtol * scale).all()):
                     err = "3-iteration result differs from the allgather schedule"
         except Exception as e:  # noqa: BLE001 - any setup failure moves to the next mode
             err = f"{type(e).__name__}: {e}"[:200]
@@ -338,6 +350,9 @@ def main():
     dev = torch.device("cuda", local)
     if world > 1:
         if args.dist_backend == "nccl":
+            if rank == 0:  # communicator setup lines (ranks, NVLS / P2P transport) in the driver's log
+                os.environ.setdefault("NCCL_DEBUG", "INFO")
+                os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
             dist.init_process_group("nccl", device_id=dev)
         else:
             dist.init_process_group("gloo")
@@ -360,13 +375,14 @@ def main():
     if world > 1:
         blk, exch_info = build_row_block(A, rank, world, dev, fmt, dtype, bounds, args, x_host, stream)
         base = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=0, dtype=dtype, bounds=bounds,
-                            exchange=blk.exchange)
+                            exchange=blk.exchange, coo_T=args.coo_T)
         blk.set_x(x_host)
         base.set_x(x_host)
     else:
         blk = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=1, dtype=dtype, bounds=bounds,
-                           vec_words=args.vec_words)
-        base = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=0, dtype=dtype, bounds=bounds)
+                           vec_words=args.vec_words, **layout_opts(args))
+        base = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=0, dtype=dtype, bounds=bounds,
+                            coo_T=args.coo_T)
     info, binfo = blk.mat.info, base.mat.info
     # our kernels per step: ELL kernel, COO kernel + fix-up; the overlap
     # exchange runs one SpMV per row part (interior / head / tail); a
@@ -511,7 +527,9 @@ def main():
         "config": {
             "workload": workload_label(args.workload),
             "format": bro_name, "m": A.m, "n": A.n, "nnz": A.nnz,
-            "vec_words": info["vec_words"],
+            "vec_words": info["vec_words"], "slice_h": info["slice_h"], "coo_T": info["coo_T"],
+            "ell_kernel": {0: None, 1: "tiny", 2: "few-slice", 3: "small-window", 4: "mid-window",
+                           5: "general"}[info["ell_kernel"]] if info["nnz_ell"] or fmt != "coo" else None,
             "l2": ("flushed (2x L2 write) before every step" if args.flush_l2 else
                    ("inputs larger than L2" if alg_bytes > L2_BYTES else "L2-resident (warm)")),
             "parallelism": f"row-block x{world}" + (f" + {exch_info['exchange']} exchange of y per step (x_(k+1) = A.x_k)"
@@ -521,9 +539,11 @@ def main():
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
                      "peak_kind": peak_kind,
-                     "kernel": f"bro_ell_spmv_od<{'double' if dtype == np.float64 else 'float'},V={info['vec_words']}>"
+                     "kernel": (f"bro_ell_{'tiny' if info['ell_kernel'] == 1 else 'od'}"
+                                f"<{'double' if dtype == np.float64 else 'float'},V={info['vec_words']},"
+                                f"R={info['slice_h'] // 32}>")
                      if fmt == "ell" else ("coo_spmv + coo_fixup" if fmt == "coo" else
-                                           "bro_ell_spmv + coo_spmv + coo_fixup"),
+                                           "bro_ell + coo_spmv + coo_fixup"),
                      "algorithmic_bytes_per_launch": alg_bytes, "kernel_ms": kern_ms,
                      "frac_of_8TBps_spec": achieved / 8000.0,
                      "read_stream_GBps": rc, "read_stream_how": "torch.sum over 2 GiB fp32 (a library "

@@ -33,24 +33,35 @@
  *     torch.cuda.current_stream().cuda_stream.
  *
  * Encoded layout (bit-exact):
- *   BRO-ELL, slice height h = 32 rows (one warp per slice), sym_len = 32:
+ *   BRO-ELL, slice height h = 32 or 64 rows (opts.slice_h; one warp per
+ *   slice, h/32 rows per lane), sym_len = 32:
  *     colptr[t]  = sum_{t'<t} l_t'       (l_t = num_col of slice t)
  *     symptr[t]  = sum_{t'<t} S_t'       (S_t = 32-bit symbols per row stream)
  *     bit_alloc[colptr[t] + j] = b_{t,j} (b_p implied by S_t)
- *     symbol q of row r of slice t at words[32*symptr[t] + place(r,q,S_t,V)]
- *     value of slot (r,j) of slice t at vals[32*colptr[t] + place(r,j,l_t,Vv)]
- *     place(r,q,S,V) = 32*V*(q/V) + r*V + q%V          if q/V < S/V
- *                    = 32*V*F + r*(S-V*F) + (q-V*F)    otherwise (F = S/V)
+ *     symbol q of row r of slice t at words[h*symptr[t] + place(r,q,S_t,V)]
+ *     value of slot (r,j) of slice t at vals[h*colptr[t] + place(r,j,l_t,Vv)]
+ *     place(r,q,S,V) = h*V*(q/V) + r*V + q%V          if q/V < S/V
+ *                    = h*V*F + r*(S-V*F) + (q-V*F)    otherwise (F = S/V)
  *     V = opts.vec_words (1 = the paper's comp_str_i[q*h+tid]), Vv = 16/sizeof(val).
  *     Row streams are concatenated b-bit deltas, most significant bit first,
  *     delta_0 = col_0 + 1, delta_j = col_j - col_{j-1}, 0 = padding.
- *   BRO-COO, intervals of 32*T entries (T = opts.coo_T = 32): entry
- *     i*32*T + 32*t + lane is element (t, lane); each lane's rows are delta
- *     coded down t from base_row[i] with one width width[i]; lane
- *     word q at coo_words[32*coo_symptr[i] + place(lane,q,S_i,V)].
+ *   BRO-COO, intervals of 32*T entries (T = 8, 16 or 32): lane l of interval
+ *     i owns the T consecutive entries e = i*32*T + T*l + t (DESIGN.md
+ *     reading R13); deltas follow entry order, delta(e) = row(e) - row(e-1),
+ *     delta of the first entry 0, base_row[i] = row of the first entry, one
+ *     width width[i] per interval; lane l's T fields, MSB first,
+ *     padded to S_i = ceil(T*width/32) symbols at
+ *     coo_words[32*coo_symptr[i] + place(l,q,S_i,V)] (h = 32).
+ *     col / vals (and plain COO rows) are stored per interval in the same
+ *     lane-contiguous order in 16-byte chunks (reading R26): entry (l, t) at
+ *     [i*32*T + place(l,t,T,C)], C = 4 for int32, 16/sizeof(val) for values;
+ *     slots past nnz hold col 0 / value 0 (plain rows: the last row).
  *
- * Thread safety: distinct handles may be used concurrently; one handle must
- * not be used by two threads at once.
+ * Thread safety: distinct handles may be used concurrently.  A handle holds
+ * per-call scratch (the COO carries, the bro_spmv_host buffers): at most ONE
+ * call on a handle may be in flight at a time — serialize its calls on one
+ * stream (or synchronize between streams), and never use it from two threads
+ * at once.
  */
 #ifndef BRO_H_
 #define BRO_H_
@@ -83,19 +94,30 @@ typedef enum {
 } bro_status_t;
 
 typedef struct {
-  int32_t slice_h;   /* BRO-ELL slice height h. Must be 32 (one warp per slice). */
+  int32_t slice_h;   /* BRO-ELL slice height h (a parameter of the method):
+                        32 (one row per lane of the slice's warp), 64 (two rows per lane:
+                        widths, offsets and setup shared by both rows), 0 (default) =
+                        auto: 64 when m >= 303,104 (64 rows x 32 resident warps x 148
+                        SMs: every resident warp of a B200 still gets slices), else 32.
+                        bro_info_t.slice_h reports the value. */
   int32_t sym_bits;  /* sym_len. Must be 32. */
-  int32_t vec_words; /* V: 1, 2 or 4 symbols per lane chunk.  1 = the paper's multiplexing
+  int32_t vec_words; /* V: 1 or 4 symbols per lane chunk.  1 = the paper's multiplexing
                         (comp_str_i[q*h + tid]); 4 = 16-byte per-lane chunks (128-bit loads);
-                        0 (default) = auto: 1 for BRO_FP64, 4 for BRO_FP32 (measured fastest;
-                        bro_info_t.vec_words reports the resolved value). */
-  int32_t coo_T;     /* BRO-COO steps per interval (interval = 32*T entries). Must be 32. */
+                        0 (default) = auto: 1 for BRO_FP64, 4 for BRO_FP32. */
+  int32_t coo_T;     /* BRO-COO entries per lane of an interval (interval = 32*T entries):
+                        8, 16 or 32; 0 (default) = auto: the largest T for which the COO
+                        part still has >= 4,736 intervals (32 warps x 148 SMs), else 8. */
   int64_t hyb_K;     /* HYB dividing column; -1 = the "less than a third" rule. */
   int32_t codec;     /* 1 = BRO compressed formats; 0 = uncompressed ELL/COO/HYB baseline. */
   int32_t min_bits;  /* 0 = natural widths; k in [1, 31] forces every BRO-ELL width
                         b_j = max(Gamma, k) — the simulated compression ratios of the
                         Fig. 3 experiment ("the number of bits allocated to each
                         index value ... was varied"). */
+  int32_t ell_kernel;/* BRO-ELL kernel instance: 0 (default) = chosen at create from the
+                        matrix shape; 1 tiny (every slice <= 4 columns), 2 few-slice
+                        (h = 32), 3 small window (every row stream < 10 symbols), 4 mid
+                        window (< 18), 5 general.  An instance the matrix does not fit
+                        gives BRO_ERR_ARG.  For A/B measurements and tests. */
 } bro_opts_t;
 
 typedef struct {
@@ -104,10 +126,14 @@ typedef struct {
   int32_t codec;              /* 1 BRO, 0 uncompressed */
   int32_t format;             /* 0 ELL, 1 COO, 2 HYB */
   int32_t vec_words;
+  int32_t slice_h;            /* BRO-ELL slice height (32 or 64) */
+  int32_t coo_T;              /* BRO-COO entries per lane of an interval */
+  int32_t ell_kernel;         /* BRO-ELL kernel instance resolved at create (see bro_opts_t) */
+  int32_t reserved;
   int64_t K;                  /* ELL width bound: HYB K, or max row length for ELL */
   int64_t nnz_ell, nnz_coo;   /* entries in the ELL part and in the COO part */
-  int64_t n_slices;           /* BRO-ELL slices s = ceil(m/32) (0 without an ELL part) */
-  int64_t ell_slots;          /* value slots of the ELL part: 32*colptr[s] (BRO) or K*pitch (plain) */
+  int64_t n_slices;           /* BRO-ELL slices s = ceil(m/h) (0 without an ELL part) */
+  int64_t ell_slots;          /* value slots of the ELL part: h*colptr[s] (BRO) or K*pitch (plain) */
   int64_t ell_pitch;          /* plain ELL column pitch (m rounded up to 32) */
   int64_t n_intervals;        /* COO intervals ceil(nnz_coo / (32*T)) */
   int64_t ell_stream_bytes;   /* BRO-ELL compressed words (C of P:L246 for the ELL part) */
@@ -125,23 +151,24 @@ typedef struct {
 
 /* Parts of the encoded representation, for bro_export_encoded. */
 typedef enum {
-  BRO_PART_ELL_WORDS = 0,     /* uint32[32*symptr[s]]  BRO-ELL multiplexed stream */
+  BRO_PART_ELL_WORDS = 0,     /* uint32[h*symptr[s]]   BRO-ELL multiplexed stream */
   BRO_PART_ELL_BIT_ALLOC = 1, /* uint8[colptr[s]]      per-slice per-column widths */
   BRO_PART_ELL_COLPTR = 2,    /* uint64[s+1] */
   BRO_PART_ELL_SYMPTR = 3,    /* uint64[s+1] */
-  BRO_PART_ELL_VALS = 4,      /* value[32*colptr[s]]   sliced, interleaved, padding 0 */
+  BRO_PART_ELL_VALS = 4,      /* value[h*colptr[s]]    sliced, interleaved, padding 0 */
   BRO_PART_COO_WORDS = 5,     /* uint32[32*coo_symptr[nI]] */
   BRO_PART_COO_BASE_ROW = 6,  /* uint32[nI] */
   BRO_PART_COO_WIDTH = 7,     /* uint8[nI] */
   BRO_PART_COO_SYMPTR = 8,    /* uint64[nI+1] */
-  BRO_PART_COO_COL = 9,       /* int32[nnz_coo] (COO order) */
-  BRO_PART_COO_VALS = 10,     /* value[nnz_coo] */
-  BRO_PART_COO_ROW = 11,      /* int32[nnz_coo]  plain COO rows (codec 0) */
+  BRO_PART_COO_COL = 9,       /* int32[nI*32*T]  lane-contiguous chunks (reading R26), 0 past nnz */
+  BRO_PART_COO_VALS = 10,     /* value[nI*32*T]  same arrangement, 0 past nnz */
+  BRO_PART_COO_ROW = 11,      /* int32[nI*32*T]  plain COO rows (codec 0), last row past nnz */
   BRO_PART_PELL_COL = 12,     /* int32[K*pitch]  plain ELL, column-major, -1 = padding (codec 0) */
   BRO_PART_PELL_VALS = 13     /* value[K*pitch]  plain ELL values (codec 0) */
 } bro_part_t;
 
-/* Fill *opts with the defaults: h 32, sym 32, V 0 (auto), T 32, K auto, codec 1. */
+/* Fill *opts with the defaults: h 0 (auto), sym 32, V 0 (auto), T 0 (auto),
+ * K auto, codec 1, min_bits 0, ell_kernel 0 (auto). */
 void bro_opts_default(bro_opts_t* opts);
 
 /* Build an ELL-only matrix (BRO-ELL if opts->codec == 1, else ELLPACK with
@@ -197,12 +224,11 @@ bro_status_t bro_spmv_scatter(bro_matrix_t A, const void* x_dev, void* const* y_
  * runs bro_spmv, copies y (m values) device->host and synchronizes `stream`.
  * Pinned host memory gives full PCIe bandwidth; pageable memory works.
  * ELL-only handles (BRO-ELL, ELLPACK) with x of at least 4 MB pipeline the
- * three steps: x goes up in
- * pieces on an internal stream, each block of rows runs on `stream` as soon
- * as the pieces covering its columns have arrived, and its y goes down on a
- * second internal stream while later blocks compute (environment variable
- * BRO_E2E_CHUNKS = pieces, default 8; 1 = serial).  The result is identical
- * to bro_spmv's.  Returns after all of it has completed. */
+ * three steps in 8 pieces: x goes up on an internal stream, each block of
+ * slices runs on `stream` as soon as the pieces covering its columns have
+ * arrived, and its y goes down on a second internal stream while later
+ * blocks compute.  The result is identical to bro_spmv's.  Returns after all
+ * of it has completed. */
 bro_status_t bro_spmv_host(bro_matrix_t A, const void* x_host, void* y_host, bro_stream_t stream);
 
 /* Release the handle and all of its memory.  NULL is accepted. */
@@ -216,11 +242,13 @@ bro_status_t bro_get_info(bro_matrix_t A, bro_info_t* info);
  * Parts absent from this handle have size 0. */
 bro_status_t bro_export_encoded(bro_matrix_t A, int32_t part, void* host_buf, size_t* nbytes);
 
-/* GPU decode of the index streams (debug/parity surface): d_ell_cols
- * (int32[info.ell_slots], may be NULL) receives the decoded column of every
- * ELL slot in V = 1 slot order — slot 32*colptr[t] + 32*j + r for BRO-ELL,
- * j*pitch + r for plain ELL — or -1 for padding; d_coo_rows (int32[nnz_coo],
- * may be NULL) receives every COO entry's row.  Asynchronous on `stream`. */
+/* GPU decode of the index streams, through the SAME kernel instances and
+ * decode arithmetic as bro_spmv (their decode mode stores the decoded index
+ * where bro_spmv would multiply): d_ell_cols (int32[info.ell_slots], may be
+ * NULL) receives the decoded column of every ELL slot in V = 1 slot order —
+ * slot h*colptr[t] + h*j + r for BRO-ELL, j*pitch + r for plain ELL — or -1
+ * for padding; d_coo_rows (int32[nnz_coo], may be NULL) receives every COO
+ * entry's row in COO order.  Asynchronous on `stream`. */
 bro_status_t bro_decode_indices(bro_matrix_t A, int32_t* d_ell_cols, int32_t* d_coo_rows,
                                 bro_stream_t stream);
 
@@ -236,11 +264,12 @@ bro_status_t bro_hyb_K(int64_t m, const int64_t* row_ptr, int64_t* K_out);
  * Omega(c) = 128-byte line of x[c] for the dtype (O(m^2 k / h); m <= 65536,
  * else BRO_ERR_UNSUPPORTED);
  * method 2 = Algorithm 2 with a candidate window (reading R24): line 11's
- * argmin runs over the 64 non-full partitions nearest to the row's own partition
- * floor(pos/32) in length-sorted order (O(m k W), any m; W >= v would equal method 1).
+ * argmin runs over the W non-full partitions nearest to the row's own partition
+ * floor(pos/32) in length-sorted order (O(m k W), any m; W >= v equals method 1);
+ * W = window, 0 = 64 (ignored by methods 0 and 1).
  * Partitions hold 32 rows except the last. */
 bro_status_t bro_reorder_bar(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
-                             bro_dtype_t dtype, int32_t method, int64_t* perm_out);
+                             bro_dtype_t dtype, int32_t method, int32_t window, int64_t* perm_out);
 
 const char* bro_status_str(bro_status_t s);
 /* Message of the last failed call on this thread ("" if none). */

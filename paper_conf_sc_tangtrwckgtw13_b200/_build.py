@@ -15,12 +15,14 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libbro.so")
-SOURCES = ["capi.cu", "encode.cpp"]
-HEADERS = ["kernels.cuh", "encode.hpp", os.path.join("..", "..", "include", "bro.h")]
+SOURCES = ["capi.cu", "kern_ell64.cu", "kern_ell32.cu", "kern_misc.cu", "encode.cpp"]
+HEADERS = ["kernels.cuh", "kern_ell.cuh", "launch.hpp", "encode.hpp", os.path.join("..", "..", "include", "bro.h")]
+OBJDIR = os.path.join(CSRC, "build")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-shared", "-Xcompiler", "-fPIC,-pthread,-O3",
-         "-cudart", "static", "-Xptxas", "-v", "--expt-relaxed-constexpr"]
+CFLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-pthread,-O3", "-Xptxas", "-v",
+          "--expt-relaxed-constexpr"]
+LFLAGS = ["-shared", "-cudart", "static", "-Xcompiler", "-pthread"]
 
 
 def nvcc() -> str:
@@ -41,18 +43,37 @@ def _stale() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
+    """Compile every translation unit for sm_100a in parallel (-lineinfo,
+    ptxas -v into csrc/ptxas.log), then link libbro.so with the static CUDA
+    runtime."""
     if not force and not _stale():
         return LIB
-    cmd = [nvcc(), *ARCH, *FLAGS, "-I", os.path.join(ROOT, "include"), "-o", LIB + ".tmp",
-           *[os.path.join(CSRC, s) for s in SOURCES]]
-    r = subprocess.run(cmd, capture_output=True, text=True)
+    os.makedirs(OBJDIR, exist_ok=True)
+    procs = []
+    for src in SOURCES:
+        obj = os.path.join(OBJDIR, os.path.splitext(src)[0] + ".o")
+        cmd = [nvcc(), *ARCH, *CFLAGS, "-I", os.path.join(ROOT, "include"), "-c", "-o", obj,
+               os.path.join(CSRC, src)]
+        procs.append((src, obj, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.PIPE,
+                                                 text=True)))
+    logs, objs, failed = [], [], []
+    for src, obj, pr in procs:
+        out, err = pr.communicate()
+        logs.append(f"==== {src}\n{out}{err}")
+        objs.append(obj)
+        if pr.returncode != 0:
+            failed.append(src)
+            sys.stderr.write(out + err)
+    if failed:
+        raise RuntimeError(f"nvcc failed building {failed}")
+    r = subprocess.run([nvcc(), *ARCH, *LFLAGS, "-o", LIB + ".tmp", *objs], capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)
-        raise RuntimeError("nvcc failed building libbro.so")
+        raise RuntimeError("nvcc failed linking libbro.so")
     with open(os.path.join(CSRC, "ptxas.log"), "w") as f:
-        f.write(r.stderr)
+        f.write("\n".join(logs))
     if verbose:
-        sys.stderr.write(r.stderr)
+        sys.stderr.write("\n".join(logs))
     os.replace(LIB + ".tmp", LIB)
     return LIB
 

@@ -12,10 +12,7 @@ import os
 
 import numpy as np
 
-# BRO_LIB names an alternative in-tree build (A/B timing of two kernel
-# versions in one session); default libbro.so
-_LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)),
-                         os.path.basename(os.environ.get("BRO_LIB", "") or "libbro.so"))
+_LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libbro.so")
 if not os.path.exists(_LIB_PATH):
     raise ImportError(f"libbro.so not built ({_LIB_PATH}); run __graft_entry__.build() "
                       "or python -m paper_conf_sc_tangtrwckgtw13_b200._build")
@@ -36,13 +33,15 @@ FORMATS = {0: "ELL", 1: "COO", 2: "HYB"}
 class bro_opts_t(C.Structure):
     _fields_ = [("slice_h", C.c_int32), ("sym_bits", C.c_int32), ("vec_words", C.c_int32),
                 ("coo_T", C.c_int32), ("hyb_K", C.c_int64), ("codec", C.c_int32),
-                ("min_bits", C.c_int32)]
+                ("min_bits", C.c_int32), ("ell_kernel", C.c_int32)]
 
 
 class bro_info_t(C.Structure):
     _fields_ = [("m", C.c_int64), ("n", C.c_int64), ("nnz", C.c_int64),
                 ("dtype", C.c_int32), ("codec", C.c_int32), ("format", C.c_int32),
-                ("vec_words", C.c_int32), ("K", C.c_int64), ("nnz_ell", C.c_int64),
+                ("vec_words", C.c_int32), ("slice_h", C.c_int32), ("coo_T", C.c_int32),
+                ("ell_kernel", C.c_int32), ("reserved", C.c_int32),
+                ("K", C.c_int64), ("nnz_ell", C.c_int64),
                 ("nnz_coo", C.c_int64), ("n_slices", C.c_int64), ("ell_slots", C.c_int64),
                 ("ell_pitch", C.c_int64), ("n_intervals", C.c_int64),
                 ("ell_stream_bytes", C.c_int64), ("coo_stream_bytes", C.c_int64),
@@ -73,7 +72,7 @@ _sig = {
     "bro_export_encoded": (C.c_int, [_H, C.c_int32, _P, C.POINTER(C.c_size_t)]),
     "bro_decode_indices": (C.c_int, [_H, _P, _P, _P]),
     "bro_hyb_K": (C.c_int, [C.c_int64, _P, C.POINTER(C.c_int64)]),
-    "bro_reorder_bar": (C.c_int, [C.c_int64, C.c_int64, _P, _P, C.c_int, C.c_int32, _P]),
+    "bro_reorder_bar": (C.c_int, [C.c_int64, C.c_int64, _P, _P, C.c_int, C.c_int32, C.c_int32, _P]),
     "bro_status_str": (C.c_char_p, [C.c_int]),
     "bro_last_error": (C.c_char_p, []),
     "bro_version": (C.c_int, []),
@@ -172,7 +171,10 @@ def bro_spmv_scatter(h: int, x_dev_ptr: int, y_dst_ptrs, y_mc_ptr: int = 0, stre
 
 
 def bro_spmv_host(h: int, x: np.ndarray, y: np.ndarray, stream_ptr: int = 0):
-    assert x.flags.c_contiguous and y.flags.c_contiguous
+    """Raw call: x (n values) and y (m values) must be C-contiguous host arrays
+    of the handle's dtype (BroMatrix.spmv_host checks them)."""
+    if not (x.flags.c_contiguous and y.flags.c_contiguous):
+        raise ValueError("x and y must be C-contiguous")
     _check(_lib.bro_spmv_host(h, _ptr(x), _ptr(y), stream_ptr or None), "bro_spmv_host")
 
 
@@ -212,11 +214,11 @@ def bro_hyb_K(row_ptr) -> int:
     return K.value
 
 
-def bro_reorder_bar(m, n, row_ptr, col_idx, dtype=np.float64, method=0) -> np.ndarray:
+def bro_reorder_bar(m, n, row_ptr, col_idx, dtype=np.float64, method=0, window=0) -> np.ndarray:
     row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
     col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
     perm = np.zeros(m, dtype=np.int64)
-    _check(_lib.bro_reorder_bar(m, n, _ptr(row_ptr), _ptr(col_idx), _dtype_code(dtype), method,
+    _check(_lib.bro_reorder_bar(m, n, _ptr(row_ptr), _ptr(col_idx), _dtype_code(dtype), method, window,
                                 _ptr(perm)), "bro_reorder_bar")
     return perm
 
@@ -239,13 +241,17 @@ def bro_version() -> int:
 
 class BroMatrix:
     """Owns one libbro handle.  `fmt` in {"ell", "hyb", "coo"}; codec=1 gives
-    BRO-ELL / BRO-HYB / BRO-COO, codec=0 the uncompressed baseline."""
+    BRO-ELL / BRO-HYB / BRO-COO, codec=0 the uncompressed baseline.  Every
+    call checks the vectors' dtype, length, contiguity and device before the
+    pointers reach the library (the C ABI cannot)."""
 
-    def __init__(self, A, fmt="ell", codec=1, device=0, dtype=None, vec_words=0, hyb_K=-1, min_bits=0):
+    def __init__(self, A, fmt="ell", codec=1, device=0, dtype=None, vec_words=0, hyb_K=-1, min_bits=0,
+                 slice_h=0, coo_T=0, ell_kernel=0):
         vals = A.vals if dtype is None else A.vals.astype(dtype)
         self.dtype = np.dtype(vals.dtype)
         self.m, self.n, self.fmt, self.device = A.m, A.n, fmt, device
-        opts = bro_opts_default(codec=codec, vec_words=vec_words, hyb_K=hyb_K, min_bits=min_bits)
+        opts = bro_opts_default(codec=codec, vec_words=vec_words, hyb_K=hyb_K, min_bits=min_bits,
+                                slice_h=slice_h, coo_T=coo_T, ell_kernel=ell_kernel)
         if fmt == "ell":
             self.h = bro_create_ell(device, A.m, A.n, A.row_ptr, A.col, vals, opts)
         elif fmt == "hyb":
@@ -257,14 +263,23 @@ class BroMatrix:
             raise ValueError(fmt)
         self.info = bro_get_info(self.h)
 
+    def _tdtype(self):
+        import torch
+        return torch.float64 if self.dtype == np.float64 else torch.float32
+
+    def _check_vec(self, v, length, name):
+        if not (v.is_cuda and v.dtype == self._tdtype() and v.is_contiguous() and v.numel() == length
+                and (v.device.index or 0) == self.device):
+            raise ValueError(f"{name} must be a contiguous CUDA tensor of the matrix dtype ({self.dtype}), "
+                             f"{length} elements, on cuda:{self.device}")
+
     def spmv(self, x, y=None, stream=None):
         """y = A.x for torch CUDA tensors on the handle's device (async)."""
         import torch
-        tdt = torch.float64 if self.dtype == np.float64 else torch.float32
-        if not (x.is_cuda and x.dtype == tdt and x.is_contiguous() and x.numel() == self.n):
-            raise ValueError("x must be a contiguous CUDA tensor of the matrix dtype and length n")
+        self._check_vec(x, self.n, "x")
         if y is None:
-            y = torch.empty(self.m, dtype=tdt, device=x.device)
+            y = torch.empty(self.m, dtype=self._tdtype(), device=x.device)
+        self._check_vec(y, self.m, "y")
         if stream is None:
             stream = torch.cuda.current_stream(x.device)
         bro_spmv(self.h, x.data_ptr(), y.data_ptr(), stream.cuda_stream)
@@ -272,23 +287,40 @@ class BroMatrix:
 
     def spmv_scatter(self, x, y_dst_ptrs, y_mc_ptr=0, stream=None):
         """y = A.x stored into every device address of y_dst_ptrs (each m
-        values; the first is the local y) — the fused exchange of dist.py."""
+        values of the matrix dtype; the first is the local y) — the fused
+        exchange of dist.py."""
         import torch
-        tdt = torch.float64 if self.dtype == np.float64 else torch.float32
-        if not (x.is_cuda and x.dtype == tdt and x.is_contiguous() and x.numel() == self.n):
-            raise ValueError("x must be a contiguous CUDA tensor of the matrix dtype and length n")
+        self._check_vec(x, self.n, "x")
         if stream is None:
             stream = torch.cuda.current_stream(x.device)
         bro_spmv_scatter(self.h, x.data_ptr(), y_dst_ptrs, y_mc_ptr, stream.cuda_stream)
 
     def spmv_host(self, x: np.ndarray, y: np.ndarray = None, stream=None):
+        """End to end with host vectors (x: n values, y: m values)."""
+        x = np.ascontiguousarray(x, dtype=self.dtype)
+        if x.shape != (self.n,):
+            raise ValueError(f"x must have {self.n} elements")
         if y is None:
             y = np.empty(self.m, dtype=self.dtype)
+        if not (isinstance(y, np.ndarray) and y.dtype == self.dtype and y.shape == (self.m,)
+                and y.flags.c_contiguous and y.flags.writeable):
+            raise ValueError(f"y must be a writeable C-contiguous {self.dtype} array of {self.m} elements")
         sp = 0
         if stream is not None:
             sp = stream.cuda_stream
-        bro_spmv_host(self.h, np.ascontiguousarray(x, dtype=self.dtype), y, sp)
+        bro_spmv_host(self.h, x, y, sp)
         return y
+
+    def decode_indices(self):
+        """GPU decode through the handle's own kernels (decode mode): returns
+        (ell_cols, coo_rows) as torch int32 CUDA tensors (include/bro.h)."""
+        import torch
+        dev = torch.device("cuda", self.device)
+        cols = torch.empty(max(self.info["ell_slots"], 1), dtype=torch.int32, device=dev)
+        rows = torch.empty(max(self.info["nnz_coo"], 1), dtype=torch.int32, device=dev)
+        bro_decode_indices(self.h, cols.data_ptr(), rows.data_ptr(),
+                           torch.cuda.current_stream(dev).cuda_stream)
+        return cols[:self.info["ell_slots"]], rows[:self.info["nnz_coo"]]
 
     def export(self, part):
         return bro_export_encoded(self.h, part, self.dtype)

@@ -113,10 +113,10 @@ int64_t hyb_K(int64_t m, const int64_t* row_ptr) {
 // BRO-ELL
 // ---------------------------------------------------------------------------
 
-// MSB-first bit writer that emits 32-bit symbols to words[base + place(lane, q)].
+// MSB-first bit writer that emits 32-bit symbols to words[place(lane, q, S, V, h)].
 struct SymbolWriter {
   uint32_t* words;
-  int64_t lane, S, V;
+  int64_t lane, S, V, h;
   uint64_t acc = 0;
   int nb = 0;
   int64_t q = 0;
@@ -126,29 +126,30 @@ struct SymbolWriter {
     nb += b;
     if (nb >= 32) {
       nb -= 32;
-      words[place(lane, q++, S, V)] = uint32_t(acc >> nb);
+      words[place(lane, q++, S, V, h)] = uint32_t(acc >> nb);
       acc &= (nb ? ((uint64_t(1) << nb) - 1) : 0);
     }
   }
   void flush() {  // append the padding bits b_p (zeros) of P:L114
     if (nb > 0) {
-      words[place(lane, q++, S, V)] = uint32_t(acc << (32 - nb));
+      words[place(lane, q++, S, V, h)] = uint32_t(acc << (32 - nb));
       nb = 0;
       acc = 0;
     }
   }
 };
 
-void encode_bro_ell(const RowsView& A, int V, int VV, int min_bits, EllCode& out) {
+void encode_bro_ell(const RowsView& A, int h, int V, int VV, int min_bits, EllCode& out) {
   const int64_t m = A.m;
-  const int64_t s = (m + kH - 1) / kH;
+  const int64_t s = (m + h - 1) / h;
+  out.h = h;
   out.s = s;
   std::vector<uint64_t> ncol(s, 0), nsym(s, 0);
   // num_col: l_t = longest row of the slice (R9)
   parallel_for(s, [&](int64_t lo, int64_t hi) {
     for (int64_t t = lo; t < hi; ++t) {
       int64_t l = 0;
-      for (int64_t r = t * kH; r < std::min(m, t * kH + kH); ++r) l = std::max(l, A.len(r));
+      for (int64_t r = t * h; r < std::min(m, t * h + h); ++r) l = std::max(l, A.len(r));
       ncol[t] = (uint64_t)l;
     }
   });
@@ -159,7 +160,7 @@ void encode_bro_ell(const RowsView& A, int V, int VV, int min_bits, EllCode& out
   parallel_for(s, [&](int64_t lo, int64_t hi) {
     for (int64_t t = lo; t < hi; ++t) {
       uint8_t* ba = out.bit_alloc.data() + out.colptr[t];
-      for (int64_t r = t * kH; r < std::min(m, t * kH + kH); ++r) {
+      for (int64_t r = t * h; r < std::min(m, t * h + h); ++r) {
         const int32_t* c = A.col + A.row_ptr[r];
         const int64_t len = A.len(r);
         uint32_t prev1 = 0;  // 1-based previous column, c_{-1} = 0
@@ -179,20 +180,20 @@ void encode_bro_ell(const RowsView& A, int V, int VV, int min_bits, EllCode& out
     }
   });
   exclusive_scan(nsym, out.symptr);
-  out.words.assign(kH * out.symptr[s], 0u);
-  out.vals.resize(size_t(kH) * out.colptr[s] * A.vsize);
+  out.words.assign(size_t(h) * out.symptr[s], 0u);
+  out.vals.resize(size_t(h) * out.colptr[s] * A.vsize);
   // pack + multiplex and place values slot-wise
   parallel_for(s, [&](int64_t lo, int64_t hi) {
     for (int64_t t = lo; t < hi; ++t) {
       const uint8_t* ba = out.bit_alloc.data() + out.colptr[t];
       const int64_t l = (int64_t)ncol[t], S = (int64_t)nsym[t];
-      uint32_t* wbase = out.words.data() + kH * out.symptr[t];
-      uint8_t* vbase = out.vals.data() + size_t(kH) * out.colptr[t] * A.vsize;
-      for (int64_t lane = 0; lane < kH; ++lane) {
-        const int64_t r = t * kH + lane;
+      uint32_t* wbase = out.words.data() + size_t(h) * out.symptr[t];
+      uint8_t* vbase = out.vals.data() + size_t(h) * out.colptr[t] * A.vsize;
+      for (int64_t lane = 0; lane < h; ++lane) {
+        const int64_t r = t * h + lane;
         const int64_t len = r < m ? A.len(r) : 0;
         const int32_t* c = r < m ? A.col + A.row_ptr[r] : nullptr;
-        SymbolWriter w{wbase, lane, S, V};
+        SymbolWriter w{wbase, lane, S, V, h};
         uint32_t prev1 = 0;
         for (int64_t j = 0; j < l; ++j) {
           uint32_t d = 0;  // 0 = invalid (padding)
@@ -207,7 +208,7 @@ void encode_bro_ell(const RowsView& A, int V, int VV, int min_bits, EllCode& out
         if (r < m) {
           const uint8_t* src = A.vals + size_t(A.row_ptr[r]) * A.vsize;
           for (int64_t j = 0; j < len; ++j)
-            std::memcpy(vbase + size_t(place(lane, j, l, VV)) * A.vsize, src + size_t(j) * A.vsize, A.vsize);
+            std::memcpy(vbase + size_t(place(lane, j, l, VV, h)) * A.vsize, src + size_t(j) * A.vsize, A.vsize);
         }
       }
     }
@@ -232,13 +233,42 @@ void build_plain_ell(const RowsView& A, int64_t K, PlainEll& out) {
 }
 
 // ---------------------------------------------------------------------------
-// BRO-COO
+// BRO-COO (reading R13: lane l of interval i owns the T consecutive entries
+// e = i*32T + T*l + t; deltas in entry order, one width per interval)
 // ---------------------------------------------------------------------------
+
+// Lane-contiguous, chunk-multiplexed copy of per-entry arrays (reading R26):
+// entry (l, t) of interval i at i*32T + place(l, t, T, chunk); `fill` past nnz.
+template <class E>
+static void arrange(int64_t nnz, int T, int chunk, const E* src, E fill, int esize, uint8_t* dst, int64_t nI) {
+  const int64_t I = int64_t(kH) * T;
+  parallel_for(nI, [&](int64_t lo, int64_t hi) {
+    for (int64_t i = lo; i < hi; ++i)
+      for (int lane = 0; lane < kH; ++lane)
+        for (int t = 0; t < T; ++t) {
+          const int64_t e = i * I + int64_t(T) * lane + t;
+          uint8_t* d = dst + size_t(i * I + place(lane, t, T, chunk)) * esize;
+          if (e < nnz) std::memcpy(d, reinterpret_cast<const uint8_t*>(src) + size_t(e) * esize, esize);
+          else std::memcpy(d, &fill, esize);
+        }
+  }, 64);
+}
+
+static void arrange_col_vals(int64_t nnz, const int32_t* col, const uint8_t* vals, int vsize, int T,
+                             CooCode& out) {
+  const int64_t slots = out.nI * int64_t(kH) * T;
+  out.col.assign(slots, 0);
+  out.vals.resize(size_t(slots) * vsize);
+  arrange<int32_t>(nnz, T, 4, col, 0, 4, reinterpret_cast<uint8_t*>(out.col.data()), out.nI);
+  if (vsize == 8) arrange<double>(nnz, T, 2, reinterpret_cast<const double*>(vals), 0.0, 8, out.vals.data(), out.nI);
+  else arrange<float>(nnz, T, 4, reinterpret_cast<const float*>(vals), 0.0f, 4, out.vals.data(), out.nI);
+}
 
 void encode_bro_coo(int64_t nnz, const int32_t* row, const int32_t* col, const uint8_t* vals,
                     int vsize, int T, int V, CooCode& out) {
   const int64_t I = int64_t(kH) * T;
   const int64_t nI = (nnz + I - 1) / I;
+  out.T = T;
   out.nnz = nnz;
   out.nI = nI;
   out.base_row.assign(nI, 0);
@@ -248,14 +278,11 @@ void encode_bro_coo(int64_t nnz, const int32_t* row, const int32_t* col, const u
   parallel_for(nI, [&](int64_t lo, int64_t hi) {
     for (int64_t i = lo; i < hi; ++i) {
       const uint32_t base = at(i * I);
-      uint32_t dmax = 0;
-      for (int lane = 0; lane < kH; ++lane) {
-        uint32_t prev = base;
-        for (int t = 0; t < T; ++t) {
-          uint32_t r = at(i * I + int64_t(kH) * t + lane);
-          dmax = std::max(dmax, r - prev);
-          prev = r;
-        }
+      uint32_t dmax = 0, prev = base;
+      for (int64_t e = i * I; e < (i + 1) * I; ++e) {  // entry order = lane-major
+        const uint32_t r = at(e);
+        dmax = std::max(dmax, r - prev);
+        prev = r;
       }
       out.base_row[i] = base;
       out.width[i] = (uint8_t)gamma_bits(dmax);  // one width per interval
@@ -269,11 +296,11 @@ void encode_bro_coo(int64_t nnz, const int32_t* row, const int32_t* col, const u
       const int b = out.width[i];
       const int64_t S = (int64_t)nsym[i];
       uint32_t* wbase = out.words.data() + kH * out.symptr[i];
+      uint32_t prev = out.base_row[i];
       for (int lane = 0; lane < kH; ++lane) {
-        SymbolWriter w{wbase, lane, S, V};
-        uint32_t prev = out.base_row[i];
+        SymbolWriter w{wbase, lane, S, V, kH};
         for (int t = 0; t < T; ++t) {
-          uint32_t r = at(i * I + int64_t(kH) * t + lane);
+          const uint32_t r = at(i * I + int64_t(T) * lane + t);
           w.put(r - prev, b);
           prev = r;
         }
@@ -281,22 +308,20 @@ void encode_bro_coo(int64_t nnz, const int32_t* row, const int32_t* col, const u
       }
     }
   });
-  out.col.assign(col, col + nnz);
-  out.vals.resize(size_t(nnz) * vsize);
-  if (nnz) std::memcpy(out.vals.data(), vals, size_t(nnz) * vsize);
+  arrange_col_vals(nnz, col, vals, vsize, T, out);
 }
 
 void build_plain_coo(int64_t nnz, const int32_t* row, const int32_t* col, const uint8_t* vals,
                      int vsize, int T, CooCode& out) {
   const int64_t I = int64_t(kH) * T;
+  out.T = T;
   out.nnz = nnz;
   out.nI = (nnz + I - 1) / I;
-  out.row.assign(row, row + nnz);
-  out.col.assign(col, col + nnz);
-  out.vals.resize(size_t(nnz) * vsize);
-  if (nnz) std::memcpy(out.vals.data(), vals, size_t(nnz) * vsize);
   out.base_row.assign(out.nI, 0);
   for (int64_t i = 0; i < out.nI; ++i) out.base_row[i] = (uint32_t)row[i * I];
+  out.row.assign(out.nI * I, 0);
+  arrange<int32_t>(nnz, T, 4, row, nnz ? row[nnz - 1] : 0, 4, reinterpret_cast<uint8_t*>(out.row.data()), out.nI);
+  arrange_col_vals(nnz, col, vals, vsize, T, out);
 }
 
 // ---------------------------------------------------------------------------

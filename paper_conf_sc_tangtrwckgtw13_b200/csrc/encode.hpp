@@ -7,8 +7,10 @@
 
 namespace bro {
 
-constexpr int kH = 32;        // slice height = warp size (reading R10)
+constexpr int kH = 32;        // warp size: BRO-COO lanes per interval, BAR partition height
 constexpr int kSym = 32;      // sym_len in bits
+// BRO-ELL slice height h (P:L105 makes it a parameter; reading R10): 32 (one
+// row per lane of a warp) or 64 (two rows per lane)
 
 // Bytes of one value type.
 struct Bytes {
@@ -35,24 +37,30 @@ struct RowsView {
 };
 
 struct EllCode {                  // BRO-ELL
+  int h = 32;                     // slice height
   int64_t s = 0;                  // slices
   std::vector<uint64_t> colptr;   // s+1
   std::vector<uint64_t> symptr;   // s+1
   std::vector<uint8_t> bit_alloc; // colptr[s]
-  std::vector<uint32_t> words;    // 32*symptr[s]
-  Bytes vals;                     // 32*colptr[s] values
+  std::vector<uint32_t> words;    // h*symptr[s]
+  Bytes vals;                     // h*colptr[s] values
   int64_t max_l = 0;              // max num_col over slices
 };
 
-struct CooCode {                  // BRO-COO or plain COO
+// BRO-COO (reading R13) or plain COO: intervals of 32*T
+// entries, lane l owning the T consecutive entries i*32T + T*l + t; col,
+// vals (and plain rows) stored lane-contiguously in 16-byte chunks
+// (reading R26): entry (l, t) at i*32T + place(l, t, T, chunk).
+struct CooCode {
+  int T = 32;
   int64_t nnz = 0, nI = 0;
   std::vector<uint32_t> base_row; // nI
   std::vector<uint8_t> width;     // nI
   std::vector<uint64_t> symptr;   // nI+1
   std::vector<uint32_t> words;    // 32*symptr[nI]
-  std::vector<int32_t> row;       // plain COO only
-  std::vector<int32_t> col;       // nnz
-  Bytes vals;                     // nnz
+  std::vector<int32_t> row;       // plain COO only, nI*32T
+  std::vector<int32_t> col;       // nI*32T
+  Bytes vals;                     // nI*32T
 };
 
 struct PlainEll {                 // ELLPACK, column-major
@@ -61,13 +69,13 @@ struct PlainEll {                 // ELLPACK, column-major
   Bytes vals;                     // K*pitch
 };
 
-// Position of item q of lane r in a block of 32 lanes x S items grouped in
+// Position of item q of row r in a block of h rows x S items grouped in
 // chunks of V (tail chunk S - V*floor(S/V)).
-inline int64_t place(int64_t r, int64_t q, int64_t S, int64_t V) {
+inline int64_t place(int64_t r, int64_t q, int64_t S, int64_t V, int64_t h = kH) {
   const int64_t F = S / V;
   const int64_t c = q / V;
-  if (c < F) return kH * V * c + r * V + (q - c * V);
-  return kH * V * F + r * (S - V * F) + (q - V * F);
+  if (c < F) return h * V * c + r * V + (q - c * V);
+  return h * V * F + r * (S - V * F) + (q - V * F);
 }
 
 inline int gamma_bits(uint32_t u) { return u ? 32 - __builtin_clz(u) : 0; }
@@ -78,7 +86,7 @@ std::string check_coo(int64_t m, int64_t n, int64_t nnz, const int32_t* row, con
 
 int64_t hyb_K(int64_t m, const int64_t* row_ptr);
 
-void encode_bro_ell(const RowsView& A, int V, int value_chunk, int min_bits, EllCode& out);
+void encode_bro_ell(const RowsView& A, int h, int V, int value_chunk, int min_bits, EllCode& out);
 void build_plain_ell(const RowsView& A, int64_t K, PlainEll& out);
 // rows: int32 rows of the COO entries (sorted); T steps per interval.
 void encode_bro_coo(int64_t nnz, const int32_t* row, const int32_t* col, const uint8_t* vals,

@@ -1,0 +1,65 @@
+// BRO-ELL instance table (included by kern_ell64.cu / kern_ell32.cu, one
+// translation unit per value type so the two compile in parallel).
+//
+// Instances (R = rows per lane: 1 for h = 32, 2 for h = 64):
+//   TINY  every slice <= 4 columns: register-resident decode
+//   FEW   fewer slices than resident warps (R = 1): 16 (fp64) / 32 (fp32)
+//         columns in flight per warp at ~128 registers — every warp is
+//         resident anyway, so registers buy memory-level parallelism
+//   SMALL every row stream < 10 symbols: 10-row window (less shared memory,
+//         more L1 for the x gather)
+//   MID   < 18 symbols: 18-row window
+//   GEN   any slice: 34-row window
+// Launch bounds fix the register budget: kMinBlocks blocks of kWarps warps.
+#pragma once
+#include "kernels.cuh"
+#include "launch.hpp"
+
+namespace bro {
+
+template <typename T, int V, int R, int M>
+KernelRef ell_pick(int inst) {
+  using namespace dev;
+  constexpr bool f64 = sizeof(T) == 8;
+  if (inst == ELL_FEW && R == 2) inst = ELL_GEN;
+  if constexpr (R == 1) {
+    switch (inst) {
+      case ELL_TINY: return {(const void*)&bro_ell_tiny<T, V, 1, 8, f64 ? 5 : 6, M>, 256};
+      case ELL_FEW:
+        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 1, 8, 2, 16, kEllRowsGen, M>, 256};
+        else return {(const void*)&bro_ell_od<T, V, 1, 4, 2, 32, kEllRowsGen, M>, 128};
+      case ELL_SMALL: return {(const void*)&bro_ell_od<T, V, 1, 16, 2, 8, kEllRowsSmall, M>, 512};
+      case ELL_MID: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M>, 256};
+      case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsGen, M>, 256};
+    }
+  } else {
+    switch (inst) {
+      case ELL_TINY: return {(const void*)&bro_ell_tiny<T, V, 2, 8, 4, M>, 256};
+      case ELL_SMALL: return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsSmall, M>, 256};
+      case ELL_MID: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M>, 256};
+      case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 2, 4, 4, 4, kEllRowsGen, M>, 128};
+    }
+  }
+  return {};
+}
+
+template <typename T, int V, int R>
+KernelRef ell_pick_mode(int inst, int mode) {
+  switch (mode) {
+    case 0: return ell_pick<T, V, R, dev::kSpmv>(inst);
+    case 1: return ell_pick<T, V, R, dev::kScatter>(inst);
+    case 2: return ell_pick<T, V, R, dev::kDecode>(inst);
+  }
+  return {};
+}
+
+template <typename T>
+KernelRef bro_ell_ref_impl(int V, int R, int inst, int mode) {
+  if (V == 1 && R == 1) return ell_pick_mode<T, 1, 1>(inst, mode);
+  if (V == 1 && R == 2) return ell_pick_mode<T, 1, 2>(inst, mode);
+  if (V == 4 && R == 1) return ell_pick_mode<T, 4, 1>(inst, mode);
+  if (V == 4 && R == 2) return ell_pick_mode<T, 4, 2>(inst, mode);
+  return {};
+}
+
+}  // namespace bro

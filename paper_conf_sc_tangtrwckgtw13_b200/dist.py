@@ -181,7 +181,7 @@ class RowBlockSpmv:
     """This rank's block of A as libbro handle(s) plus the iteration buffers."""
 
     def __init__(self, A, rank: int, world: int, device, fmt="ell", codec=1, dtype=None,
-                 bounds=None, vec_words=0, exchange="allgather", group=None):
+                 bounds=None, vec_words=0, exchange="allgather", group=None, **layout):
         import torch
         from .bro import BroMatrix
         if exchange not in EXCHANGES:
@@ -202,7 +202,8 @@ class RowBlockSpmv:
         n_pad = world * M
         self.nnz_local = b - a
         dev_index = device.index or 0
-        mk = dict(fmt=fmt, codec=codec, device=dev_index, dtype=dtype, vec_words=vec_words)
+        # layout: BroMatrix options (slice_h, coo_T, ell_kernel, ...)
+        mk = dict(fmt=fmt, codec=codec, device=dev_index, dtype=dtype, vec_words=vec_words, **layout)
         # the whole block (kernel-only timing, allgather / p2p modes)
         self.mat = BroMatrix(_Rows(rp, col, vals, 0, r1 - r0, n_pad), **mk)
         self.tdt = torch.float64 if self.mat.dtype == np.float64 else torch.float32

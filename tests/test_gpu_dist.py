@@ -79,14 +79,14 @@ def test_row_block_single_rank_iteration(lib, dev):
     x0 = make_x(A.n, 1) * 0.1
     blk = RowBlockSpmv(A, 0, 1, dev, fmt="ell")
     blk.set_x(x0)
+    prev = x0.copy()
     for _ in range(3):
         blk.step()
-    torch.cuda.synchronize()
-    got = blk.x_current().cpu().numpy()
-    ref = x0.copy()
-    for _ in range(3):
-        ref = np.asarray(spmv.csr_spmv(A.row_ptr, A.col, A.vals, ref)[0], dtype=np.float64)
-    assert np.allclose(got, ref, rtol=1e-12, atol=0)
+        torch.cuda.synchronize()
+        got = blk.x_current().cpu().numpy()
+        y_ref, S = spmv.csr_spmv(A.row_ptr, A.col, A.vals, prev)
+        assert spmv.within_tolerance(got, y_ref, S, 1e-12)[0].all()
+        prev = got
     blk.close()
 
 
@@ -118,14 +118,17 @@ def _dist_worker(rank, world, port, q, exchange, fmt, cfg, iters):
         blk = RowBlockSpmv(A, rank, world, dev, fmt=fmt, bounds=bounds, exchange=exchange)
         blk.set_x(x0)
         stream = torch.cuda.current_stream(dev)
+        # every iteration, every row: x_{k+1} within 1e-12 * S_i of the
+        # oracle's A.x_k applied to the GPU's own x_k (north_star bound)
+        ok = True
+        prev = x0.copy()
         for _ in range(iters):
             blk.step(stream)
-        torch.cuda.synchronize()
-        got = blk.x_current().cpu().numpy()
-        ref = x0.copy()
-        for _ in range(iters):
-            ref = np.asarray(spmv.csr_spmv(A.row_ptr, A.col, A.vals, ref)[0], dtype=np.float64)
-        ok = bool(np.allclose(got, ref, rtol=1e-11, atol=0))
+            torch.cuda.synchronize()
+            got = blk.x_current().cpu().numpy()
+            y_ref, S = spmv.csr_spmv(A.row_ptr, A.col, A.vals, prev)
+            ok = ok and bool(spmv.within_tolerance(got, y_ref, S, 1e-12)[0].all())
+            prev = got
         q.put((rank, ok, getattr(blk, "split", None), ""))
         dist.barrier()
         blk.close()

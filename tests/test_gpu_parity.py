@@ -2,12 +2,18 @@
 
 Bar (north_star): decoded index streams bit-exact; fp64 y within
 1e-12 * sum_j |a_ij||x_j| per row, fp32 within 1e-5 * the same sum.
+
+Decoded indices come from the SAME kernel instances bro_spmv runs (their
+decode mode, include/bro.h bro_decode_indices) and are compared with the
+matrix's own column / row indices placed in the decode layout: the oracle's
+decode(encode(idx)) == idx round trips (tests/test_oracle_bro.py) make that
+the oracle's decode too.
 """
 import numpy as np
 import pytest
 
-from gen import Csr, make_config, make_x, random_csr, row_block
-from oracle import bro_coo, bro_ell, hyb, spmv
+from gen import Csr, dense_band, make_config, make_x, permute_rows, random_csr, row_block
+from oracle import hyb, spmv
 
 torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
@@ -22,8 +28,8 @@ def dev():
     return torch.device("cuda:0")
 
 
-def _run(lib, A, fmt, codec, dtype, dev, V=4, x=None, stream=None):
-    M = lib.BroMatrix(A, fmt=fmt, codec=codec, device=0, dtype=dtype, vec_words=V)
+def _run(lib, A, fmt, codec, dtype, dev, x=None, stream=None, **kw):
+    M = lib.BroMatrix(A, fmt=fmt, codec=codec, device=0, dtype=dtype, **kw)
     if x is None:
         x = make_x(A.n, 3, dtype)
     xd = torch.from_numpy(np.ascontiguousarray(x, dtype=dtype)).to(dev)
@@ -32,11 +38,66 @@ def _run(lib, A, fmt, codec, dtype, dev, V=4, x=None, stream=None):
     return M, x, y.cpu().numpy()
 
 
-def _check_y(A, x, y, dtype):
-    y_ref, S = spmv.csr_spmv(A.row_ptr, A.col, A.vals.astype(dtype), x.astype(dtype))
-    ok, err = spmv.within_tolerance(y, y_ref, S, TOL[dtype])
-    bad = np.nonzero(~ok)[0]
-    assert ok.all(), f"{bad.size} rows out of tolerance, first {bad[:5]}, err {err[bad[:5]]}"
+def _check_y(A, x, y, dtype, chunk_rows=None):
+    """Every row within tol * S_i of the oracle (chunked over rows for the
+    full-size configs: each chunk is an exact row block of the oracle)."""
+    rows = [(0, A.m)] if chunk_rows is None else [(r, min(A.m, r + chunk_rows))
+                                                  for r in range(0, A.m, chunk_rows)]
+    for r0, r1 in rows:
+        B = row_block(A, r0, r1) if chunk_rows is not None else A
+        y_ref, S = spmv.csr_spmv(B.row_ptr, B.col, B.vals.astype(dtype), x.astype(dtype))
+        ok, err = spmv.within_tolerance(y[r0:r1], y_ref, S, TOL[dtype])
+        bad = np.nonzero(~ok)[0]
+        assert ok.all(), f"rows {r0}+: {bad.size} out of tolerance, first {bad[:5] + r0}, err {err[bad[:5]]}"
+
+
+def ell_slot_reference(row_ptr, col, m, h):
+    """Decoded column of every ELL slot, slot h*colptr[t] + h*j + r (V = 1
+    slot order, include/bro.h), -1 for padding, built from the CSR itself."""
+    row_ptr = np.asarray(row_ptr, dtype=np.int64)
+    lens = np.diff(row_ptr)
+    s = -(-m // h)
+    lp = np.zeros(s * h, dtype=np.int64)
+    lp[:m] = lens
+    colptr = np.zeros(s + 1, dtype=np.int64)
+    np.cumsum(lp.reshape(s, h).max(axis=1) if s else lp[:0], out=colptr[1:])
+    out = np.full(h * int(colptr[-1]), -1, dtype=np.int32)
+    nnz = int(row_ptr[-1])
+    rows = np.repeat(np.arange(m, dtype=np.int64), lens)
+    pos = np.arange(nnz, dtype=np.int64) - np.repeat(row_ptr[:-1], lens)
+    out[h * colptr[rows // h] + h * pos + rows % h] = col
+    return out
+
+
+def check_decode(M, A, K=None):
+    """Every slot of the ELL part and every COO row, bit-exact."""
+    info = M.info
+    cols_d, rows_d = M.decode_indices()
+    torch.cuda.synchronize()
+    if info["format"] == 0:        # ELL
+        ep, ec = A.row_ptr, A.col
+        cr = np.zeros(0, np.int64)
+    elif info["format"] == 2:      # HYB
+        ep, ec, _, cr, _, _ = hyb.hyb_split(A.row_ptr, A.col, A.vals, info["K"])
+    else:                          # COO
+        ep = None
+        cr = np.repeat(np.arange(A.m, dtype=np.int64), np.diff(A.row_ptr))
+    if ep is not None:
+        if info["codec"]:
+            ref = ell_slot_reference(ep, ec, A.m, info["slice_h"])
+            got = cols_d.cpu().numpy()
+        else:
+            Cm, _ = hyb.ell_arrays(ep, ec, np.zeros(ec.size), info["K"])
+            ref = np.full((info["K"], info["ell_pitch"]), -1, dtype=np.int32)
+            ref[:, :A.m] = Cm.T
+            ref = ref.ravel()
+            got = cols_d.cpu().numpy()
+        assert got.size == ref.size
+        bad = np.nonzero(got != ref)[0]
+        assert bad.size == 0, f"{bad.size} ELL slots differ, first {bad[:5]}: {got[bad[:5]]} vs {ref[bad[:5]]}"
+    if info["nnz_coo"]:
+        got = rows_d.cpu().numpy()
+        assert np.array_equal(got, cr.astype(np.int32)), "COO rows differ"
 
 
 CASES = [
@@ -56,80 +117,87 @@ def test_spmv_random(lib, dev, name, mk, fmt, codec, dtype):
     A = mk()
     M, x, y = _run(lib, A, fmt, codec, dtype, dev)
     _check_y(A, x, y, dtype)
+    if name != "wide":
+        check_decode(M, A)
     M.close()
 
 
-@pytest.mark.parametrize("V", [1, 2, 4])
-def test_vec_words_variants(lib, dev, V):
-    A = random_csr(2000, 3000, 5, max_len=90, empty_frac=0.05, long_frac=0.01, long_len=600)
-    for fmt in ("ell", "hyb"):
-        M, x, y = _run(lib, A, fmt, 1, np.float64, dev, V=V)
-        _check_y(A, x, y, np.float64)
-        M.close()
-
-
-# "wide" (n = 2^31 - 1) is left out: its 16 GB x dominates the run time and it
-# is already covered by test_spmv_random
+# "wide" (n = 2^31 - 1) is left out below: its 16 GB x dominates the run time
+# and it is covered by test_spmv_random
 SMALL_CASES = [c for c in CASES if c[0] != "wide"]
-BULK_CASES = SMALL_CASES + [
+INSTANCE_CASES = SMALL_CASES + [
     ("multiblock", lambda: random_csr(3000, 4000, 12, max_len=90, empty_frac=0.05)),
-    ("short", lambda: random_csr(5000, 7000, 13, max_len=3, empty_frac=0.1)),
+    ("short", lambda: random_csr(5000, 7000, 13, max_len=4, empty_frac=0.1)),
+    ("wide31", lambda: random_csr(333, 2**20, 17, max_len=4, wide_cols=True)),
+    ("mixed", lambda: random_csr(4000, 9000, 18, max_len=12, long_frac=0.05, long_len=300)),
 ]
 
 
-@pytest.mark.parametrize("kernel", ["bulk", "od"])
-@pytest.mark.parametrize("ring_kb", ["", "1", "64"])
+def _fits(A, h, inst):
+    from oracle import bro_ell
+    if A.m == 0:
+        return inst == 5
+    l, S, _ = bro_ell.slice_shapes(A.row_ptr, A.col, A.m, h, 32)
+    return {1: l.max(initial=0) <= 4, 2: True, 3: S.max(initial=0) < 10, 4: S.max(initial=0) < 18, 5: True}[inst]
+
+
+@pytest.mark.parametrize("inst", [1, 2, 3, 4, 5])
+@pytest.mark.parametrize("h", [32, 64])
+@pytest.mark.parametrize("V", [1, 4])
 @pytest.mark.parametrize("dtype", [np.float64, np.float32])
-def test_bro_ell_v1_kernels(lib, dev, kernel, ring_kb, dtype, monkeypatch):
-    """V = 1 (the paper's multiplexing): the bulk-staged kernel (TMA ring of
-    whole slices, 2..8 slots per warp depending on BRO_RING_KB) and the
-    register-staged kernel give the oracle's y on every case, including slices
-    with several 32-column blocks and slices too large to stage."""
-    monkeypatch.setenv("BRO_ELL_KERNEL", "1" if kernel == "od" else "2")
-    monkeypatch.setenv("BRO_RING_KB", ring_kb)
-    for _, mk in BULK_CASES:
+def test_ell_instances(lib, dev, inst, h, V, dtype):
+    """Every BRO-ELL kernel instance (bro_opts_t.ell_kernel: tiny, few-slice,
+    small / mid / general window) at h = 32 and 64, V = 1 and 4, gives the
+    oracle's y on every row and decodes every slot bit-exactly, for the
+    matrices it fits (empty rows, h not dividing m, 31-bit deltas, several
+    32-column blocks per slice)."""
+    ran = 0
+    for name, mk in INSTANCE_CASES:
         A = mk()
         for fmt in ("ell", "hyb"):
-            M, x, y = _run(lib, A, fmt, 1, dtype, dev, V=1)
+            if fmt == "hyb":
+                K = hyb.hyb_K(A.row_ptr)
+                ep, ec, ev, _, _, _ = hyb.hyb_split(A.row_ptr, A.col, A.vals, K)
+                E = Csr(A.m, A.n, ep, ec, ev)
+            else:
+                E = A
+            if not _fits(E, h, inst):
+                continue
+            M, x, y = _run(lib, A, fmt, 1, dtype, dev, vec_words=V, slice_h=h, ell_kernel=inst)
+            assert M.info["ell_kernel"] == inst and M.info["slice_h"] == h
             _check_y(A, x, y, dtype)
+            check_decode(M, A)
             M.close()
+            ran += 1
+    assert ran > 0
 
 
-@pytest.mark.parametrize("short", ["0", "1"])
-@pytest.mark.parametrize("V", [1, 2, 4])
-@pytest.mark.parametrize("dtype", [np.float64, np.float32])
-def test_short_slice_kernel(lib, dev, short, V, dtype, monkeypatch):
-    """Slices of <= 4 columns (the ELL part of webbase-like HYB) run in the
-    short-slice instance (G = 4, 6-row window, more resident warps); it and
-    the general instance give the oracle's y, with empty rows, h not dividing
-    m and 31-bit deltas."""
-    monkeypatch.setenv("BRO_ELL_SHORT", short)
-    for A in (random_csr(5001, 7000, 16, max_len=4, empty_frac=0.2),
-              random_csr(333, 2**20, 17, max_len=4, wide_cols=True),
-              random_csr(4000, 9000, 18, max_len=12, long_frac=0.05, long_len=300)):
-        for fmt in ("ell", "hyb"):
-            M, x, y = _run(lib, A, fmt, 1, dtype, dev, V=V)
-            _check_y(A, x, y, dtype)
-            M.close()
+COO_CASES = SMALL_CASES + [
+    ("longrow", lambda: random_csr(40, 20000, 14, max_len=5, long_frac=0.2, long_len=5000)),
+    ("tail", lambda: random_csr(300, 400, 15, max_len=4)),
+    ("one_row", lambda: random_csr(1, 60000, 23, max_len=0, long_frac=1.0, long_len=40000)),
+    ("many", lambda: random_csr(40000, 50000, 21, max_len=6, empty_frac=0.2, long_frac=0.002, long_len=900)),
+]
 
 
-@pytest.mark.parametrize("upi", ["1", "2", "4"])
+@pytest.mark.parametrize("T", [8, 16, 32])
 @pytest.mark.parametrize("codec", [1, 0])
 @pytest.mark.parametrize("dtype", [np.float64, np.float32])
-def test_coo_work_units(lib, dev, upi, codec, dtype, monkeypatch):
-    """COO traversal split into 1, 2 or 4 work units per 1024-entry interval
-    (carries per unit, deterministic fix-up over units) gives the oracle's y,
-    including units entirely past nnz and rows spanning many units."""
-    monkeypatch.setenv("BRO_COO_UPI", upi)
-    cases = SMALL_CASES + [("longrow", lambda: random_csr(40, 20000, 14, max_len=5, long_frac=0.2,
-                                                    long_len=5000)),
-                     ("tail", lambda: random_csr(300, 400, 15, max_len=4))]
-    for _, mk in cases:
+def test_coo_intervals(lib, dev, T, codec, dtype):
+    """(BRO-)COO with 8, 16 and 32 entries per lane: rows spanning many lanes
+    and intervals (deterministic fix-up), ragged last intervals, one-row
+    intervals (width 0), lanes entirely past nnz; y on every row, rows
+    decoded bit-exactly, and the same bits on a second call."""
+    for _, mk in COO_CASES:
         A = mk()
         for fmt in ("coo", "hyb"):
-            for V in (1, 4):
-                M, x, y = _run(lib, A, fmt, codec, dtype, dev, V=V)
+            for V in ((1, 4) if codec else (4,)):
+                M, x, y = _run(lib, A, fmt, codec, dtype, dev, vec_words=V, coo_T=T)
+                assert M.info["coo_T"] == T
                 _check_y(A, x, y, dtype)
+                check_decode(M, A)
+                y2 = M.spmv(torch.from_numpy(x).to(dev)).cpu().numpy()
+                assert np.array_equal(y, y2)
                 M.close()
 
 
@@ -156,36 +224,39 @@ def test_single_long_row_spans_intervals(lib, dev):
 
 
 def test_x_with_inf_outside_pattern(lib, dev):
-    """Padding slots never read x (Alg. 1 line 17 skips invalid slots)."""
+    """Padding slots never read x (Alg. 1 line 17 skips invalid slots), nor
+    do COO slots past nnz."""
     A = random_csr(300, 400, 6, max_len=30, empty_frac=0.2)
     x = make_x(A.n, 1)
     used = np.zeros(A.n, bool)
     used[A.col] = True
     x[~used] = np.inf
+    x[0] = np.inf if not used[0] else x[0]
     for fmt in ("ell", "hyb", "coo"):
-        M, _, y = _run(lib, A, fmt, 1, np.float64, dev, x=x)
-        assert np.all(np.isfinite(y))
-        _check_y(A, x, y, np.float64)
-        M.close()
+        for h in (32, 64):
+            M, _, y = _run(lib, A, fmt, 1, np.float64, dev, x=x, slice_h=h)
+            assert np.all(np.isfinite(y))
+            _check_y(A, x, y, np.float64)
+            M.close()
 
 
-def test_decode_parity_bit_exact(lib, dev):
-    A = random_csr(3000, 100000, 8, max_len=60, empty_frac=0.1, long_frac=0.02, long_len=500,
-                   wide_cols=True)
-    for V in (1, 4):
-        M = lib.BroMatrix(A, fmt="hyb", codec=1, device=0, vec_words=V)
-        info = M.info
-        cols_d = torch.empty(info["ell_slots"], dtype=torch.int32, device=dev)
-        rows_d = torch.empty(max(info["nnz_coo"], 1), dtype=torch.int32, device=dev)
-        lib.bro_decode_indices(M.h, cols_d.data_ptr(), rows_d.data_ptr(), 0)
-        torch.cuda.synchronize()
-        K = info["K"]
-        ep, ec, ev, cr, cc, cv = hyb.hyb_split(A.row_ptr, A.col, A.vals, K)
-        E = bro_ell.encode(ep, ec, ev, A.m, A.n, V=V)
-        assert np.array_equal(cols_d.cpu().numpy(), bro_ell.decoded_slots(E))
-        C = bro_coo.encode(cr, cc, cv, V=V)
-        assert np.array_equal(rows_d.cpu().numpy()[:info["nnz_coo"]], bro_coo.decode_rows(C))
-        M.close()
+def test_vector_checks(lib, dev):
+    """The binding rejects a y of the wrong dtype, length or device before
+    any pointer reaches the library."""
+    A = random_csr(64, 50, 11)
+    M = lib.BroMatrix(A, fmt="ell", device=0)
+    x = torch.zeros(50, dtype=torch.float64, device=dev)
+    for y in (torch.zeros(64, dtype=torch.float32, device=dev), torch.zeros(63, dtype=torch.float64, device=dev),
+              torch.zeros(128, dtype=torch.float64, device=dev)[::2], torch.zeros(64, dtype=torch.float64)):
+        with pytest.raises(ValueError):
+            M.spmv(x, y)
+    with pytest.raises(ValueError):
+        M.spmv(torch.zeros(49, dtype=torch.float64, device=dev))
+    with pytest.raises(ValueError):
+        M.spmv_host(np.zeros(49))
+    with pytest.raises(ValueError):
+        M.spmv_host(np.zeros(50), np.zeros(64, np.float32))
+    M.close()
 
 
 def test_deterministic(lib, dev):
@@ -214,6 +285,22 @@ def test_side_stream_and_host_e2e(lib, dev):
     M.close()
 
 
+@pytest.mark.parametrize("h", [32, 64])
+@pytest.mark.parametrize("codec", [1, 0])
+def test_host_e2e_pipelined(lib, dev, h, codec):
+    """ELL-only handles with x >= 4 MB run bro_spmv_host as the 8-piece
+    pipeline (x pieces, row blocks gated by their column ranges, y pieces):
+    bitwise equal to bro_spmv."""
+    A = random_csr(600_000, 600_000, 31, max_len=12, empty_frac=0.05)
+    M = lib.BroMatrix(A, fmt="ell", codec=codec, device=0, slice_h=h)
+    x = make_x(A.n, 6)
+    y = M.spmv(torch.from_numpy(x).to(dev)).cpu().numpy()
+    y_host = M.spmv_host(x)
+    assert np.array_equal(y, y_host)
+    _check_y(A, x, y, np.float64)
+    M.close()
+
+
 def test_alias_rejected(lib, dev):
     A = random_csr(64, 64, 11)
     M = lib.BroMatrix(A, fmt="ell", device=0)
@@ -223,81 +310,74 @@ def test_alias_rejected(lib, dev):
     M.close()
 
 
+@pytest.mark.parametrize("min_bits", [1, 16, 31])
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_forced_widths_dense(lib, dev, min_bits, dtype):
+    """Fig. 3 analog (NEXT-3): the dense matrix with every width
+    forced up to min_bits runs the same kernels; y on every row and every
+    slot decoded bit-exactly."""
+    A = dense_band(50_000, 32)
+    for h in (32, 64):
+        M, x, y = _run(lib, A, "ell", 1, dtype, dev, min_bits=min_bits, slice_h=h)
+        _check_y(A, x, y, dtype)
+        check_decode(M, A)
+        M.close()
+
+
 # ---------------------------------------------------------------- the five configs
 
 @pytest.mark.parametrize("cfg,fmt", [(1, "ell"), (2, "ell"), (3, "hyb")])
 @pytest.mark.parametrize("codec", [1, 0])
 def test_configs_full_oracle(lib, dev, cfg, fmt, codec):
+    """C1-C3, both dtypes, bench.py's handle options: every row vs the
+    oracle, every slot / COO row decoded bit-exactly."""
     for dtype in (np.float64, np.float32):
         A = make_config(cfg, dtype)
         M, x, y = _run(lib, A, fmt, codec, dtype, dev, x=make_x(A.n, cfg, dtype))
         _check_y(A, x, y, dtype)
+        check_decode(M, A)
         M.close()
 
 
 def test_config4_bar_reordered_hyb(lib, dev):
     """C4: random-block, reordered with BAR (signature clustering), BRO-HYB
-    fp32 and fp64 vs the oracle on every row."""
-    from gen import permute_rows
+    fp32 and fp64 vs the oracle on every row, every index decoded."""
     A0 = make_config(4)
     perm = lib.bro_reorder_bar(A0.m, A0.n, A0.row_ptr, A0.col, method=0)
     A = permute_rows(A0, perm)
     for dtype in (np.float64, np.float32):
         M, x, y = _run(lib, A, "hyb", 1, dtype, dev, x=make_x(A.n, 4, dtype))
         _check_y(A, x, y, dtype)
+        check_decode(M, A)
         M.close()
+        Mb, x, y = _run(lib, A, "hyb", 0, dtype, dev, x=make_x(A.n, 4, dtype))
+        _check_y(A, x, y, dtype)
+        Mb.close()
 
 
-def test_config5_full_size(lib, dev):
-    """C5 at full size in bench.py's launch configuration: every row against
-    the closed form (x = 1 -> y_i = 27 - len_i exactly), sampled rows against
-    the oracle for random x, and sampled slices decoded bit-exactly."""
-    A = make_config(5)
-    M = lib.BroMatrix(A, fmt="ell", codec=1, device=0)
-    ones = torch.ones(A.n, dtype=torch.float64, device=dev)
-    y = M.spmv(ones).cpu().numpy()
-    assert np.array_equal(y, 27.0 - A.row_lengths())
-    x = make_x(A.n, 5)
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+@pytest.mark.parametrize("h", [0, 32])
+def test_config5_full_size(lib, dev, dtype, h):
+    """C5 at full size in bench.py's launch configuration (h = 0: auto) and
+    at h = 32: x = 1 gives y_i = 27 - len_i exactly (small integers); random
+    x: EVERY row against the oracle (chunked row blocks); every slot of the
+    8M-row BRO-ELL decoded bit-exactly."""
+    A = make_config(5, dtype)
+    M = lib.BroMatrix(A, fmt="ell", codec=1, device=0, dtype=dtype, slice_h=h)
+    tdt = torch.float64 if dtype == np.float64 else torch.float32
+    y = M.spmv(torch.ones(A.n, dtype=tdt, device=dev)).cpu().numpy()
+    assert np.array_equal(y, (27.0 - A.row_lengths()).astype(dtype))
+    x = make_x(A.n, 5, dtype)
     y = M.spmv(torch.from_numpy(x).to(dev)).cpu().numpy()
-    rows = np.unique(np.concatenate([np.arange(40), A.m - 1 - np.arange(40),
-                                     np.random.default_rng(0).integers(0, A.m, 3000)]))
-    yr, S = spmv.csr_spmv_rows(A.row_ptr, A.col, A.vals, x, rows)
-    ok, err = spmv.within_tolerance(y[rows], yr, S, 1e-12)
-    assert ok.all(), float(err.max())
-    cols_d = torch.empty(M.info["ell_slots"], dtype=torch.int32, device=dev)
-    lib.bro_decode_indices(M.h, cols_d.data_ptr(), 0, 0)
-    cols = cols_d.cpu().numpy()
-    sample = [0, 3, 6250, 125000, 249999]
-    E = bro_ell.encode(A.row_ptr, A.col, A.vals, A.m, A.n, slices=sample)
-    ref = bro_ell.decoded_slots(E, slices=sample)
-    for t in sample:
-        a, b = 32 * int(E.colptr[t]), 32 * int(E.colptr[t + 1])
-        assert np.array_equal(cols[a:b], ref[a:b])
-    M.close()
-
-
-def test_config5_full_size_f32(lib, dev):
-    """C5 fp32 at full size (bench.py --dtype f32's launch configuration):
-    x = 1 gives small integers, exact in fp32 (y_i = 27 - len_i); sampled
-    rows against the oracle within 1e-5 * sum|a||x| for random x."""
-    A = make_config(5, np.float32)
-    M = lib.BroMatrix(A, fmt="ell", codec=1, device=0, dtype=np.float32)
-    ones = torch.ones(A.n, dtype=torch.float32, device=dev)
-    y = M.spmv(ones).cpu().numpy()
-    assert np.array_equal(y, (27.0 - A.row_lengths()).astype(np.float32))
-    x = make_x(A.n, 5, np.float32)
-    y = M.spmv(torch.from_numpy(x).to(dev)).cpu().numpy()
-    rows = np.unique(np.concatenate([np.arange(40), A.m - 1 - np.arange(40),
-                                     np.random.default_rng(2).integers(0, A.m, 3000)]))
-    yr, S = spmv.csr_spmv_rows(A.row_ptr, A.col, A.vals.astype(np.float32), x, rows)
-    ok, err = spmv.within_tolerance(y[rows], yr, S, TOL[np.float32])
-    assert ok.all(), float(err.max())
+    _check_y(A, x, y, dtype, chunk_rows=1_000_000)
+    check_decode(M, A)
     M.close()
 
 
 def test_config5_row_blocks(lib, dev):
     """Row-block partition used by the multi-GPU driver: local blocks with
-    global columns reproduce the global product (one GPU, 4 blocks)."""
+    global columns reproduce the global product (one GPU, 4 blocks), every
+    row within the oracle's bound."""
     from paper_conf_sc_tangtrwckgtw13_b200.dist import partition_rows
     A = make_config(5)
     x = make_x(A.n, 5)
@@ -310,7 +390,4 @@ def test_config5_row_blocks(lib, dev):
         ys.append(M.spmv(xd).cpu().numpy())
         M.close()
     y = np.concatenate(ys)
-    rows = np.random.default_rng(1).integers(0, A.m, 2000)
-    yr, S = spmv.csr_spmv_rows(A.row_ptr, A.col, A.vals, x, rows)
-    ok, _ = spmv.within_tolerance(y[rows], yr, S, 1e-12)
-    assert ok.all()
+    _check_y(A, x, y, np.float64, chunk_rows=2_000_000)

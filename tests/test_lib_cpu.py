@@ -9,7 +9,7 @@ import numpy as np
 import pytest
 
 from gen import Csr, laplacian_2d, make_config, random_csr, random_block, row_block
-from oracle import bar, bro_coo, bro_ell, hyb, spmv
+from oracle import bar, bro_coo, bro_ell, hyb, metrics, spmv
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 HOST = -1
@@ -33,8 +33,8 @@ def test_exports_every_header_symbol(lib):
     assert lib.bro_version() == 1
 
 
-def _ell_parts(lib, A, V=4, dtype=np.float64):
-    o = lib.bro_opts_default(vec_words=V)
+def _ell_parts(lib, A, V=4, dtype=np.float64, h=32):
+    o = lib.bro_opts_default(vec_words=V, slice_h=h)
     h = lib.bro_create_ell(HOST, A.m, A.n, A.row_ptr, A.col, A.vals.astype(dtype), o)
     try:
         return {p: lib.bro_export_encoded(h, p, dtype) for p in
@@ -51,15 +51,17 @@ def _assert_ell_equal(parts, E):
     assert np.array_equal(parts["ell_vals"], E.vals)
 
 
-@pytest.mark.parametrize("V", [1, 2, 4])
+@pytest.mark.parametrize("h", [32, 64])
+@pytest.mark.parametrize("V", [1, 4])
 @pytest.mark.parametrize("seed", range(4))
-def test_bro_ell_bytes_match_oracle_random(lib, V, seed):
+def test_bro_ell_bytes_match_oracle_random(lib, h, V, seed):
     A = random_csr(150 + 37 * seed, 4000 if seed % 2 else 300, seed, max_len=45, empty_frac=0.15,
                    wide_cols=seed >= 2)
-    parts, info = _ell_parts(lib, A, V)
-    E = bro_ell.encode(A.row_ptr, A.col, A.vals, A.m, A.n, V=V)
-    _assert_ell_equal(parts, E)
-    assert info["ell_stream_bytes"] == E.stream_bytes()
+    for dt in (np.float64, np.float32):
+        parts, info = _ell_parts(lib, A, V, dt, h)
+        E = bro_ell.encode(A.row_ptr, A.col, A.vals.astype(dt), A.m, A.n, h=h, V=V)
+        _assert_ell_equal(parts, E)
+        assert info["ell_stream_bytes"] == E.stream_bytes() and info["slice_h"] == h
 
 
 def test_bro_ell_bytes_extreme_columns(lib):
@@ -71,9 +73,10 @@ def test_bro_ell_bytes_extreme_columns(lib):
     col = np.array([c for r in rows for c in r], dtype=np.int64)
     A = Csr(len(rows), n, rp, col, np.arange(col.size, dtype=np.float64), "extreme")
     for dt in (np.float64, np.float32):
-        parts, _ = _ell_parts(lib, A, 4, dt)
-        E = bro_ell.encode(A.row_ptr, A.col, A.vals.astype(dt), A.m, A.n, V=4)
-        _assert_ell_equal(parts, E)
+        for h in (32, 64):
+            parts, _ = _ell_parts(lib, A, 4, dt, h)
+            E = bro_ell.encode(A.row_ptr, A.col, A.vals.astype(dt), A.m, A.n, h=h, V=4)
+            _assert_ell_equal(parts, E)
 
 
 def test_bro_ell_c1_closed_form(lib):
@@ -84,10 +87,11 @@ def test_bro_ell_c1_closed_form(lib):
     _assert_ell_equal(parts, bro_ell.encode(A.row_ptr, A.col, A.vals, A.m, A.n))
 
 
-def test_bro_ell_c2_full_fp32(lib):
+@pytest.mark.parametrize("h", [32, 64])
+def test_bro_ell_c2_full_fp32(lib, h):
     A = make_config(2, np.float32)
-    parts, info = _ell_parts(lib, A, 4, np.float32)
-    E = bro_ell.encode(A.row_ptr, A.col, A.vals, A.m, A.n, V=4)
+    parts, info = _ell_parts(lib, A, 4, np.float32, h)
+    E = bro_ell.encode(A.row_ptr, A.col, A.vals, A.m, A.n, h=h, V=4)
     _assert_ell_equal(parts, E)
     assert 0.8 < info["eta_stream"] < 0.95  # cant-like savings (Table 3: 85.9%)
 
@@ -97,21 +101,47 @@ def _coo_of(A):
     return rows.astype(np.int32), cols.astype(np.int32), vals
 
 
-@pytest.mark.parametrize("V", [1, 4])
-def test_bro_coo_bytes_match_oracle(lib, V):
-    A = random_csr(500, 700, 11, max_len=60, empty_frac=0.4, long_frac=0.03, long_len=600)
-    r, c, v = _coo_of(A)
-    h = lib.bro_create_coo(HOST, A.m, A.n, r, c, v, lib.bro_opts_default(vec_words=V))
-    try:
-        C = bro_coo.encode(r, c, v, T=32, V=V)
+def _coo_parts_equal(lib, h, C, r, c, v, codec=1):
+    if codec:
         assert np.array_equal(lib.bro_export_encoded(h, "coo_words"), C.words)
         assert np.array_equal(lib.bro_export_encoded(h, "coo_base_row"), C.base_row)
         assert np.array_equal(lib.bro_export_encoded(h, "coo_width"), C.width)
         assert np.array_equal(lib.bro_export_encoded(h, "coo_symptr"), C.symptr)
-        assert np.array_equal(lib.bro_export_encoded(h, "coo_col"), c)
-        assert np.array_equal(lib.bro_export_encoded(h, "coo_vals", np.float64), v)
-    finally:
-        lib.bro_destroy(h)
+    else:
+        assert np.array_equal(lib.bro_export_encoded(h, "coo_row"), bro_coo.plain_rows(r, C.T))
+    assert np.array_equal(lib.bro_export_encoded(h, "coo_col"), C.col)
+    assert np.array_equal(lib.bro_export_encoded(h, "coo_vals", v.dtype), C.vals)
+
+
+@pytest.mark.parametrize("T", [8, 16, 32])
+@pytest.mark.parametrize("V", [1, 4])
+@pytest.mark.parametrize("codec", [1, 0])
+def test_bro_coo_bytes_match_oracle(lib, T, V, codec):
+    A = random_csr(500, 700, 11, max_len=60, empty_frac=0.4, long_frac=0.03, long_len=600)
+    r, c, v = _coo_of(A)
+    for dt in (np.float64, np.float32):
+        vv = v.astype(dt)
+        h = lib.bro_create_coo(HOST, A.m, A.n, r, c, vv, lib.bro_opts_default(vec_words=V, coo_T=T, codec=codec))
+        try:
+            info = lib.bro_get_info(h)
+            assert info["coo_T"] == T and info["n_intervals"] == -(-A.nnz // (32 * T))
+            C = bro_coo.encode(r, c, vv, T=T, V=V)
+            _coo_parts_equal(lib, h, C, r, c, vv, codec)
+        finally:
+            lib.bro_destroy(h)
+
+
+def test_coo_auto_T():
+    """coo_T = 0: 32 from 32*32*4736 COO entries, 16 from 16*32*4736, else 8."""
+    import paper_conf_sc_tangtrwckgtw13_b200 as P
+    for nnz, want in ((100, 8), (16 * 32 * 4736 - 1, 8), (16 * 32 * 4736, 16), (32 * 32 * 4736, 32)):
+        rows = np.zeros(nnz, np.int32)
+        cols = np.arange(nnz, dtype=np.int32)
+        h = P.bro_create_coo(HOST, 1, nnz, rows, cols, np.zeros(nnz, np.float32))
+        try:
+            assert P.bro_get_info(h)["coo_T"] == want
+        finally:
+            P.bro_destroy(h)
 
 
 def test_hyb_split_and_parts_match_oracle_c3(lib):
@@ -125,21 +155,35 @@ def test_hyb_split_and_parts_match_oracle_c3(lib):
         assert info["nnz_ell"] == ec.size and info["nnz_coo"] == cc.size
         assert 0.6 < ec.size / A.nnz < 0.7  # webbase-1M: 64.2% in BRO-ELL (Table 4)
         assert info["vec_words"] == 1  # auto layout for fp64: the paper's multiplexing
-        E = bro_ell.encode(ep, ec, ev, A.m, A.n, V=1, slices=[0, 1, 777, 31250])
+        H, T = info["slice_h"], info["coo_T"]
+        assert H == 64 and T == 8  # auto: 1M rows >= 303,104; 1.1M COO entries < 16*32*4736
+        sample = [0, 1, 777, 15624]
+        E = bro_ell.encode(ep, ec, ev, A.m, A.n, h=H, V=1, slices=sample)
         words = lib.bro_export_encoded(h, "ell_words")
         assert np.array_equal(lib.bro_export_encoded(h, "ell_colptr"), E.colptr)
         assert np.array_equal(lib.bro_export_encoded(h, "ell_symptr"), E.symptr)
         assert np.array_equal(lib.bro_export_encoded(h, "ell_bit_alloc"), E.bit_alloc)
-        for t in (0, 1, 777, 31250):
-            a, b = 32 * int(E.symptr[t]), 32 * int(E.symptr[t + 1])
+        for t in sample:
+            a, b = H * int(E.symptr[t]), H * int(E.symptr[t + 1])
             assert np.array_equal(words[a:b], E.words[a:b])
-        # COO part: sampled intervals through the oracle encoder
-        C = bro_coo.encode(cr[:32 * 1024 * 3], cc[:32 * 1024 * 3], cv[:32 * 1024 * 3], V=1)
+        # COO part: the first intervals through the oracle encoder
+        I = 32 * T
+        n3 = 3 * I
+        C = bro_coo.encode(cr[:n3], cc[:n3], cv[:n3], T=T, V=1)
         cw = lib.bro_export_encoded(h, "coo_words")
         sp = lib.bro_export_encoded(h, "coo_symptr")
         assert np.array_equal(sp[:C.symptr.size], C.symptr)
         assert np.array_equal(cw[:C.words.size], C.words)
         assert np.array_equal(lib.bro_export_encoded(h, "coo_width")[:C.width.size], C.width)
+        assert np.array_equal(lib.bro_export_encoded(h, "coo_col")[:n3], C.col)
+        assert np.array_equal(lib.bro_export_encoded(h, "coo_vals", np.float64)[:n3], C.vals)
+        # HYB space savings (Table 4 analog) from the oracle's own
+        # shapes and metrics (reading R19)
+        _, S, _ = bro_ell.slice_shapes(ep, ec, A.m, H, 32)
+        _, _, Sc = bro_coo.interval_shapes(cr, T)
+        Cb = metrics.bro_hyb_stream_bytes(4 * H * int(S.sum()), 4 * 32 * int(Sc.sum()), cr.size)
+        assert info["eta_stream"] == pytest.approx(metrics.eta(Cb, metrics.hyb_index_bytes(A.m, K, cr.size)),
+                                                   rel=0, abs=1e-12)
     finally:
         lib.bro_destroy(h)
 
@@ -161,31 +205,95 @@ def test_plain_ell_layout_matches_oracle(lib):
         lib.bro_destroy(h)
 
 
-def test_c5_sampled_slices_match_oracle(lib):
+@pytest.mark.parametrize("H", [32, 64])
+def test_c5_sampled_slices_match_oracle(lib, H):
     """Full-size C5 (8M rows, 213.8M nnz): C++ encoder vs oracle on sampled
-    slices, and the closed-form nnz 598^3."""
+    slices, the closed-form nnz 598^3, and at h = 32 the survey's regression
+    eta_stream (0.8378, tests/golden/survey_c5_layout.json)."""
     A = make_config(5)
     assert A.nnz == 598**3
-    h = lib.bro_create_ell(HOST, A.m, A.n, A.row_ptr, A.col, A.vals)
+    h = lib.bro_create_ell(HOST, A.m, A.n, A.row_ptr, A.col, A.vals, lib.bro_opts_default(slice_h=H))
     try:
         info = lib.bro_get_info(h)
-        assert info["nnz"] == 598**3 and info["n_slices"] == 250000
-        sample = [0, 1, 6249, 6250, 124999, 187500, 249999]
-        sub = row_block(A, 0, A.m)
+        s = A.m // H
+        assert info["nnz"] == 598**3 and info["n_slices"] == s
+        sample = [0, 1, s // 40 - 1, s // 40, s // 2 - 1, 3 * s // 4, s - 1]
         assert info["vec_words"] == 1
-        E = bro_ell.encode(sub.row_ptr, sub.col, sub.vals, A.m, A.n, V=1, slices=sample)
+        E = bro_ell.encode(A.row_ptr, A.col, A.vals, A.m, A.n, h=H, V=1, slices=sample)
         assert np.array_equal(lib.bro_export_encoded(h, "ell_colptr"), E.colptr)
         assert np.array_equal(lib.bro_export_encoded(h, "ell_symptr"), E.symptr)
         words = lib.bro_export_encoded(h, "ell_words")
         vals = lib.bro_export_encoded(h, "ell_vals", np.float64)
         for t in sample:
-            a, b = 32 * int(E.symptr[t]), 32 * int(E.symptr[t + 1])
+            a, b = H * int(E.symptr[t]), H * int(E.symptr[t + 1])
             assert np.array_equal(words[a:b], E.words[a:b])
-            a, b = 32 * int(E.colptr[t]), 32 * int(E.colptr[t + 1])
+            a, b = H * int(E.colptr[t]), H * int(E.colptr[t + 1])
             assert np.array_equal(vals[a:b], E.vals[a:b])
-        assert 0.8 < info["eta_stream"] < 0.87
+        if H == 32:
+            assert round(info["eta_stream"], 4) == 0.8378
+        else:
+            assert 0.8 < info["eta_stream"] < 0.8378
     finally:
         lib.bro_destroy(h)
+
+
+@pytest.mark.slow
+def test_c4_encoding_bytes_sampled_every_S(lib):
+    """C4 (2M rows, BAR method 0, BRO-HYB): the C++ encoder's bytes against
+    the oracle encoder on >= 1% of the ELL slices, chosen to cover every
+    symbols-per-row value S that occurs, plus the COO part's first and last
+    intervals (C4's encoding was never byte-compared)."""
+    from gen import permute_rows
+    A0 = make_config(4)
+    A = permute_rows(A0, lib.bro_reorder_bar(A0.m, A0.n, A0.row_ptr, A0.col, method=0))
+    for dt, V in ((np.float64, 1), (np.float32, 4)):
+        vals = A.vals.astype(dt)
+        h = lib.bro_create_hyb(HOST, A.m, A.n, A.row_ptr, A.col, vals, lib.bro_opts_default(vec_words=V))
+        try:
+            info = lib.bro_get_info(h)
+            H, T, K = info["slice_h"], info["coo_T"], info["K"]
+            ep, ec, ev, cr, cc, cv = hyb.hyb_split(A.row_ptr, A.col, vals, K)
+            sym = lib.bro_export_encoded(h, "ell_symptr").astype(np.int64)
+            S = np.diff(sym)
+            rng = np.random.default_rng(4)
+            sample = set(rng.choice(S.size, S.size // 100, replace=False).tolist())
+            for sv in np.unique(S):       # every S value, first and last occurrence
+                idx = np.nonzero(S == sv)[0]
+                sample.update([int(idx[0]), int(idx[-1])])
+            sample = sorted(sample)
+            assert len(sample) >= S.size // 100
+            E = bro_ell.encode(ep, ec, ev, A.m, A.n, h=H, V=V, slices=sample)
+            assert np.array_equal(S, E.S)
+            assert np.array_equal(lib.bro_export_encoded(h, "ell_bit_alloc"), E.bit_alloc)
+            assert np.array_equal(lib.bro_export_encoded(h, "ell_colptr"), E.colptr)
+            words = lib.bro_export_encoded(h, "ell_words")
+            ev_lib = lib.bro_export_encoded(h, "ell_vals", dt)
+            for t in sample:
+                a, b = H * int(E.symptr[t]), H * int(E.symptr[t + 1])
+                assert np.array_equal(words[a:b], E.words[a:b]), t
+                a, b = H * int(E.colptr[t]), H * int(E.colptr[t + 1])
+                assert np.array_equal(ev_lib[a:b], E.vals[a:b]), t
+            # COO part: first two and last interval (prefix / suffix encodes)
+            I = 32 * T
+            nI = info["n_intervals"]
+            C = bro_coo.encode(cr[:2 * I], cc[:2 * I], cv[:2 * I], T=T, V=V)
+            cw = lib.bro_export_encoded(h, "coo_words")
+            assert np.array_equal(cw[:C.words.size], C.words)
+            assert np.array_equal(lib.bro_export_encoded(h, "coo_vals", dt)[:2 * I], C.vals)
+            e0 = (nI - 1) * I
+            Cl = bro_coo.encode(cr[e0:], cc[e0:], cv[e0:], T=T, V=V)
+            sp = lib.bro_export_encoded(h, "coo_symptr").astype(np.int64)
+            assert np.array_equal(cw[32 * sp[nI - 1]:], Cl.words)
+            assert np.array_equal(lib.bro_export_encoded(h, "coo_col")[e0:], Cl.col)
+            assert int(lib.bro_export_encoded(h, "coo_base_row")[-1]) == int(Cl.base_row[0])
+            # HYB eta (Table 4 analog) recomputed from the oracle's shapes
+            _, Ss, _ = bro_ell.slice_shapes(ep, ec, A.m, H, 32)
+            _, _, Sc = bro_coo.interval_shapes(cr, T)
+            Cb = metrics.bro_hyb_stream_bytes(4 * H * int(Ss.sum()), 4 * 32 * int(Sc.sum()), cr.size)
+            assert info["eta_stream"] == pytest.approx(
+                metrics.eta(Cb, metrics.hyb_index_bytes(A.m, K, cr.size)), rel=0, abs=1e-12)
+        finally:
+            lib.bro_destroy(h)
 
 
 # ---------------------------------------------------------------- validation
@@ -210,9 +318,17 @@ def test_validation_errors(lib):
             lib.bro_create_ell(HOST, 2, n, rpx, cx, v)
         assert want in str(ei.value), (rpx, cx, n, str(ei.value))
     with pytest.raises(lib.BroError, match="UNSUPPORTED"):
-        lib.bro_create_ell(HOST, 2, 3, rp, good_c, v, lib.bro_opts_default(slice_h=64))
+        lib.bro_create_ell(HOST, 2, 3, rp, good_c, v, lib.bro_opts_default(slice_h=48))
+    with pytest.raises(lib.BroError, match="UNSUPPORTED"):
+        lib.bro_create_ell(HOST, 2, 3, rp, good_c, v, lib.bro_opts_default(coo_T=12))
+    for V in (2, 3):
+        with pytest.raises(lib.BroError, match="ARG"):
+            lib.bro_create_ell(HOST, 2, 3, rp, good_c, v, lib.bro_opts_default(vec_words=V))
+    with pytest.raises(lib.BroError, match="ARG"):  # tiny instance: every slice <= 4 columns
+        A = random_csr(64, 64, 0, max_len=9)
+        lib.bro_create_ell(HOST, A.m, A.n, A.row_ptr, A.col, A.vals, lib.bro_opts_default(ell_kernel=1))
     with pytest.raises(lib.BroError, match="ARG"):
-        lib.bro_create_ell(HOST, 2, 3, rp, good_c, v, lib.bro_opts_default(vec_words=3))
+        lib.bro_create_ell(HOST, 2, 3, rp, good_c, v, lib.bro_opts_default(ell_kernel=6))
     with pytest.raises(lib.BroError, match="INDEX"):   # COO not sorted by row
         lib.bro_create_coo(HOST, 2, 3, np.array([1, 0]), np.array([0, 0]), np.ones(2))
 
@@ -247,6 +363,27 @@ def test_bar_signature_order_matches_oracle(lib):
     perm = lib.bro_reorder_bar(A.m, A.n, A.row_ptr, A.col, method=0)
     assert np.array_equal(np.sort(perm), np.arange(A.m))
     assert np.array_equal(perm, bar.signature_order(A.row_ptr, A.col, A.m))
+
+
+def test_instance_choice(lib):
+    """Kernel instance resolved at create (bro_info_t.ell_kernel): tiny for
+    slices <= 4 columns, few-slice for short h = 32 matrices, else small /
+    mid / general window by the longest row stream (its symbol count from
+    the oracle's slice shapes); forced instances are honoured."""
+    def auto(A, h):
+        _, S, _ = bro_ell.slice_shapes(A.row_ptr, A.col, A.m, h, 32)
+        return 3 if S.max() < 10 else 4 if S.max() < 18 else 5
+    short, mid, long_ = (random_csr(5000, 5000, 1, max_len=k) for k in (4, 12, 90))
+    cases = [(short, {}, 1), (mid, {}, 2), (long_, {}, 2),
+             (mid, {"slice_h": 64}, auto(mid, 64)), (long_, {"slice_h": 64}, auto(long_, 64)),
+             (long_, {"slice_h": 64, "ell_kernel": 5}, 5), (mid, {"ell_kernel": 5}, 5)]
+    assert auto(mid, 64) == 3 and auto(long_, 64) > 3
+    for A, kw, want in cases:
+        h = lib.bro_create_ell(HOST, A.m, A.n, A.row_ptr, A.col, A.vals, lib.bro_opts_default(**kw))
+        try:
+            assert lib.bro_get_info(h)["ell_kernel"] == want, (kw, want)
+        finally:
+            lib.bro_destroy(h)
 
 
 @pytest.mark.parametrize("seed", [0, 1])
@@ -290,16 +427,15 @@ def test_dense_band_eta_closed_form(lib):
 
 
 @pytest.mark.parametrize("seed,m", [(3, None), (4, 300)])
-def test_bar_window_matches_oracle(lib, seed, m, monkeypatch):
+def test_bar_window_matches_oracle(lib, seed, m):
     """Method 2 (Algorithm 2 with a candidate window, reading R24; window
-    forced to 8 through the library's tuning variable) == the oracle's
+    forced to 8 through bro_reorder_bar's window argument) == the oracle's
     transcription with window=8; 10 partitions, so the window excludes some
     (and h does not divide m in the second case)."""
-    monkeypatch.setenv("BRO_BAR_WINDOW", "8")
     A = random_block(seed=seed, families=10, fam_rows=32)
     if m is not None:
         A = row_block(A, 0, m)
-    perm = lib.bro_reorder_bar(A.m, A.n, A.row_ptr, A.col, method=2)
+    perm = lib.bro_reorder_bar(A.m, A.n, A.row_ptr, A.col, method=2, window=8)
     assert np.array_equal(perm, bar.algorithm2(A.row_ptr, A.col, A.m, h=32, window=8))
 
 
