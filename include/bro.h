@@ -51,7 +51,8 @@
  *     delta of the first entry 0, base_row[i] = row of the first entry, one
  *     width width[i] per interval; lane l's T fields, MSB first,
  *     padded to S_i = ceil(T*width/32) symbols at
- *     coo_words[32*coo_symptr[i] + place(l,q,S_i,V)] (h = 32).
+ *     coo_words[32*coo_symptr[i] + 32*q + l] (the paper's V = 1 multiplexing,
+ *     whatever opts.vec_words says).
  *     col / vals (and plain COO rows) are stored per interval in the same
  *     lane-contiguous order in 16-byte chunks (reading R26): entry (l, t) at
  *     [i*32*T + place(l,t,T,C)], C = 4 for int32, 16/sizeof(val) for values;
@@ -117,7 +118,8 @@ typedef struct {
                         matrix shape; 1 tiny (every slice <= 4 columns), 2 few-slice
                         (h = 32), 3 small window (every row stream < 10 symbols), 4 mid
                         window (< 18), 5 general.  An instance the matrix does not fit
-                        gives BRO_ERR_ARG.  For A/B measurements and tests. */
+                        gives BRO_ERR_ARG.  For A/B measurements and tests (6..10: A/B
+                        candidates of the small / mid window instances). */
 } bro_opts_t;
 
 typedef struct {

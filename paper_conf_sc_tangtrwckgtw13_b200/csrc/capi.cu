@@ -156,7 +156,8 @@ bro_status_t check_opts(const bro_opts_t& o) {
   if (o.codec != 0 && o.codec != 1) return fail(BRO_ERR_ARG, "codec must be 0 or 1");
   if (o.hyb_K < -1) return fail(BRO_ERR_ARG, "hyb_K must be >= -1");
   if (o.min_bits < 0 || o.min_bits > 31) return fail(BRO_ERR_ARG, "min_bits must be in [0, 31]");
-  if (o.ell_kernel < 0 || o.ell_kernel > bro::ELL_GEN) return fail(BRO_ERR_ARG, "ell_kernel must be in [0, 5]");
+  if (o.ell_kernel < 0 || o.ell_kernel > bro::ELL_LAST)
+    return fail(BRO_ERR_ARG, "ell_kernel must be in [0, " + std::to_string(bro::ELL_LAST) + "]");
   return BRO_OK;
 }
 
@@ -230,6 +231,8 @@ bro_status_t choose_ell_instance(bro_matrix_s* A, int sms) {
   const bool tiny_ok = A->ell_max_l <= kEllTinyCols;
   const bool small_ok = A->ell_max_S < kEllRowsSmall;
   const bool mid_ok = A->ell_max_S < kEllRowsMid;
+  const bool small_family = want == ELL_SMALL || (want >= ELL_X_SMALL_L1 && want <= ELL_X_SMALL_PF1_L1);
+  const bool mid_family = want == ELL_MID || want == ELL_X_MID_PF1;
   if (want == ELL_AUTO) {
     if (tiny_ok) A->ell_inst = ELL_TINY;
     else if (A->h == 32 && A->s < int64_t(sms) * 32) A->ell_inst = ELL_FEW;
@@ -238,7 +241,7 @@ bro_status_t choose_ell_instance(bro_matrix_s* A, int sms) {
     else A->ell_inst = ELL_GEN;
     return BRO_OK;
   }
-  if ((want == ELL_TINY && !tiny_ok) || (want == ELL_SMALL && !small_ok) || (want == ELL_MID && !mid_ok))
+  if ((want == ELL_TINY && !tiny_ok) || (small_family && !small_ok) || (mid_family && !mid_ok))
     return fail(BRO_ERR_ARG, "ell_kernel " + std::to_string(want) + " does not fit this matrix (longest slice " +
                                  std::to_string(A->ell_max_l) + " columns, longest row stream " +
                                  std::to_string(A->ell_max_S) + " symbols)");
@@ -275,8 +278,8 @@ bro_status_t resolve_kernels(bro_matrix_s* A) {
     }
   }
   if (A->has_coo && !st) {
-    st = resolve(A->coo_k[0], bro::coo_ref<T>(V, A->opts.codec == 1, A->coo_T, 0), sms, "COO");
-    if (!st) st = resolve(A->coo_k[2], bro::coo_ref<T>(V, A->opts.codec == 1, A->coo_T, 2), sms, "COO decode");
+    st = resolve(A->coo_k[0], bro::coo_ref<T>(A->opts.codec == 1, A->coo_T, 0), sms, "COO");
+    if (!st) st = resolve(A->coo_k[2], bro::coo_ref<T>(A->opts.codec == 1, A->coo_T, 2), sms, "COO decode");
     if (!st) st = resolve(A->fix_k, bro::fixup_ref<T>(), sms, "COO fix-up");
   }
   if (!st) st = resolve(A->rep_k, bro::replicate_ref<T>(), sms, "replicate");
@@ -342,7 +345,9 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
         }
       }
       if (o.codec)
-        bro::encode_bro_coo(A->nnz_coo, cr.data(), cc.data(), cv.data(), A->vsize, A->coo_T, o.vec_words, A->coo);
+        // COO lane streams always use the paper's V = 1 multiplexing (a lane's
+        // word q at 32q + lane: one coalesced 128-byte row per q, staged by cp.async)
+        bro::encode_bro_coo(A->nnz_coo, cr.data(), cc.data(), cv.data(), A->vsize, A->coo_T, 1, A->coo);
       else
         bro::build_plain_coo(A->nnz_coo, cr.data(), cc.data(), cv.data(), A->vsize, A->coo_T, A->coo);
       A->nI = A->coo.nI;
@@ -487,7 +492,9 @@ cudaError_t launch_ell(const bro_matrix_s* A, int mode, const T* x, const bro::d
                           static_cast<const T*>(A->d_ell_vals), x};
     return launch(L, persistent_grid(L, p.s), st, p, y, dec);
   }
-  bro::dev::PellDev<T> p{r1 - r0, A->K, A->pitch, A->d_pell_col + r0, static_cast<const T*>(A->d_ell_vals) + r0, x};
+  // decode mode covers the padding rows [m, pitch) too (they hold -1)
+  const int64_t rows = mode == 2 && b0 == 0 ? A->pitch : r1 - r0;
+  bro::dev::PellDev<T> p{rows, A->K, A->pitch, A->d_pell_col + r0, static_cast<const T*>(A->d_ell_vals) + r0, x};
   return launch(L, (p.m + L.k.threads - 1) / L.k.threads, st, p, y, dec);
 }
 

@@ -20,35 +20,32 @@ static KernelRef plain_ell_impl(int mode) {
   return {};
 }
 
-template <typename T, int V, bool kBro, int TT>
+template <typename T, bool kBro, int TT>
 static KernelRef coo_pick(int mode) {
   using namespace dev;
-  if (mode == 2) return {(const void*)&coo_spmv<T, V, kBro, TT, kCooWarps, kCooMinBlocks, kDecode>, 32 * kCooWarps};
-  return {(const void*)&coo_spmv<T, V, kBro, TT, kCooWarps, kCooMinBlocks, kSpmv>, 32 * kCooWarps};
+  if (mode == 2) return {(const void*)&coo_spmv<T, kBro, TT, kCooWarps, kCooMinBlocks, kDecode>, 32 * kCooWarps};
+  return {(const void*)&coo_spmv<T, kBro, TT, kCooWarps, kCooMinBlocks, kSpmv>, 32 * kCooWarps};
 }
 
-template <typename T, int V, bool kBro>
+template <typename T, bool kBro>
 static KernelRef coo_pick_t(int TT, int mode) {
   switch (TT) {
-    case 8: return coo_pick<T, V, kBro, 8>(mode);
-    case 16: return coo_pick<T, V, kBro, 16>(mode);
-    case 32: return coo_pick<T, V, kBro, 32>(mode);
+    case 8: return coo_pick<T, kBro, 8>(mode);
+    case 16: return coo_pick<T, kBro, 16>(mode);
+    case 32: return coo_pick<T, kBro, 32>(mode);
   }
   return {};
 }
 
 template <typename T>
-static KernelRef coo_impl(int V, bool bro, int TT, int mode) {
-  if (!bro) return coo_pick_t<T, 4, false>(TT, mode);
-  if (V == 1) return coo_pick_t<T, 1, true>(TT, mode);
-  if (V == 4) return coo_pick_t<T, 4, true>(TT, mode);
-  return {};
+static KernelRef coo_impl(bool bro, int TT, int mode) {
+  return bro ? coo_pick_t<T, true>(TT, mode) : coo_pick_t<T, false>(TT, mode);
 }
 
 template <> KernelRef plain_ell_ref<double>(int mode) { return plain_ell_impl<double>(mode); }
 template <> KernelRef plain_ell_ref<float>(int mode) { return plain_ell_impl<float>(mode); }
-template <> KernelRef coo_ref<double>(int V, bool bro, int TT, int mode) { return coo_impl<double>(V, bro, TT, mode); }
-template <> KernelRef coo_ref<float>(int V, bool bro, int TT, int mode) { return coo_impl<float>(V, bro, TT, mode); }
+template <> KernelRef coo_ref<double>(bool bro, int TT, int mode) { return coo_impl<double>(bro, TT, mode); }
+template <> KernelRef coo_ref<float>(bool bro, int TT, int mode) { return coo_impl<float>(bro, TT, mode); }
 template <> KernelRef fixup_ref<double>() { return {(const void*)&dev::coo_fixup<double>, 256}; }
 template <> KernelRef fixup_ref<float>() { return {(const void*)&dev::coo_fixup<float>, 256}; }
 template <> KernelRef replicate_ref<double>() { return {(const void*)&dev::replicate_y<double>, 256}; }

@@ -230,7 +230,9 @@ __device__ __forceinline__ void load_vals(T* v, const T* vs, int j, int l, int l
 
 // Copy symbol rows [qa, qa + nrows) of this lane's R rows into
 // win[((q - qa) * 32 + lane) * R + k] (zeros past S) plus one zero guard row.
-template <int V, int R>
+// kL1: symbol words through the L1-allocating read-only path (__ldg) instead
+// of the no-allocate streaming load (V = 1 only).
+template <int V, int R, bool kL1 = false>
 __device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __restrict__ wb, int S, int qa,
                                               int nrows, int lane) {
   constexpr int H = 32 * R;
@@ -239,7 +241,8 @@ __device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __r
       const int q = qa + r;
       uint32_t w[R];
 #pragma unroll
-      for (int k = 0; k < R; ++k) w[k] = q < S ? ld_stream_u32(wb + H * q + 32 * k + lane) : 0u;
+      for (int k = 0; k < R; ++k)
+        w[k] = q < S ? (kL1 ? __ldg(wb + H * q + 32 * k + lane) : ld_stream_u32(wb + H * q + 32 * k + lane)) : 0u;
       if constexpr (R == 1) win[r * 32 + lane] = w[0];
       else reinterpret_cast<uint2*>(win)[r * 32 + lane] = make_uint2(w[0], w[1]);
     }
@@ -286,7 +289,18 @@ __device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __r
 // G columns per group; kRows window rows per warp (34 holds any 32-column
 // block: <= 33 symbol rows + a zero guard row; smaller windows for matrices
 // whose row streams are all shorter leave more of the SM's memory to L1).
-template <typename T, int V, int R, int kWarps, int kMinBlocks, int G, int kRows, int kMode>
+// L2 prefetch (TMA engine, no registers, no shared memory) of [p, p + bytes);
+// p and bytes multiples of 16.
+__device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" :: "l"(p), "r"(bytes) : "memory");
+}
+
+// kPf > 0: at the start of a slice, lane 0 asks the TMA engine to prefetch
+// into L2 the values, symbols and widths of the slice this warp handles kPf
+// slices later, so its own loads of that slice hit L2 instead of HBM.
+// kL1: symbol staging through the L1-allocating path.
+template <typename T, int V, int R, int kWarps, int kMinBlocks, int G, int kRows, int kMode, int kPf = 0,
+          bool kL1 = false>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   constexpr int H = 32 * R;
@@ -312,6 +326,17 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
       __syncwarp();
     }
     const Meta mt = metas[w][k32];
+    if constexpr (kPf > 0 && kMode != kDecode) {
+      if (lane == 0 && k32 + kPf < 32 && t + kPf * stride < p.s) {
+        const Meta nx = metas[w][k32 + kPf];
+        if (nx.l > 0) {
+          prefetch_l2(p.vals + H * nx.c0, uint32_t(H * nx.l * sizeof(T)));
+          prefetch_l2(p.words + H * nx.q0, uint32_t(H * nx.S * 4));
+          const uint64_t b0 = nx.c0 & ~uint64_t(15), b1 = (nx.c0 + uint64_t(nx.l) + 15) & ~uint64_t(15);
+          prefetch_l2(p.bit_alloc + b0, uint32_t(b1 - b0));
+        }
+      }
+    }
     const int l = mt.l;
     const int S = mt.S;
     const uint32_t* wb = p.words + H * mt.q0;
@@ -328,7 +353,7 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
       const int b = lane < nb ? int(__ldg(ba + jb + lane)) : 0;
       if (jb == 0) {  // first block starts at symbol 0: stage without waiting for the scan
         __syncwarp();
-        stage_symbols<V, R>(win, wb, S, 0, min(S, kRows - 1), lane);
+        stage_symbols<V, R, kL1>(win, wb, S, 0, min(S, kRows - 1), lane);
       }
       int incl = b;  // inclusive scan of the widths over the block
 #pragma unroll
@@ -341,7 +366,7 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
       const int nrows = tot > 0 ? ((obase + tot - 1) >> 5) - qa + 1 : 0;
       if (jb > 0) {
         __syncwarp();
-        stage_symbols<V, R>(win, wb, S, qa, nrows, lane);
+        stage_symbols<V, R, kL1>(win, wb, S, qa, nrows, lane);
       }
       {
         const int rel = b ? obase + incl - b - 32 * qa : 0;  // column jb+lane inside the window
@@ -588,7 +613,12 @@ __device__ __forceinline__ int coo_field(const uint32_t* wl, int t, int b) {
   return int(shr_clamp(__funnelshift_l(p[32], p[0], uint32_t(o & 31)), uint32_t(32 - b)));
 }
 
-template <typename T, int V, bool kBro, int TT, int kWarps, int kMinBlocks, int kMode>
+__device__ __forceinline__ void cp_async4(uint32_t* dst, const uint32_t* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
+               "l"(src) : "memory");
+}
+
+template <typename T, bool kBro, int TT, int kWarps, int kMinBlocks, int kMode>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   constexpr int I = 32 * TT;
@@ -605,37 +635,19 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   const T* vb = p.vals + e0;
   int b = 0;
   const uint32_t* wl = cwin[w] + lane;
-  int row = first;  // running row of this lane (BRO)
   if constexpr (kBro) {
+    // the lane streams' words (V = 1: word q of lane l at 32q + l) go to the
+    // [q][lane] window by cp.async, in flight together with the first batch's
+    // col / vals and x gathers below
     b = int(p.width[i]);
     if (b > 0) {  // b = 0: one row for the whole interval, empty stream
       const uint64_t q0 = p.symptr[i];
       const int S = int(p.symptr[i + 1] - q0);
-      const uint32_t* wb = p.words + 32 * q0;
-      uint32_t* win = cwin[w];
-      if constexpr (V == 1) {
-        for (int q = 0; q < S; ++q) win[32 * q + lane] = ld_stream_u32(wb + 32 * q + lane);
-      } else {
-        const int F = S >> 2, Vp = S - 4 * F;
-        for (int c = 0; c < F; ++c) {
-          const uint4 v = ld_stream_u4(wb + 128 * c + 4 * lane);
-          win[32 * (4 * c) + lane] = v.x; win[32 * (4 * c + 1) + lane] = v.y;
-          win[32 * (4 * c + 2) + lane] = v.z; win[32 * (4 * c + 3) + lane] = v.w;
-        }
-        for (int e = 0; e < Vp; ++e) win[32 * (4 * F + e) + lane] = ld_stream_u32(wb + 128 * F + Vp * lane + e);
-      }
-      win[32 * S + lane] = 0u;
-      __syncwarp();
-      int tot = 0;  // pass 1: sum of this lane's deltas
-#pragma unroll 8
-      for (int t = 0; t < TT; ++t) tot += coo_field(wl, t, b);
-      int incl = tot;
-#pragma unroll
-      for (int off = 1; off < 32; off <<= 1) {
-        const int o = __shfl_up_sync(0xffffffffu, incl, off);
-        if (lane >= off) incl += o;
-      }
-      row = first + incl - tot;  // row of the entry before this lane's first (its deltas follow)
+      const uint32_t* wb = p.words + 32 * q0 + lane;
+      uint32_t* win = cwin[w] + lane;
+      for (int q = 0; q < S; ++q) cp_async4(win + 32 * q, wb + 32 * q);
+      asm volatile("cp.async.commit_group;" ::: "memory");
+      win[32 * S] = 0u;
     }
   }
   // per-lane segment state: f = row of the lane's first entry, A = partial of
@@ -643,19 +655,37 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   int f = 0, cr = 0;
   T A = T(0), cur = T(0);
   bool one = true;
+  int row = first;  // running row of this lane (BRO)
 #pragma unroll
   for (int nb = 0; nb < NB; ++nb) {
     const int t0 = 8 * nb;
     int r[8], c[8];
-    T v[8];
+    T v[8], xv[8];
     if constexpr (kMode != kDecode) {
       load8_s32(c, cb, t0, lane);
       Vec8<T> vv;
       vv.load(vb, t0, lane);
 #pragma unroll
       for (int k = 0; k < 8; ++k) v[k] = vv.v[k];
+#pragma unroll
+      for (int k = 0; k < 8; ++k)  // slots past nnz hold col 0 / value 0: no gather
+        xv[k] = TT * lane + t0 + k < lim ? ldg_x(p.x + c[k]) : T(0);
     }
     if constexpr (kBro) {
+      if (nb == 0 && b > 0) {
+        asm volatile("cp.async.wait_group 0;" ::: "memory");
+        __syncwarp();
+        int tot = 0;  // pass 1: sum of this lane's deltas
+#pragma unroll 8
+        for (int t = 0; t < TT; ++t) tot += coo_field(wl, t, b);
+        int incl = tot;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+          const int o = __shfl_up_sync(0xffffffffu, incl, off);
+          if (lane >= off) incl += o;
+        }
+        row = first + incl - tot;  // row of the entry before this lane's first (its deltas follow)
+      }
 #pragma unroll
       for (int k = 0; k < 8; ++k) {
         if (b > 0) row += coo_field(wl, t0 + k, b);
@@ -669,25 +699,20 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
       for (int k = 0; k < 8; ++k)
         if (TT * lane + t0 + k < lim) dec[e0 + TT * lane + t0 + k] = r[k];
     } else {
-      T prod[8];
 #pragma unroll
       for (int k = 0; k < 8; ++k) {
-        const bool ok = TT * lane + t0 + k < lim;  // slots past nnz hold col 0 / value 0: skip the gather
-        prod[k] = ok ? v[k] * ldg_x(p.x + c[k]) : T(0);
-      }
-#pragma unroll
-      for (int k = 0; k < 8; ++k) {
+        const T prod = v[k] * xv[k];
         if (nb == 0 && k == 0) {
           f = r[0];
           cr = r[0];
-          cur = prod[0];
+          cur = prod;
         } else if (r[k] != cr) {  // the segment of row cr ends inside this lane
           if (one) { A = cur; one = false; }
           else atomicAdd(y + cr, cur);  // interior segment (row > first): complete, unique to this lane
           cr = r[k];
-          cur = prod[k];
+          cur = prod;
         } else {
-          cur += prod[k];
+          cur += prod;
         }
       }
     }

@@ -13,7 +13,10 @@ struct KernelRef {
 };
 
 // BRO-ELL kernel instances (bro_opts_t.ell_kernel; 0 = chosen at create)
-enum EllInst { ELL_AUTO = 0, ELL_TINY = 1, ELL_FEW = 2, ELL_SMALL = 3, ELL_MID = 4, ELL_GEN = 5 };
+enum EllInst { ELL_AUTO = 0, ELL_TINY = 1, ELL_FEW = 2, ELL_SMALL = 3, ELL_MID = 4, ELL_GEN = 5,
+               // A/B candidates (measured, then folded into the instances above or removed)
+               ELL_X_SMALL_L1 = 6, ELL_X_SMALL_PF1 = 7, ELL_X_SMALL_PF2 = 8, ELL_X_SMALL_PF1_L1 = 9,
+               ELL_X_MID_PF1 = 10, ELL_LAST = 10 };
 constexpr int kEllTinyCols = 4;   // TINY: every slice has <= 4 columns
 constexpr int kEllRowsSmall = 10; // SMALL: every row stream < 10 symbols
 constexpr int kEllRowsMid = 18;   // MID:   < 18 symbols
@@ -22,7 +25,7 @@ constexpr int kEllRowsGen = 34;   // GEN:   any
 // mode: 0 = y = A.x, 1 = scatter (y into every destination), 2 = decode
 template <typename T> KernelRef bro_ell_ref(int V, int R, int inst, int mode);
 template <typename T> KernelRef plain_ell_ref(int mode);
-template <typename T> KernelRef coo_ref(int V, bool bro, int TT, int mode);  // mode 0 or 2
+template <typename T> KernelRef coo_ref(bool bro, int TT, int mode);  // mode 0 or 2
 template <typename T> KernelRef fixup_ref();
 template <typename T> KernelRef replicate_ref();
 
