@@ -622,57 +622,70 @@ template <typename T, bool kBro, int TT, int kWarps, int kMinBlocks, int kMode>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   constexpr int I = 32 * TT;
-  constexpr int NB = TT / 8;
+  constexpr int CH = TT < 16 ? TT : 16;  // entries per lane loaded at once (one chunk)
+  constexpr int NC = TT / CH;
   __shared__ uint32_t cwin[kWarps][kBro ? (TT + 1) * 32 : 1];  // <= T symbol rows + a zero guard row
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
   const int64_t i = int64_t(blockIdx.x) * kWarps + w;
   if (i >= p.nI) return;
   const int64_t e0 = i * I;
-  const int lim = int(min(int64_t(I), p.nnz - e0));  // valid entries of the interval
-  const int first = int(p.base_row[i]);              // row of the interval's first entry
   const int32_t* cb = p.col + e0;
   const T* vb = p.vals + e0;
-  int b = 0;
-  const uint32_t* wl = cwin[w] + lane;
-  if constexpr (kBro) {
-    // the lane streams' words (V = 1: word q of lane l at 32q + l) go to the
-    // [q][lane] window by cp.async, in flight together with the first batch's
-    // col / vals and x gathers below
-    b = int(p.width[i]);
-    if (b > 0) {  // b = 0: one row for the whole interval, empty stream
-      const uint64_t q0 = p.symptr[i];
-      const int S = int(p.symptr[i + 1] - q0);
-      const uint32_t* wb = p.words + 32 * q0 + lane;
-      uint32_t* win = cwin[w] + lane;
-      for (int q = 0; q < S; ++q) cp_async4(win + 32 * q, wb + 32 * q);
-      asm volatile("cp.async.commit_group;" ::: "memory");
-      win[32 * S] = 0u;
-    }
-  }
   // per-lane segment state: f = row of the lane's first entry, A = partial of
   // its first segment, cr / cur = current (trailing) segment
   int f = 0, cr = 0;
   T A = T(0), cur = T(0);
   bool one = true;
-  int row = first;  // running row of this lane (BRO)
+  int b = 0, row = 0, first = 0, lim = 0;
+  const uint32_t* wl = cwin[w] + lane;
 #pragma unroll
-  for (int nb = 0; nb < NB; ++nb) {
-    const int t0 = 8 * nb;
-    int r[8], c[8];
-    T v[8], xv[8];
+  for (int ch = 0; ch < NC; ++ch) {
+    // the chunk's col / vals (and plain rows) first: nothing they need
+    // depends on the interval header, so their round trip overlaps the
+    // header -> word staging chain below
+    int r[CH], c[CH];
+    T v[CH];
     if constexpr (kMode != kDecode) {
-      load8_s32(c, cb, t0, lane);
-      Vec8<T> vv;
-      vv.load(vb, t0, lane);
 #pragma unroll
-      for (int k = 0; k < 8; ++k) v[k] = vv.v[k];
+      for (int u = 0; u < CH / 8; ++u) {
+        load8_s32(c + 8 * u, cb, CH * ch + 8 * u, lane);
+        Vec8<T> vv;
+        vv.load(vb, CH * ch + 8 * u, lane);
 #pragma unroll
-      for (int k = 0; k < 8; ++k)  // slots past nnz hold col 0 / value 0: no gather
-        xv[k] = TT * lane + t0 + k < lim ? ldg_x(p.x + c[k]) : T(0);
+        for (int k = 0; k < 8; ++k) v[8 * u + k] = vv.v[k];
+      }
+    }
+    if constexpr (!kBro) {
+#pragma unroll
+      for (int u = 0; u < CH / 8; ++u) load8_s32(r + 8 * u, p.rows + e0, CH * ch + 8 * u, lane);
+    }
+    if (ch == 0) {
+      lim = int(min(int64_t(I), p.nnz - e0));  // valid entries of the interval
+      first = int(p.base_row[i]);              // row of the interval's first entry
+      row = first;
+      if constexpr (kBro) {
+        // lane words (V = 1: word q of lane l at 32q + l) -> [q][lane] window
+        b = int(p.width[i]);
+        if (b > 0) {  // b = 0: one row for the whole interval, empty stream
+          const uint64_t q0 = p.symptr[i];
+          const int S = int(p.symptr[i + 1] - q0);
+          const uint32_t* wb = p.words + 32 * q0 + lane;
+          uint32_t* win = cwin[w] + lane;
+          for (int q = 0; q < S; ++q) cp_async4(win + 32 * q, wb + 32 * q);
+          asm volatile("cp.async.commit_group;" ::: "memory");
+          win[32 * S] = 0u;
+        }
+      }
+    }
+    T xv[CH];
+    if constexpr (kMode != kDecode) {
+#pragma unroll
+      for (int k = 0; k < CH; ++k)  // slots past nnz hold col 0 / value 0: no gather
+        xv[k] = TT * lane + CH * ch + k < lim ? ldg_x(p.x + c[k]) : T(0);
     }
     if constexpr (kBro) {
-      if (nb == 0 && b > 0) {
+      if (ch == 0 && b > 0) {
         asm volatile("cp.async.wait_group 0;" ::: "memory");
         __syncwarp();
         int tot = 0;  // pass 1: sum of this lane's deltas
@@ -687,22 +700,20 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
         row = first + incl - tot;  // row of the entry before this lane's first (its deltas follow)
       }
 #pragma unroll
-      for (int k = 0; k < 8; ++k) {
-        if (b > 0) row += coo_field(wl, t0 + k, b);
+      for (int k = 0; k < CH; ++k) {
+        if (b > 0) row += coo_field(wl, CH * ch + k, b);
         r[k] = row;
       }
-    } else {
-      load8_s32(r, p.rows + e0, t0, lane);
     }
     if constexpr (kMode == kDecode) {
 #pragma unroll
-      for (int k = 0; k < 8; ++k)
-        if (TT * lane + t0 + k < lim) dec[e0 + TT * lane + t0 + k] = r[k];
+      for (int k = 0; k < CH; ++k)
+        if (TT * lane + CH * ch + k < lim) dec[e0 + TT * lane + CH * ch + k] = r[k];
     } else {
 #pragma unroll
-      for (int k = 0; k < 8; ++k) {
+      for (int k = 0; k < CH; ++k) {
         const T prod = v[k] * xv[k];
-        if (nb == 0 && k == 0) {
+        if (ch == 0 && k == 0) {
           f = r[0];
           cr = r[0];
           cur = prod;

@@ -56,10 +56,16 @@ def main():
         peak = float(json.load(f)["hbm_gbs"])
     flush_buf = torch.empty(2 * bench.L2_BYTES // 4, dtype=torch.int32, device=dev)
 
+    clocks = []
+
     def timeit(M):
         small = M.info["algorithmic_bytes"] < 4 * bench.L2_BYTES
         fl = (lambda: flush_buf.fill_(1)) if small else None
+        ck = bench.ClockSampler(0)
+        ck.start()
         ms = bench.time_steps(lambda: M.spmv(x, y, stream), a.steps, a.warmup, stream, fl)
+        c = ck.stop() or {}
+        clocks.append(f"{c.get('sm_mhz')}MHz{'/' + ','.join(c['reasons']) if c.get('reasons') else ''}")
         return ms, M.info["algorithmic_bytes"]
 
     base = P.BroMatrix(A, fmt=fmt, codec=0, device=0, dtype=dtype, **parse_opts(a.baseline_opts))
@@ -67,7 +73,7 @@ def main():
     yb = y.clone()
     bmean = float(bms.mean())
     print(f"{a.workload} {a.dtype} {fmt}: baseline {bmean * 1e3:.1f} us "
-          f"{bbytes / (bmean * 1e-3) / 1e9:.0f} GB/s ({bbytes / 1e6:.1f} MB)", flush=True)
+          f"{bbytes / (bmean * 1e-3) / 1e9:.0f} GB/s ({bbytes / 1e6:.1f} MB) {clocks[-1]}", flush=True)
     base.close()
     for v in a.variants:
         M = P.BroMatrix(A, fmt=fmt, codec=1, device=0, dtype=dtype, **parse_opts(v))
@@ -78,7 +84,7 @@ def main():
         i = M.info
         print(f"  {v:40s} {mean * 1e3:8.1f} us (p50 {p50 * 1e3:7.1f})  {gbs:6.0f} GB/s  frac {gbs / peak:.3f}  "
               f"x{bmean / mean:.3f}  h={i['slice_h']} T={i['coo_T']} inst={i['ell_kernel']} "
-              f"eta={i['eta_stream']:.3f} MB={nb / 1e6:.1f} ok={bool(ok)}", flush=True)
+              f"eta={i['eta_stream']:.3f} MB={nb / 1e6:.1f} ok={bool(ok)} {clocks[-1]}", flush=True)
         M.close()
 
 
