@@ -637,7 +637,8 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   int f = 0, cr = 0;
   T A = T(0), cur = T(0);
   bool one = true;
-  int b = 0, row = 0, first = 0, lim = 0;
+  int b = 0, S = 0, row = 0, first = 0, lim = 0;
+  uint32_t w0 = 0, w1 = 0;
   const uint32_t* wl = cwin[w] + lane;
 #pragma unroll
   for (int ch = 0; ch < NC; ++ch) {
@@ -665,16 +666,22 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
       first = int(p.base_row[i]);              // row of the interval's first entry
       row = first;
       if constexpr (kBro) {
-        // lane words (V = 1: word q of lane l at 32q + l) -> [q][lane] window
         b = int(p.width[i]);
         if (b > 0) {  // b = 0: one row for the whole interval, empty stream
           const uint64_t q0 = p.symptr[i];
-          const int S = int(p.symptr[i + 1] - q0);
-          const uint32_t* wb = p.words + 32 * q0 + lane;
-          uint32_t* win = cwin[w] + lane;
-          for (int q = 0; q < S; ++q) cp_async4(win + 32 * q, wb + 32 * q);
-          asm volatile("cp.async.commit_group;" ::: "memory");
-          win[32 * S] = 0u;
+          S = int(p.symptr[i + 1] - q0);
+          const uint32_t* wb = p.words + 32 * q0 + lane;  // V = 1: word q of lane l at 32q + l
+          if (S <= 2) {
+            // short streams (T*b <= 64 bits; C3/C4 intervals have small row
+            // gaps): the lane's <= 2 words in registers, no window
+            w0 = ld_stream_u32(wb);
+            w1 = S > 1 ? ld_stream_u32(wb + 32) : 0u;
+          } else {  // the lane words -> [q][lane] window by cp.async
+            uint32_t* win = cwin[w] + lane;
+            for (int q = 0; q < S; ++q) cp_async4(win + 32 * q, wb + 32 * q);
+            asm volatile("cp.async.commit_group;" ::: "memory");
+            win[32 * S] = 0u;
+          }
         }
       }
     }
@@ -685,24 +692,49 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
         xv[k] = TT * lane + CH * ch + k < lim ? ldg_x(p.x + c[k]) : T(0);
     }
     if constexpr (kBro) {
-      if (ch == 0 && b > 0) {
-        asm volatile("cp.async.wait_group 0;" ::: "memory");
-        __syncwarp();
-        int tot = 0;  // pass 1: sum of this lane's deltas
-#pragma unroll 8
-        for (int t = 0; t < TT; ++t) tot += coo_field(wl, t, b);
-        int incl = tot;
+      if (b > 0 && S <= 2) {
+        // field t = bits [t*b, t*b + b) of the 64-bit stream w0:w1, MSB first
+        const uint64_t W = (uint64_t(w0) << 32) | w1;
+        int d[CH];
 #pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {
-          const int o = __shfl_up_sync(0xffffffffu, incl, off);
-          if (lane >= off) incl += o;
+        for (int k = 0; k < CH; ++k) d[k] = int((W << ((CH * ch + k) * b)) >> (64 - b));
+        if (ch == 0) {
+          int tot = 0;  // sum of this lane's deltas (all T fields)
+#pragma unroll
+          for (int t = 0; t < TT; ++t) tot += int((W << (t * b)) >> (64 - b));
+          int incl = tot;
+#pragma unroll
+          for (int off = 1; off < 32; off <<= 1) {
+            const int o = __shfl_up_sync(0xffffffffu, incl, off);
+            if (lane >= off) incl += o;
+          }
+          row = first + incl - tot;  // row of the entry before this lane's first
         }
-        row = first + incl - tot;  // row of the entry before this lane's first (its deltas follow)
-      }
 #pragma unroll
-      for (int k = 0; k < CH; ++k) {
-        if (b > 0) row += coo_field(wl, CH * ch + k, b);
-        r[k] = row;
+        for (int k = 0; k < CH; ++k) {
+          row += d[k];
+          r[k] = row;
+        }
+      } else {
+        if (ch == 0 && b > 0) {
+          asm volatile("cp.async.wait_group 0;" ::: "memory");
+          __syncwarp();
+          int tot = 0;  // pass 1: sum of this lane's deltas
+#pragma unroll 8
+          for (int t = 0; t < TT; ++t) tot += coo_field(wl, t, b);
+          int incl = tot;
+#pragma unroll
+          for (int off = 1; off < 32; off <<= 1) {
+            const int o = __shfl_up_sync(0xffffffffu, incl, off);
+            if (lane >= off) incl += o;
+          }
+          row = first + incl - tot;  // row of the entry before this lane's first (its deltas follow)
+        }
+#pragma unroll
+        for (int k = 0; k < CH; ++k) {
+          if (b > 0) row += coo_field(wl, CH * ch + k, b);
+          r[k] = row;
+        }
       }
     }
     if constexpr (kMode == kDecode) {

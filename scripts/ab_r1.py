@@ -19,8 +19,8 @@ def build_r1():
     lib = os.path.join(d, "libbro_r1.so")
     cmd = ["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-std=c++17", "-lineinfo", "-shared",
            "-Xcompiler", "-fPIC,-pthread,-O3", "-cudart", "static", "--expt-relaxed-constexpr",
-           "-I", os.path.join(d, "include"), "-o", lib, os.path.join(d, "csrc", "capi.cu"),
-           os.path.join(d, "csrc", "encode.cpp")]
+           "-I", os.path.join(d, "include"), "-o", lib, os.path.join(d, "a", "csrc", "capi.cu"),
+           os.path.join(d, "a", "csrc", "encode.cpp")]
     subprocess.run(cmd, check=True)
     return lib
 
