@@ -231,8 +231,9 @@ bro_status_t choose_ell_instance(bro_matrix_s* A, int sms) {
   const bool tiny_ok = A->ell_max_l <= kEllTinyCols;
   const bool small_ok = A->ell_max_S < kEllRowsSmall;
   const bool mid_ok = A->ell_max_S < kEllRowsMid;
-  const bool small_family = want == ELL_SMALL || (want >= ELL_X6 && want <= ELL_X10 && want != ELL_X9);
-  const bool mid_family = want == ELL_MID || want == ELL_X9;
+  const bool small_family = want == ELL_SMALL || want == ELL_X6 || want == ELL_X7 || want == ELL_X10 ||
+                            (A->h == 64 && want == ELL_X8);
+  const bool mid_family = want == ELL_MID || want == ELL_X9 || (A->h == 32 && want == ELL_X8);
   if (want == ELL_AUTO) {
     if (tiny_ok) A->ell_inst = ELL_TINY;
     else if (A->h == 32 && A->s < int64_t(sms) * 32) A->ell_inst = ELL_FEW;
@@ -404,8 +405,8 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
       } else {
         UP(A->d_coo_row, A->coo.row);
       }
-      // per-interval carries of the fix-up
-      const size_t nU = size_t(A->nI);
+      // carries of the fix-up: one per work unit (<= max(intervals, warps per block))
+      const size_t nU = size_t(std::max<int64_t>(A->nI, 32));
       if (st == BRO_OK) st = dev_upload(A, &A->d_cf, nullptr, nU * A->vsize);
       if (st == BRO_OK) st = dev_upload(A, &A->d_cl, nullptr, nU * A->vsize);
       if (st == BRO_OK) st = dev_upload(A, &A->d_last_row, nullptr, nU * 4);
@@ -505,9 +506,11 @@ bro::dev::CooDev<T> coo_dev(const bro_matrix_s* A, const T* x) {
                             static_cast<T*>(A->d_cf), static_cast<T*>(A->d_cl), A->d_first_row, A->d_last_row};
 }
 
+// Persistent COO grid: one work unit (a contiguous range of intervals) per
+// resident warp, at most one per interval; the fix-up runs over the units.
 int64_t coo_grid(const bro_matrix_s* A, const Launch& L) {
   const int64_t w = L.k.warps_per_block();
-  return (A->nI + w - 1) / w;  // one warp per interval
+  return std::max<int64_t>(1, std::min(A->nI, L.resident_blocks * w) / w);
 }
 
 // y = A.x stored into every destination of yo (yo.p[0] = the local y on A's
@@ -529,9 +532,10 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
   if (e == cudaSuccess && A->has_coo && A->nI > 0) {
     bro::dev::CooDev<T> p = coo_dev<T>(A, x);
     int32_t* none = nullptr;
-    e = launch(A->coo_k[0], coo_grid(A, A->coo_k[0]), st, p, y, none);
+    const int64_t grid = coo_grid(A, A->coo_k[0]);
+    e = launch(A->coo_k[0], grid, st, p, y, none);
     if (e == cudaSuccess) {
-      int64_t nU = A->nI;
+      int64_t nU = grid * A->coo_k[0].k.warps_per_block();
       const int32_t* fr = A->d_first_row;
       const int32_t* lr = A->d_last_row;
       const T* cf = static_cast<const T*>(A->d_cf);
