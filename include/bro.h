@@ -120,6 +120,9 @@ typedef struct {
                         window (< 18), 5 general.  An instance the matrix does not fit
                         gives BRO_ERR_ARG.  For A/B measurements and tests (6..10: A/B
                         candidates of the small / mid window instances). */
+  int32_t coo_prefetch; /* BRO-COO / COO: 0 (default) = auto (on when the part needs more
+                        than one wave of warps: each warp asks the TMA engine to prefetch
+                        into L2 the interval one resident wave ahead), 1 = on, 2 = off. */
 } bro_opts_t;
 
 typedef struct {

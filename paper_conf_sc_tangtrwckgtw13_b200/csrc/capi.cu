@@ -156,6 +156,7 @@ bro_status_t check_opts(const bro_opts_t& o) {
   if (o.codec != 0 && o.codec != 1) return fail(BRO_ERR_ARG, "codec must be 0 or 1");
   if (o.hyb_K < -1) return fail(BRO_ERR_ARG, "hyb_K must be >= -1");
   if (o.min_bits < 0 || o.min_bits > 31) return fail(BRO_ERR_ARG, "min_bits must be in [0, 31]");
+  if (o.coo_prefetch < 0 || o.coo_prefetch > 2) return fail(BRO_ERR_ARG, "coo_prefetch must be 0, 1 or 2");
   if (o.ell_kernel < 0 || o.ell_kernel > bro::ELL_LAST)
     return fail(BRO_ERR_ARG, "ell_kernel must be in [0, " + std::to_string(bro::ELL_LAST) + "]");
   return BRO_OK;
@@ -234,6 +235,10 @@ bro_status_t choose_ell_instance(bro_matrix_s* A, int sms) {
   const bool small_family = want == ELL_SMALL || want == ELL_X6 || want == ELL_X7 || want == ELL_X10 ||
                             (A->h == 64 && want == ELL_X8);
   const bool mid_family = want == ELL_MID || want == ELL_X9 || (A->h == 32 && want == ELL_X8);
+  // (X6: small + prefetch; X7: small + prefetch + pipelined groups, 24 warps/SM;
+  //  X8: h=32 mid + prefetch / h=64 small + prefetch + pipelined, 16 warps/SM;
+  //  X9: mid + prefetch + pipelined; X10: h=32 small + prefetch + pipelined G=8,
+  //  16 warps / h=64 small + prefetch, 16 warps)
   if (want == ELL_AUTO) {
     if (tiny_ok) A->ell_inst = ELL_TINY;
     else if (A->h == 32 && A->s < int64_t(sms) * 32) A->ell_inst = ELL_FEW;
@@ -503,14 +508,12 @@ template <typename T>
 bro::dev::CooDev<T> coo_dev(const bro_matrix_s* A, const T* x) {
   return bro::dev::CooDev<T>{A->nnz_coo, A->nI, A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr,
                             A->d_coo_row, A->d_coo_col, static_cast<const T*>(A->d_coo_vals), x,
-                            static_cast<T*>(A->d_cf), static_cast<T*>(A->d_cl), A->d_first_row, A->d_last_row};
+                            static_cast<T*>(A->d_cf), static_cast<T*>(A->d_cl), A->d_first_row, A->d_last_row, 0};
 }
 
-// Persistent COO grid: one work unit (a contiguous range of intervals) per
-// resident warp, at most one per interval; the fix-up runs over the units.
 int64_t coo_grid(const bro_matrix_s* A, const Launch& L) {
   const int64_t w = L.k.warps_per_block();
-  return std::max<int64_t>(1, std::min(A->nI, L.resident_blocks * w) / w);
+  return (A->nI + w - 1) / w;  // one warp per interval
 }
 
 // y = A.x stored into every destination of yo (yo.p[0] = the local y on A's
@@ -532,10 +535,12 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
   if (e == cudaSuccess && A->has_coo && A->nI > 0) {
     bro::dev::CooDev<T> p = coo_dev<T>(A, x);
     int32_t* none = nullptr;
-    const int64_t grid = coo_grid(A, A->coo_k[0]);
-    e = launch(A->coo_k[0], grid, st, p, y, none);
+    // prefetch one resident wave ahead, when there is more than one wave
+    const int64_t wave = A->coo_k[0].resident_blocks * A->coo_k[0].k.warps_per_block();
+    p.pf = A->opts.coo_prefetch != 2 && A->nI > wave ? wave : 0;
+    e = launch(A->coo_k[0], coo_grid(A, A->coo_k[0]), st, p, y, none);
     if (e == cudaSuccess) {
-      int64_t nU = grid * A->coo_k[0].k.warps_per_block();
+      int64_t nU = A->nI;
       const int32_t* fr = A->d_first_row;
       const int32_t* lr = A->d_last_row;
       const T* cf = static_cast<const T*>(A->d_cf);
@@ -671,6 +676,7 @@ void bro_opts_default(bro_opts_t* o) {
   o->codec = 1;
   o->min_bits = 0;
   o->ell_kernel = 0;
+  o->coo_prefetch = 0;
 }
 
 bro_status_t bro_create_ell(int device, bro_dtype_t dtype, int64_t m, int64_t n, const int64_t* row_ptr,

@@ -31,12 +31,12 @@ KernelRef ell_pick(int inst) {
       case ELL_SMALL: return {(const void*)&bro_ell_od<T, V, 1, 16, 2, 8, kEllRowsSmall, M>, 512};
       case ELL_MID: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M>, 256};
       case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsGen, M>, 256};
-      // A/B candidates: small window + TMA L2 prefetch of the next slice
+      // A/B candidates: small window + TMA L2 prefetch of the next slice (+ pipelined groups)
       case ELL_X6: return {(const void*)&bro_ell_od<T, V, 1, 16, 2, 8, kEllRowsSmall, M, 1>, 512};
-      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 1, 16, 2, 8, kEllRowsSmall, M, 1, false, 2>, 512};
+      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 1, 8, 3, 4, kEllRowsSmall, M, 1, false, 0, true>, 256};
       case ELL_X8: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M, 1>, 256};
-      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M, 1, false, 2>, 256};
-      case ELL_X10: return {(const void*)&bro_ell_od<T, V, 1, 16, 2, 8, kEllRowsSmall, M, 1, false, 3>, 512};
+      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 1, 8, 3, 4, kEllRowsMid, M, 1, false, 0, true>, 256};
+      case ELL_X10: return {(const void*)&bro_ell_od<T, V, 1, 8, 2, 8, kEllRowsSmall, M, 1, false, 0, true>, 256};
     }
   } else {
     switch (inst) {
@@ -45,9 +45,9 @@ KernelRef ell_pick(int inst) {
       case ELL_MID: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M>, 256};
       case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 2, 4, 4, 4, kEllRowsGen, M>, 128};
       case ELL_X6: return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsSmall, M, 1>, 256};
-      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsSmall, M, 1, false, 2>, 256};
-      case ELL_X8: return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsSmall, M, 1, false, 3>, 256};
-      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M, 1, false, 2>, 256};
+      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 2, kEllRowsSmall, M, 1, false, 0, true>, 256};
+      case ELL_X8: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsSmall, M, 1, false, 0, true>, 256};
+      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M, 1, false, 0, true>, 256};
       case ELL_X10: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsSmall, M, 1>, 256};
     }
   }

@@ -193,6 +193,7 @@ struct CooDev {           // (BRO-)COO part
   T* cl;                  // per interval: partial of its last row
   int32_t* first_row;
   int32_t* last_row;
+  int64_t pf;             // L2 prefetch distance in intervals (0 = none)
 };
 
 // ------------------------------------------------------------------ BRO-ELL values
@@ -311,11 +312,12 @@ __device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
 // into L2 the values, symbols and widths of the slice this warp handles kPf
 // slices later, so its own loads of that slice hit L2 instead of HBM.
 // kL1: symbol staging through the L1-allocating path.
+// kPipe: software-pipelined column groups (group g+1 issued before group g's FMAs).
 // kPfAt: when the prefetch is issued — 0 at the slice start, k (1..3) once the
 // warp reaches column k*l/4 of the current slice (a later trigger keeps fewer
 // prefetched bytes waiting in L2 per warp, so more warps can prefetch).
 template <typename T, int V, int R, int kWarps, int kMinBlocks, int G, int kRows, int kMode, int kPf = 0,
-          bool kL1 = false, int kPfAt = 0>
+          bool kL1 = false, int kPfAt = 0, bool kPipe = false>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   constexpr int H = 32 * R;
@@ -391,18 +393,23 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
                                       uint32_t(rel & 31) | ((32u - uint32_t(b)) << 8));
       }
       __syncwarp();
-      for (int g = 0; g < nb; g += G) {
+      // one group = G columns of the block: its R x G values, decoded columns
+      // and x gathers (padding slots: delta 0, no gather, no FMA; Alg. 1 line 17)
+      struct Grp {
+        T v[R][G];
+        T xv[R][G];
+        int cidx[R][G];
+        bool ok[R][G];
+      };
+      auto issue = [&](Grp& q, int g) {  // loads of group g: values, decode, gathers
         if constexpr (kPf > 0 && kPfAt > 0 && kMode != kDecode) {
           const int at = (kPfAt * l) >> 2;  // trigger column
           if (jb + g <= at && at < jb + g + G) prefetch_next();
         }
-        T v[R][G];
         if constexpr (kMode != kDecode) {
 #pragma unroll
-          for (int k = 0; k < R; ++k) load_vals<T, G, H>(v[k], vs, jb + g, l, lfull, 32 * k + lane);
+          for (int k = 0; k < R; ++k) load_vals<T, G, H>(q.v[k], vs, jb + g, l, lfull, 32 * k + lane);
         }
-        int cidx[R][G];
-        bool ok[R][G];
 #pragma unroll
         for (int kk = 0; kk < G; ++kk) {
           const uint2 mm = cm[g + kk];  // broadcast
@@ -422,8 +429,8 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
             // funnelshift_l uses the low 5 bits of mm.y (= r); bits 8.. hold 32-b
             const uint32_t d = shr_clamp(__funnelshift_l(lo[k], hi[k], mm.y), sh);
             col[k] += int(d);
-            cidx[k][kk] = col[k];
-            ok[k][kk] = d != 0u;
+            q.cidx[k][kk] = col[k];
+            q.ok[k][kk] = d != 0u;
           }
         }
         if constexpr (kMode == kDecode) {
@@ -432,19 +439,41 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
           for (int k = 0; k < R; ++k)
 #pragma unroll
             for (int kk = 0; kk < G; ++kk)
-              if (g + kk < nb) dec[H * (mt.c0 + jb + g + kk) + 32 * k + lane] = ok[k][kk] ? cidx[k][kk] : -1;
+              if (g + kk < nb) dec[H * (mt.c0 + jb + g + kk) + 32 * k + lane] = q.ok[k][kk] ? q.cidx[k][kk] : -1;
         } else {
-          T xv[R][G];
 #pragma unroll
           for (int k = 0; k < R; ++k)
 #pragma unroll
             for (int kk = 0; kk < G; ++kk)
-              if (ok[k][kk]) xv[k][kk] = ldg_x(p.x + cidx[k][kk]);
+              if (q.ok[k][kk]) q.xv[k][kk] = ldg_x(p.x + q.cidx[k][kk]);
+        }
+      };
+      auto consume = [&](const Grp& q) {
+        if constexpr (kMode != kDecode) {
 #pragma unroll
           for (int k = 0; k < R; ++k)
 #pragma unroll
             for (int kk = 0; kk < G; ++kk)
-              if (ok[k][kk]) sum[k] = fma(v[k][kk], xv[k][kk], sum[k]);  // padding (delta 0) skipped, Alg. 1 line 17
+              if (q.ok[k][kk]) sum[k] = fma(q.v[k][kk], q.xv[k][kk], sum[k]);
+        }
+      };
+      if constexpr (!kPipe) {
+        for (int g = 0; g < nb; g += G) {
+          Grp q;
+          issue(q, g);
+          consume(q);
+        }
+      } else {
+        // software pipeline: group g+G's values and gathers are in flight
+        // while group g's FMAs wait for theirs
+        Grp qa, qb;
+        issue(qa, 0);
+        for (int g = 0; g < nb; g += 2 * G) {
+          if (g + G < nb) issue(qb, g + G);
+          consume(qa);
+          if (g + G >= nb) break;
+          if (g + 2 * G < nb) issue(qa, g + 2 * G);
+          consume(qb);
         }
       }
       obase += tot;
@@ -639,14 +668,7 @@ __device__ __forceinline__ void cp_async4(uint32_t* dst, const uint32_t* src) {
                "l"(src) : "memory");
 }
 
-// Persistent warps: warp u walks the contiguous intervals [iA, iB) =
-// [u*nI/nW, (u+1)*nI/nW) of its work unit.  Per 32 intervals one round trip
-// fetches their headers lane-parallel (broadcast by shuffle); at the start of
-// interval k lane 0 asks the TMA engine to prefetch interval k+kPf's col,
-// vals and words into L2.  Rows continue across the unit's intervals (the
-// trailing segment is carried), so only the unit's first and last rows go
-// through the fix-up: nU = nW units instead of nI intervals.
-template <typename T, bool kBro, int TT, int kWarps, int kMinBlocks, int kMode, int kPf = 1>
+template <typename T, bool kBro, int TT, int kWarps, int kMinBlocks, int kMode>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   constexpr int I = 32 * TT;
@@ -655,113 +677,89 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   __shared__ uint32_t cwin[kWarps][kBro ? (TT + 1) * 32 : 1];  // <= T symbol rows + a zero guard row
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
-  const int64_t nW = int64_t(gridDim.x) * kWarps;
-  const int64_t u = int64_t(blockIdx.x) * kWarps + w;  // this warp's work unit
-  const int64_t iA = u * p.nI / nW, iB = (u + 1) * p.nI / nW;
-  if (iA >= iB) {  // (the launcher keeps nW <= nI) an empty unit: a row no interval holds
-    if (kMode != kDecode && lane == 0) { p.first_row[u] = -1; p.last_row[u] = -1; p.cf[u] = T(0); p.cl[u] = T(0); }
-    return;
-  }
+  const int64_t i = int64_t(blockIdx.x) * kWarps + w;
+  if (i >= p.nI) return;
+  const int64_t e0 = i * I;
+  const int32_t* cb = p.col + e0;
+  const T* vb = p.vals + e0;
+  // per-lane segment state: f = row of the lane's first entry, A = partial of
+  // its first segment, cr / cur = current (trailing) segment
+  int f = 0, cr = 0;
+  T A = T(0), cur = T(0);
+  bool one = true;
+  int b = 0, S = 0, row = 0, first = 0, lim = 0;
+  uint32_t w0 = 0, w1 = 0;
   const uint32_t* wl = cwin[w] + lane;
-  // headers of intervals [kb, kb + 32) of the unit, lane j holding interval kb + j
-  int h_base = 0, h_b = 0, h_S = 0;
-  uint64_t h_q0 = 0;
-  auto fetch_headers = [&](int64_t i0) {
-    const int64_t il = i0 + lane;
-    if (il < iB) {
-      h_base = int(p.base_row[il]);
-      if constexpr (kBro) {
-        h_b = int(p.width[il]);
-        h_q0 = p.symptr[il];
-        h_S = int(p.symptr[il + 1] - h_q0);
+#pragma unroll
+  for (int ch = 0; ch < NC; ++ch) {
+    // the chunk's col / vals (and plain rows) first: nothing they need
+    // depends on the interval header, so their round trip overlaps the
+    // header -> word staging chain below
+    int r[CH], c[CH];
+    T v[CH];
+    if constexpr (kMode != kDecode) {
+#pragma unroll
+      for (int u = 0; u < CH / 8; ++u) {
+        load8_s32(c + 8 * u, cb, CH * ch + 8 * u, lane);
+        Vec8<T> vv;
+        vv.load(vb, CH * ch + 8 * u, lane);
+#pragma unroll
+        for (int k = 0; k < 8; ++k) v[8 * u + k] = vv.v[k];
       }
     }
-  };
-  const int unit_first = int(p.base_row[iA]);
-  int crow = unit_first;  // row of the carried (trailing) segment
-  T carry = T(0);
-  auto emit = [&](int rr, T val) {
-    if (rr == unit_first) p.cf[u] = val;
-    else atomicAdd(y + rr, val);
-  };
-  for (int64_t i = iA; i < iB; ++i) {
-    const int kk = int((i - iA) & 31);
-    if (kk == 0) fetch_headers(i);
-    const int first = __shfl_sync(0xffffffffu, h_base, kk);  // row of the interval's first entry
-    int b = 0, S = 0;
-    uint64_t q0 = 0;
-    if constexpr (kBro) {
-      b = __shfl_sync(0xffffffffu, h_b, kk);
-      S = __shfl_sync(0xffffffffu, h_S, kk);
-      q0 = __shfl_sync(0xffffffffu, h_q0, kk);
+    if constexpr (!kBro) {
+#pragma unroll
+      for (int u = 0; u < CH / 8; ++u) load8_s32(r + 8 * u, p.rows + e0, CH * ch + 8 * u, lane);
     }
-    if constexpr (kPf > 0 && kMode != kDecode) {
-      const int kn = kk + kPf;
-      if (i + kPf < iB && kn < 32) {
-        const uint64_t qn = __shfl_sync(0xffffffffu, h_q0, kn);
-        const int Sn = __shfl_sync(0xffffffffu, h_S, kn);
-        if (lane == 0) {
-          prefetch_l2(p.col + (i + kPf) * I, uint32_t(I * 4));
-          prefetch_l2(p.vals + (i + kPf) * I, uint32_t(I * sizeof(T)));
-          if constexpr (kBro) {
-            if (Sn > 0) prefetch_l2(p.words + 32 * qn, uint32_t(128 * Sn));
-          } else {
-            prefetch_l2(p.rows + (i + kPf) * I, uint32_t(I * 4));
+    if (ch == 0) {
+      lim = int(min(int64_t(I), p.nnz - e0));  // valid entries of the interval
+      first = int(p.base_row[i]);              // row of the interval's first entry
+      row = first;
+      // L2 prefetch (TMA engine) of the interval one resident wave ahead:
+      // the warp that will run it then finds its col / vals / words in L2
+      const int64_t ip = i + p.pf;
+      uint64_t qp = 0, qp1 = 0;
+      const bool do_pf = kMode != kDecode && p.pf > 0 && lane == 0 && ip < p.nI;
+      if (do_pf) {
+        prefetch_l2(p.col + ip * I, uint32_t(I * 4));
+        prefetch_l2(p.vals + ip * I, uint32_t(I * sizeof(T)));
+        if constexpr (kBro) { qp = p.symptr[ip]; qp1 = p.symptr[ip + 1]; }
+        else prefetch_l2(p.rows + ip * I, uint32_t(I * 4));
+      }
+      if constexpr (kBro) {
+        b = int(p.width[i]);
+        if (b > 0) {  // b = 0: one row for the whole interval, empty stream
+          const uint64_t q0 = p.symptr[i];
+          S = int(p.symptr[i + 1] - q0);
+          const uint32_t* wb = p.words + 32 * q0 + lane;  // V = 1: word q of lane l at 32q + l
+          if (S <= 2) {
+            // short streams (T*b <= 64 bits; C3/C4 intervals have small row
+            // gaps): the lane's <= 2 words in registers, no window
+            w0 = ld_stream_u32(wb);
+            w1 = S > 1 ? ld_stream_u32(wb + 32) : 0u;
+          } else {  // the lane words -> [q][lane] window by cp.async
+            uint32_t* win = cwin[w] + lane;
+            for (int q = 0; q < S; ++q) cp_async4(win + 32 * q, wb + 32 * q);
+            asm volatile("cp.async.commit_group;" ::: "memory");
+            win[32 * S] = 0u;
           }
         }
+        if (do_pf && qp1 > qp) prefetch_l2(p.words + 32 * qp, uint32_t(128 * (qp1 - qp)));
       }
     }
-    const int64_t e0 = i * I;
-    const int32_t* cb = p.col + e0;
-    const T* vb = p.vals + e0;
-    const int lim = int(min(int64_t(I), p.nnz - e0));  // valid entries of the interval
-    uint32_t w0 = 0, w1 = 0;
+    T xv[CH];
+    if constexpr (kMode != kDecode) {
+#pragma unroll
+      for (int k = 0; k < CH; ++k)  // slots past nnz hold col 0 / value 0: no gather
+        xv[k] = TT * lane + CH * ch + k < lim ? ldg_x(p.x + c[k]) : T(0);
+    }
     if constexpr (kBro) {
-      if (b > 0) {  // b = 0: one row for the whole interval, empty stream
-        const uint32_t* wb = p.words + 32 * q0 + lane;  // V = 1: word q of lane l at 32q + l
-        if (S <= 2) {
-          // short streams (T*b <= 64 bits; C3/C4 intervals have small row
-          // gaps): the lane's <= 2 words in registers, no window
-          w0 = ld_stream_u32(wb);
-          w1 = S > 1 ? ld_stream_u32(wb + 32) : 0u;
-        } else {  // the lane words -> [q][lane] window by cp.async
-          __syncwarp();
-          uint32_t* win = cwin[w] + lane;
-          for (int q = 0; q < S; ++q) cp_async4(win + 32 * q, wb + 32 * q);
-          asm volatile("cp.async.commit_group;" ::: "memory");
-          win[32 * S] = 0u;
-        }
-      }
-    }
-    // per-lane segment state: f = row of the lane's first entry, A = partial
-    // of its first segment, cr / cur = current (trailing) segment
-    int f = 0, cr = 0;
-    T A = T(0), cur = T(0);
-    bool one = true;
-    int row = first;  // running row of this lane (BRO)
-#pragma unroll
-    for (int ch = 0; ch < NC; ++ch) {
-      int r[CH], c[CH];
-      T v[CH], xv[CH];
-      if constexpr (kMode != kDecode) {
-#pragma unroll
-        for (int q = 0; q < CH / 8; ++q) {
-          load8_s32(c + 8 * q, cb, CH * ch + 8 * q, lane);
-          Vec8<T> vv;
-          vv.load(vb, CH * ch + 8 * q, lane);
-#pragma unroll
-          for (int k = 0; k < 8; ++k) v[8 * q + k] = vv.v[k];
-        }
-#pragma unroll
-        for (int k = 0; k < CH; ++k)  // slots past nnz hold col 0 / value 0: no gather
-          xv[k] = TT * lane + CH * ch + k < lim ? ldg_x(p.x + c[k]) : T(0);
-      }
-      if constexpr (!kBro) {
-#pragma unroll
-        for (int q = 0; q < CH / 8; ++q) load8_s32(r + 8 * q, p.rows + e0, CH * ch + 8 * q, lane);
-      } else if (b > 0 && S <= 2) {
+      if (b > 0 && S <= 2) {
         // field t = bits [t*b, t*b + b) of the 64-bit stream w0:w1, MSB first
         const uint64_t W = (uint64_t(w0) << 32) | w1;
+        int d[CH];
+#pragma unroll
+        for (int k = 0; k < CH; ++k) d[k] = int((W << ((CH * ch + k) * b)) >> (64 - b));
         if (ch == 0) {
           int tot = 0;  // sum of this lane's deltas (all T fields)
 #pragma unroll
@@ -776,7 +774,7 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
         }
 #pragma unroll
         for (int k = 0; k < CH; ++k) {
-          row += int((W << ((CH * ch + k) * b)) >> (64 - b));
+          row += d[k];
           r[k] = row;
         }
       } else {
@@ -800,67 +798,62 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
           r[k] = row;
         }
       }
-      if constexpr (kMode == kDecode) {
+    }
+    if constexpr (kMode == kDecode) {
 #pragma unroll
-        for (int k = 0; k < CH; ++k)
-          if (TT * lane + CH * ch + k < lim) dec[e0 + TT * lane + CH * ch + k] = r[k];
-      } else {
+      for (int k = 0; k < CH; ++k)
+        if (TT * lane + CH * ch + k < lim) dec[e0 + TT * lane + CH * ch + k] = r[k];
+    } else {
 #pragma unroll
-        for (int k = 0; k < CH; ++k) {
-          const T prod = v[k] * xv[k];
-          if (ch == 0 && k == 0) {
-            f = r[0];
-            cr = r[0];
-            cur = prod;
-          } else if (r[k] != cr) {  // the segment of row cr ends inside this lane
-            if (one) { A = cur; one = false; }
-            else atomicAdd(y + cr, cur);  // interior segment (row > unit's first): complete, unique here
-            cr = r[k];
-            cur = prod;
-          } else {
-            cur += prod;
-          }
+      for (int k = 0; k < CH; ++k) {
+        const T prod = v[k] * xv[k];
+        if (ch == 0 && k == 0) {
+          f = r[0];
+          cr = r[0];
+          cur = prod;
+        } else if (r[k] != cr) {  // the segment of row cr ends inside this lane
+          if (one) { A = cur; one = false; }
+          else atomicAdd(y + cr, cur);  // interior segment (row > first): complete, unique to this lane
+          cr = r[k];
+          cur = prod;
+        } else {
+          cur += prod;
         }
       }
     }
-    if constexpr (kMode != kDecode) {
-      if (one) A = cur;
-      // segmented scan over the lanes, lane 0 continuing the carried segment:
-      // C_out(l) = cur_l + [one_l && link_l] C_out(l-1)
-      const int L = cr;
-      const int Lprev = __shfl_up_sync(0xffffffffu, L, 1);
-      const bool link = lane == 0 ? crow == f : Lprev == f;
-      T co = cur;
-      bool open = one && link;
-      if (lane == 0 && open) co += carry;
-#pragma unroll
-      for (int off = 1; off < 32; off <<= 1) {
-        const T o = __shfl_up_sync(0xffffffffu, co, off);
-        const int op = __shfl_up_sync(0xffffffffu, int(open), off);
-        if (lane >= off && open) co += o;
-        if (lane >= off) open = open && op;
-      }
-      T cin = __shfl_up_sync(0xffffffffu, co, 1);
-      if (lane == 0) cin = carry;
-      if (!link) cin = T(0);
-      if (lane == 0 && !link) emit(crow, carry);  // the carried row ended before this interval
-      if (!one) emit(f, A + cin);                 // first segment complete inside this lane
-      const int fnext = __shfl_down_sync(0xffffffffu, f, 1);
-      if (lane < 31 && fnext != L) emit(L, co);   // trailing segment complete at this lane
-      carry = __shfl_sync(0xffffffffu, co, 31);
-      crow = __shfl_sync(0xffffffffu, L, 31);
-    }
   }
-  if constexpr (kMode != kDecode) {
-    if (lane == 0) {  // the unit's first and last rows go to the fix-up
-      p.first_row[u] = unit_first;
-      p.last_row[u] = crow;
-      if (crow == unit_first) {
-        p.cf[u] = carry;
-        p.cl[u] = T(0);
-      } else {
-        p.cl[u] = carry;
-      }
+  if constexpr (kMode == kDecode) return;
+  if (one) A = cur;
+  // segmented scan over the lanes: C_out(l) = cur_l + [one_l && link_l] C_out(l-1)
+  const int L = cr;
+  const int Lprev = __shfl_up_sync(0xffffffffu, L, 1);
+  const bool link = lane > 0 && Lprev == f;  // this lane's first row continues the previous lane's last
+  T co = cur;
+  bool open = one && link;
+#pragma unroll
+  for (int off = 1; off < 32; off <<= 1) {
+    const T o = __shfl_up_sync(0xffffffffu, co, off);
+    const int op = __shfl_up_sync(0xffffffffu, int(open), off);
+    if (lane >= off && open) co += o;
+    if (lane >= off) open = open && op;
+  }
+  T cin = __shfl_up_sync(0xffffffffu, co, 1);
+  if (!link) cin = T(0);
+  auto emit = [&](int rr, T val) {
+    if (rr == first) p.cf[i] = val;
+    else atomicAdd(y + rr, val);
+  };
+  if (!one) emit(f, A + cin);  // first segment complete inside this lane
+  const int fnext = __shfl_down_sync(0xffffffffu, f, 1);
+  if (lane < 31 && fnext != L) emit(L, co);  // trailing segment complete at this lane
+  if (lane == 31) {  // the interval's last row: its partial is carried
+    p.first_row[i] = first;
+    p.last_row[i] = L;
+    if (L == first) {
+      p.cf[i] = co;
+      p.cl[i] = T(0);
+    } else {
+      p.cl[i] = co;
     }
   }
 }
