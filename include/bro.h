@@ -120,9 +120,10 @@ typedef struct {
                         window (< 18), 5 general.  An instance the matrix does not fit
                         gives BRO_ERR_ARG.  For A/B measurements and tests (6..10: A/B
                         candidates of the small / mid window instances). */
-  int32_t coo_prefetch; /* BRO-COO / COO: 0 (default) = auto (on when the part needs more
-                        than one wave of warps: each warp asks the TMA engine to prefetch
-                        into L2 the interval one resident wave ahead), 1 = on, 2 = off. */
+  int32_t pdl;       /* HYB / COO: 0 (default) = 1 = the COO kernel is launched as a
+                        programmatic dependent of the ELL kernel (its loads, decode and x
+                        gathers overlap the ELL kernel's tail; it waits before updating y),
+                        and the fix-up as one of the COO kernel; 2 = plain stream order. */
 } bro_opts_t;
 
 typedef struct {

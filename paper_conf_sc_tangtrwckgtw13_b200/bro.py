@@ -33,7 +33,7 @@ FORMATS = {0: "ELL", 1: "COO", 2: "HYB"}
 class bro_opts_t(C.Structure):
     _fields_ = [("slice_h", C.c_int32), ("sym_bits", C.c_int32), ("vec_words", C.c_int32),
                 ("coo_T", C.c_int32), ("hyb_K", C.c_int64), ("codec", C.c_int32),
-                ("min_bits", C.c_int32), ("ell_kernel", C.c_int32), ("coo_prefetch", C.c_int32)]
+                ("min_bits", C.c_int32), ("ell_kernel", C.c_int32), ("pdl", C.c_int32)]
 
 
 class bro_info_t(C.Structure):
@@ -246,12 +246,12 @@ class BroMatrix:
     pointers reach the library (the C ABI cannot)."""
 
     def __init__(self, A, fmt="ell", codec=1, device=0, dtype=None, vec_words=0, hyb_K=-1, min_bits=0,
-                 slice_h=0, coo_T=0, ell_kernel=0, coo_prefetch=0):
+                 slice_h=0, coo_T=0, ell_kernel=0, pdl=0):
         vals = A.vals if dtype is None else A.vals.astype(dtype)
         self.dtype = np.dtype(vals.dtype)
         self.m, self.n, self.fmt, self.device = A.m, A.n, fmt, device
         opts = bro_opts_default(codec=codec, vec_words=vec_words, hyb_K=hyb_K, min_bits=min_bits,
-                                slice_h=slice_h, coo_T=coo_T, ell_kernel=ell_kernel, coo_prefetch=coo_prefetch)
+                                slice_h=slice_h, coo_T=coo_T, ell_kernel=ell_kernel, pdl=pdl)
         if fmt == "ell":
             self.h = bro_create_ell(device, A.m, A.n, A.row_ptr, A.col, vals, opts)
         elif fmt == "hyb":

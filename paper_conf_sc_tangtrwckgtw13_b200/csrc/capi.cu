@@ -156,7 +156,7 @@ bro_status_t check_opts(const bro_opts_t& o) {
   if (o.codec != 0 && o.codec != 1) return fail(BRO_ERR_ARG, "codec must be 0 or 1");
   if (o.hyb_K < -1) return fail(BRO_ERR_ARG, "hyb_K must be >= -1");
   if (o.min_bits < 0 || o.min_bits > 31) return fail(BRO_ERR_ARG, "min_bits must be in [0, 31]");
-  if (o.coo_prefetch < 0 || o.coo_prefetch > 2) return fail(BRO_ERR_ARG, "coo_prefetch must be 0, 1 or 2");
+  if (o.pdl < 0 || o.pdl > 2) return fail(BRO_ERR_ARG, "pdl must be 0, 1 or 2");
   if (o.ell_kernel < 0 || o.ell_kernel > bro::ELL_LAST)
     return fail(BRO_ERR_ARG, "ell_kernel must be in [0, " + std::to_string(bro::ELL_LAST) + "]");
   return BRO_OK;
@@ -465,6 +465,25 @@ cudaError_t launch(const Launch& L, int64_t grid, cudaStream_t st, Args&... args
   return cudaLaunchKernel(L.k.fn, dim3(unsigned(grid)), dim3(unsigned(L.k.threads)), a, 0, st);
 }
 
+// Launch as a programmatic dependent of the previous kernel on the stream
+// (PDL): it may start while that kernel drains; it waits (griddepcontrol.wait)
+// before touching what that kernel writes.
+template <typename... Args>
+cudaError_t launch_pdl(const Launch& L, int64_t grid, cudaStream_t st, Args&... args) {
+  if (grid <= 0) return cudaSuccess;
+  void* a[] = {static_cast<void*>(&args)...};
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(unsigned(grid));
+  cfg.blockDim = dim3(unsigned(L.k.threads));
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelExC(&cfg, L.k.fn, a);
+}
+
 // Persistent grids: as many blocks as the device keeps resident, capped by the work.
 int64_t persistent_grid(const Launch& L, int64_t units) {
   const int64_t w = L.k.warps_per_block();
@@ -508,7 +527,7 @@ template <typename T>
 bro::dev::CooDev<T> coo_dev(const bro_matrix_s* A, const T* x) {
   return bro::dev::CooDev<T>{A->nnz_coo, A->nI, A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr,
                             A->d_coo_row, A->d_coo_col, static_cast<const T*>(A->d_coo_vals), x,
-                            static_cast<T*>(A->d_cf), static_cast<T*>(A->d_cl), A->d_first_row, A->d_last_row, 0};
+                            static_cast<T*>(A->d_cf), static_cast<T*>(A->d_cl), A->d_first_row, A->d_last_row};
 }
 
 int64_t coo_grid(const bro_matrix_s* A, const Launch& L) {
@@ -535,17 +554,20 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
   if (e == cudaSuccess && A->has_coo && A->nI > 0) {
     bro::dev::CooDev<T> p = coo_dev<T>(A, x);
     int32_t* none = nullptr;
-    // prefetch one resident wave ahead, when there is more than one wave
-    const int64_t wave = A->coo_k[0].resident_blocks * A->coo_k[0].k.warps_per_block();
-    p.pf = A->opts.coo_prefetch != 2 && A->nI > wave ? wave : 0;
-    e = launch(A->coo_k[0], coo_grid(A, A->coo_k[0]), st, p, y, none);
+    // the COO kernel overlaps the ELL kernel's tail, the fix-up the COO
+    // kernel's (programmatic dependent launches, bro_opts_t.pdl)
+    const bool pdl = A->opts.pdl != 2;
+    const bool after_ell = A->has_ell && pdl;
+    e = after_ell ? launch_pdl(A->coo_k[0], coo_grid(A, A->coo_k[0]), st, p, y, none)
+                  : launch(A->coo_k[0], coo_grid(A, A->coo_k[0]), st, p, y, none);
     if (e == cudaSuccess) {
       int64_t nU = A->nI;
       const int32_t* fr = A->d_first_row;
       const int32_t* lr = A->d_last_row;
       const T* cf = static_cast<const T*>(A->d_cf);
       const T* cl = static_cast<const T*>(A->d_cl);
-      e = launch(A->fix_k, (nU + 255) / 256, st, nU, fr, lr, cf, cl, y);
+      e = pdl ? launch_pdl(A->fix_k, (nU + 255) / 256, st, nU, fr, lr, cf, cl, y)
+              : launch(A->fix_k, (nU + 255) / 256, st, nU, fr, lr, cf, cl, y);
     }
   }
   if (e == cudaSuccess && !fused && A->m > 0 && multi) {
@@ -676,7 +698,7 @@ void bro_opts_default(bro_opts_t* o) {
   o->codec = 1;
   o->min_bits = 0;
   o->ell_kernel = 0;
-  o->coo_prefetch = 0;
+  o->pdl = 0;
 }
 
 bro_status_t bro_create_ell(int device, bro_dtype_t dtype, int64_t m, int64_t n, const int64_t* row_ptr,

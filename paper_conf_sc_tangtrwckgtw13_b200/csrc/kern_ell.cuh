@@ -45,7 +45,7 @@ KernelRef ell_pick(int inst) {
       case ELL_MID: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M>, 256};
       case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 2, 4, 4, 4, kEllRowsGen, M>, 128};
       case ELL_X6: return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsSmall, M, 1>, 256};
-      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 2, kEllRowsSmall, M, 1, false, 0, true>, 256};
+      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, f64 ? 2 : 4, kEllRowsSmall, M, 1, false, 0, true>, 256};
       case ELL_X8: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsSmall, M, 1, false, 0, true>, 256};
       case ELL_X9: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M, 1, false, 0, true>, 256};
       case ELL_X10: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsSmall, M, 1>, 256};

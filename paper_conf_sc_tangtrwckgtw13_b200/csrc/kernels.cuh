@@ -193,8 +193,14 @@ struct CooDev {           // (BRO-)COO part
   T* cl;                  // per interval: partial of its last row
   int32_t* first_row;
   int32_t* last_row;
-  int64_t pf;             // L2 prefetch distance in intervals (0 = none)
 };
+
+// Programmatic dependent launch (PDL): a kernel launched with the
+// programmatic-serialization attribute may start while the previous kernel
+// of the stream finishes; it must execute griddepcontrol.wait before it
+// touches memory that kernel writes.  Without the attribute both are no-ops.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_launch_dependents() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
 // ------------------------------------------------------------------ BRO-ELL values
 // G values of row r (slot columns j .. j+G-1) of a slice of H rows: 16-byte
@@ -320,6 +326,7 @@ template <typename T, int V, int R, int kWarps, int kMinBlocks, int G, int kRows
           bool kL1 = false, int kPfAt = 0, bool kPipe = false>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
+  static_assert(G % Chunk<T>::N == 0, "a column group holds whole 16-byte value chunks");
   constexpr int H = 32 * R;
   struct Meta { uint64_t c0, q0; int l, S; };
   __shared__ __align__(16) uint32_t window[kWarps][kRows * H];
@@ -327,6 +334,7 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   __shared__ Meta metas[kWarps][32];     // metadata of this warp's next 32 slices
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
+  if constexpr (kMode == kSpmv) pdl_launch_dependents();  // a HYB handle's COO part may be scheduled
   uint32_t* win = window[w];
   const uint2* cm = colmeta[w];
   const char* win_lane = reinterpret_cast<const char*>(win + lane * R);
@@ -504,6 +512,7 @@ bro_ell_tiny(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   __shared__ Meta metas[kWarps][32];  // metadata of this warp's next 32 slices
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
+  if constexpr (kMode == kSpmv) pdl_launch_dependents();  // a HYB handle's COO part may be scheduled
   const int64_t stride = int64_t(gridDim.x) * kWarps;
   int k32 = 0;
   for (int64_t t = int64_t(blockIdx.x) * kWarps + w; t < p.s; t += stride, k32 = (k32 + 1) & 31) {
@@ -586,6 +595,7 @@ __global__ void __launch_bounds__(kThreads)
 ell_spmv(const PellDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   constexpr int G = 8;
   const int64_t row = int64_t(blockIdx.x) * kThreads + threadIdx.x;
+  if constexpr (kMode == kSpmv) pdl_launch_dependents();  // a HYB handle's COO part may be scheduled
   if (row >= p.m) return;
   if constexpr (kMode == kDecode) {
     for (int64_t j = 0; j < p.K; ++j) dec[j * p.pitch + row] = ld_stream_s32(p.col + j * p.pitch + row);
@@ -678,6 +688,7 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
   const int64_t i = int64_t(blockIdx.x) * kWarps + w;
+  if constexpr (kMode != kDecode) pdl_launch_dependents();  // the fix-up may be scheduled
   if (i >= p.nI) return;
   const int64_t e0 = i * I;
   const int32_t* cb = p.col + e0;
@@ -715,17 +726,6 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
       lim = int(min(int64_t(I), p.nnz - e0));  // valid entries of the interval
       first = int(p.base_row[i]);              // row of the interval's first entry
       row = first;
-      // L2 prefetch (TMA engine) of the interval one resident wave ahead:
-      // the warp that will run it then finds its col / vals / words in L2
-      const int64_t ip = i + p.pf;
-      uint64_t qp = 0, qp1 = 0;
-      const bool do_pf = kMode != kDecode && p.pf > 0 && lane == 0 && ip < p.nI;
-      if (do_pf) {
-        prefetch_l2(p.col + ip * I, uint32_t(I * 4));
-        prefetch_l2(p.vals + ip * I, uint32_t(I * sizeof(T)));
-        if constexpr (kBro) { qp = p.symptr[ip]; qp1 = p.symptr[ip + 1]; }
-        else prefetch_l2(p.rows + ip * I, uint32_t(I * 4));
-      }
       if constexpr (kBro) {
         b = int(p.width[i]);
         if (b > 0) {  // b = 0: one row for the whole interval, empty stream
@@ -744,7 +744,6 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
             win[32 * S] = 0u;
           }
         }
-        if (do_pf && qp1 > qp) prefetch_l2(p.words + 32 * qp, uint32_t(128 * (qp1 - qp)));
       }
     }
     T xv[CH];
@@ -804,6 +803,9 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
       for (int k = 0; k < CH; ++k)
         if (TT * lane + CH * ch + k < lim) dec[e0 + TT * lane + CH * ch + k] = r[k];
     } else {
+      // everything above only read constant inputs; y (stored by the ELL
+      // part of a HYB handle) is updated from here on
+      if (ch == 0) pdl_wait();
 #pragma unroll
       for (int k = 0; k < CH; ++k) {
         const T prod = v[k] * xv[k];
@@ -923,6 +925,7 @@ template <typename T>
 __global__ void coo_fixup(int64_t nU, const int32_t* __restrict__ first, const int32_t* __restrict__ last_row,
                           const T* __restrict__ cf, const T* __restrict__ cl, T* __restrict__ y) {
   const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  pdl_wait();  // the carries come from the COO kernel
   if (i >= nU) return;
   const int F = first[i];
   const int L = last_row[i];

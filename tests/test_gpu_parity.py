@@ -393,3 +393,20 @@ def test_config5_row_blocks(lib, dev):
         M.close()
     y = np.concatenate(ys)
     _check_y(A, x, y, np.float64, chunk_rows=2_000_000)
+
+
+@pytest.mark.parametrize("fmt", ["hyb", "coo"])
+@pytest.mark.parametrize("codec", [1, 0])
+def test_pdl_chain_same_bits(lib, dev, fmt, codec):
+    """The COO kernel launched as a programmatic dependent of the ELL kernel
+    (and the fix-up of the COO kernel) gives the same bits as plain stream
+    order (bro_opts_t.pdl = 2), and the oracle's y."""
+    A = random_csr(30000, 30000, 41, max_len=9, empty_frac=0.1, long_frac=0.01, long_len=2000)
+    x = make_x(A.n, 7)
+    ys = []
+    for pdl in (0, 2):
+        M, _, y = _run(lib, A, fmt, codec, np.float64, dev, x=x, pdl=pdl)
+        _check_y(A, x, y, np.float64)
+        ys.append(y)
+        M.close()
+    assert np.array_equal(ys[0], ys[1])
