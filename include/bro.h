@@ -99,7 +99,8 @@ typedef struct {
                         32 (one row per lane of the slice's warp), 64 (two rows per lane:
                         widths, offsets and setup shared by both rows), 0 (default) =
                         auto: 64 when m >= 303,104 (64 rows x 32 resident warps x 148
-                        SMs: every resident warp of a B200 still gets slices), else 32.
+                        SMs: every resident warp of a B200 still gets slices) and some
+                        row of the ELL part has more than 4 entries, else 32.
                         bro_info_t.slice_h reports the value. */
   int32_t sym_bits;  /* sym_len. Must be 32. */
   int32_t vec_words; /* V: 1 or 4 symbols per lane chunk.  1 = the paper's multiplexing

@@ -232,13 +232,8 @@ bro_status_t choose_ell_instance(bro_matrix_s* A, int sms) {
   const bool tiny_ok = A->ell_max_l <= kEllTinyCols;
   const bool small_ok = A->ell_max_S < kEllRowsSmall;
   const bool mid_ok = A->ell_max_S < kEllRowsMid;
-  const bool small_family = want == ELL_SMALL || want == ELL_X6 || want == ELL_X7 || want == ELL_X10 ||
-                            (A->h == 64 && want == ELL_X8);
-  const bool mid_family = want == ELL_MID || want == ELL_X9 || (A->h == 32 && want == ELL_X8);
-  // (X6: small + prefetch; X7: small + prefetch + pipelined groups, 24 warps/SM;
-  //  X8: h=32 mid + prefetch / h=64 small + prefetch + pipelined, 16 warps/SM;
-  //  X9: mid + prefetch + pipelined; X10: h=32 small + prefetch + pipelined G=8,
-  //  16 warps / h=64 small + prefetch, 16 warps)
+  const bool small_family = want == ELL_SMALL;
+  const bool mid_family = want == ELL_MID || (want >= ELL_X6 && want <= ELL_X10);  // X6..X10: mid-window A/B
   if (want == ELL_AUTO) {
     if (tiny_ok) A->ell_inst = ELL_TINY;
     else if (A->h == 32 && A->s < int64_t(sms) * 32) A->ell_inst = ELL_FEW;
@@ -308,7 +303,16 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
   A->format = format;
   A->m = m; A->n = n; A->nnz = row_ptr[m];
   A->K = K;
-  A->h = o.codec && o.slice_h ? o.slice_h : (o.codec && m >= kAutoH64Rows ? 64 : 32);
+  if (o.codec && o.slice_h) {
+    A->h = o.slice_h;
+  } else if (o.codec && m >= kAutoH64Rows && format != FMT_COO) {
+    // h = 64 for big matrices, except when every row of the ELL part has <= 4
+    // entries (the tiny instance: no setup for two rows to share)
+    int64_t maxlen = 0;
+    for (int64_t i = 0; i < m && maxlen <= bro::kEllTinyCols; ++i)
+      maxlen = std::max(maxlen, std::min(K, row_ptr[i + 1] - row_ptr[i]));
+    A->h = maxlen > bro::kEllTinyCols ? 64 : 32;
+  }
   A->opts.slice_h = A->h;
   const uint8_t* v8 = static_cast<const uint8_t*>(vals);
   try {

@@ -28,27 +28,38 @@ KernelRef ell_pick(int inst) {
       case ELL_FEW:
         if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 1, 8, 2, 16, kEllRowsGen, M>, 256};
         else return {(const void*)&bro_ell_od<T, V, 1, 4, 2, 32, kEllRowsGen, M>, 128};
-      case ELL_SMALL: return {(const void*)&bro_ell_od<T, V, 1, 16, 2, 8, kEllRowsSmall, M>, 512};
+      case ELL_SMALL:
+        // fp64: 24 warps/SM, pipelined 4-column groups, TMA L2 prefetch of the
+        // warp's next slice (C5 343 -> 339 us); fp32: 32 warps/SM, 8 columns
+        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 1, 8, 3, 4, kEllRowsSmall, M, 1, false, 0, true>, 256};
+        else return {(const void*)&bro_ell_od<T, V, 1, 16, 2, 8, kEllRowsSmall, M>, 512};
       case ELL_MID: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M>, 256};
       case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsGen, M>, 256};
-      // A/B candidates: small window + TMA L2 prefetch of the next slice (+ pipelined groups)
-      case ELL_X6: return {(const void*)&bro_ell_od<T, V, 1, 16, 2, 8, kEllRowsSmall, M, 1>, 512};
-      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 1, 8, 3, 4, kEllRowsSmall, M, 1, false, 0, true>, 256};
-      case ELL_X8: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M, 1>, 256};
-      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 1, 8, 3, 4, kEllRowsMid, M, 1, false, 0, true>, 256};
-      case ELL_X10: return {(const void*)&bro_ell_od<T, V, 1, 8, 2, 8, kEllRowsSmall, M, 1, false, 0, true>, 256};
+      // A/B candidates (mid window)
+      case ELL_X6: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M, 1>, 256};
+      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 1, 8, 3, 4, kEllRowsMid, M, 1, false, 0, true>, 256};
+      case ELL_X8: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M, 1, false, 2>, 256};
+      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 1, 8, 2, 8, kEllRowsMid, M, 1, false, 0, true>, 256};
+      case ELL_X10: return {(const void*)&bro_ell_od<T, V, 1, 8, 5, 4, kEllRowsMid, M>, 256};
     }
   } else {
     switch (inst) {
       case ELL_TINY: return {(const void*)&bro_ell_tiny<T, V, 2, 8, 4, M>, 256};
-      case ELL_SMALL: return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsSmall, M>, 256};
+      case ELL_SMALL:
+        // TMA L2 prefetch of the warp's next slice; the prefetched bytes wait in
+        // L2 for about one slice time, so the warps per SM are chosen to keep
+        // them near 35-40 MB chip-wide: 16 warps (fp64, 14.7 KB slices of C5),
+        // 32 warps (fp32, 8.7 KB)
+        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsSmall, M, 1>, 256};
+        else return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsSmall, M, 1>, 256};
       case ELL_MID: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M>, 256};
       case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 2, 4, 4, 4, kEllRowsGen, M>, 128};
-      case ELL_X6: return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsSmall, M, 1>, 256};
-      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, f64 ? 2 : 4, kEllRowsSmall, M, 1, false, 0, true>, 256};
-      case ELL_X8: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsSmall, M, 1, false, 0, true>, 256};
-      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M, 1, false, 0, true>, 256};
-      case ELL_X10: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsSmall, M, 1>, 256};
+      // A/B candidates (mid window)
+      case ELL_X6: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M, 1>, 256};
+      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsMid, M, 1>, 256};
+      case ELL_X8: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 8, kEllRowsMid, M>, 256};
+      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsMid, M, 1, false, 2>, 256};
+      case ELL_X10: return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 2 * Chunk<T>::N, kEllRowsMid, M>, 256};
     }
   }
   return {};

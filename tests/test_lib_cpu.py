@@ -156,7 +156,7 @@ def test_hyb_split_and_parts_match_oracle_c3(lib):
         assert 0.6 < ec.size / A.nnz < 0.7  # webbase-1M: 64.2% in BRO-ELL (Table 4)
         assert info["vec_words"] == 1  # auto layout for fp64: the paper's multiplexing
         H, T = info["slice_h"], info["coo_T"]
-        assert H == 64 and T == 8  # auto: 1M rows >= 303,104; 1.1M COO entries < 16*32*4736
+        assert H == 32 and T == 8  # auto: ELL part rows <= K = 2 (tiny); 1.1M COO entries < 16*32*4736
         sample = [0, 1, 777, 15624]
         E = bro_ell.encode(ep, ec, ev, A.m, A.n, h=H, V=1, slices=sample)
         words = lib.bro_export_encoded(h, "ell_words")
