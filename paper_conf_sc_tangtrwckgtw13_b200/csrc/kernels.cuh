@@ -237,28 +237,27 @@ __device__ __forceinline__ void load_vals(T* v, const T* vs, int j, int l, int l
 
 // Copy symbol rows [qa, qa + nrows) of this lane's R rows into
 // win[((q - qa) * 32 + lane) * R + k] (zeros past S) plus one zero guard row.
-// kL1: symbol words through the L1-allocating read-only path (__ldg) instead
-// of the no-allocate streaming load (V = 1 only).
-template <int V, int R, bool kL1 = false>
+// Copy symbol rows [qa, qa + nrows) of this lane's R rows into
+// win[((q - qa) * 32 + lane) * R + k] (zeros past S) plus one zero guard row.
+// kB rows per batch, every load of a batch issued before its first store, so
+// a window of n rows arrives in ceil(n / kB) round trips (the group loop's
+// registers are free at this point of the slice).
+template <int V, int R, int kB>
 __device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __restrict__ wb, int S, int qa,
                                               int nrows, int lane) {
   constexpr int H = 32 * R;
   if constexpr (V == 1) {
-    // 4 rows per step, every load issued before the first store: the rows of
-    // a slice arrive in ceil(nrows / 4) round trips, not one per row pair
-    for (int r0 = 0; r0 < nrows; r0 += 4) {
-      uint32_t w[4][R];
+    for (int r0 = 0; r0 < nrows; r0 += kB) {
+      uint32_t w[kB][R];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
+      for (int u = 0; u < kB; ++u) {
         const int q = qa + r0 + u;
 #pragma unroll
         for (int k = 0; k < R; ++k)
-          w[u][k] = (r0 + u < nrows && q < S)
-                        ? (kL1 ? __ldg(wb + H * q + 32 * k + lane) : ld_stream_u32(wb + H * q + 32 * k + lane))
-                        : 0u;
+          w[u][k] = (r0 + u < nrows && q < S) ? ld_stream_u32(wb + H * q + 32 * k + lane) : 0u;
       }
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
+      for (int u = 0; u < kB; ++u) {
         if (r0 + u < nrows) {
           if constexpr (R == 1) win[(r0 + u) * 32 + lane] = w[u][0];
           else reinterpret_cast<uint2*>(win)[(r0 + u) * 32 + lane] = make_uint2(w[u][0], w[u][1]);
@@ -267,29 +266,37 @@ __device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __r
     }
   } else {
     static_assert(V == 4, "V must be 1 or 4");
+    constexpr int kC = (kB + 3) / 4 + 1;  // 16-byte chunks covering kB rows at any alignment
     const int F = S >> 2;
     const int Vp = S - 4 * F;
     const int c_lo = qa >> 2, c_hi = (qa + nrows - 1) >> 2;
-    for (int c = c_lo; c <= c_hi; ++c) {
-      uint32_t w4[R][4];
+    for (int c0 = c_lo; c0 <= c_hi; c0 += kC) {
+      uint32_t w4[kC][R][4];
 #pragma unroll
-      for (int k = 0; k < R; ++k) {
-        const int row = 32 * k + lane;
-        if (c < F) {
-          const uint4 v = ld_stream_u4(wb + H * 4 * c + 4 * row);
-          w4[k][0] = v.x; w4[k][1] = v.y; w4[k][2] = v.z; w4[k][3] = v.w;
-        } else {
+      for (int cc = 0; cc < kC; ++cc) {
+        const int c = c0 + cc;
 #pragma unroll
-          for (int e = 0; e < 4; ++e)
-            w4[k][e] = (c == F && e < Vp) ? ld_stream_u32(wb + H * 4 * F + Vp * row + e) : 0u;
+        for (int k = 0; k < R; ++k) {
+          const int row = 32 * k + lane;
+          if (c <= c_hi && c < F) {
+            const uint4 v = ld_stream_u4(wb + H * 4 * c + 4 * row);
+            w4[cc][k][0] = v.x; w4[cc][k][1] = v.y; w4[cc][k][2] = v.z; w4[cc][k][3] = v.w;
+          } else {
+#pragma unroll
+            for (int e = 0; e < 4; ++e)
+              w4[cc][k][e] = (c <= c_hi && c == F && e < Vp) ? ld_stream_u32(wb + H * 4 * F + Vp * row + e) : 0u;
+          }
         }
       }
 #pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const int r = 4 * c + e - qa;
-        if (r >= 0 && r < nrows) {
-          if constexpr (R == 1) win[r * 32 + lane] = w4[0][e];
-          else reinterpret_cast<uint2*>(win)[r * 32 + lane] = make_uint2(w4[0][e], w4[1][e]);
+      for (int cc = 0; cc < kC; ++cc) {
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const int r = 4 * (c0 + cc) + e - qa;
+          if (c0 + cc <= c_hi && r >= 0 && r < nrows) {
+            if constexpr (R == 1) win[r * 32 + lane] = w4[cc][0][e];
+            else reinterpret_cast<uint2*>(win)[r * 32 + lane] = make_uint2(w4[cc][0][e], w4[cc][1][e]);
+          }
         }
       }
     }
@@ -317,7 +324,6 @@ __device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
 // kPf > 0: at the start of a slice, lane 0 asks the TMA engine to prefetch
 // into L2 the values, symbols and widths of the slice this warp handles kPf
 // slices later, so its own loads of that slice hit L2 instead of HBM.
-// kL1: symbol staging through the L1-allocating path.
 // kPipe: software-pipelined column groups (group g+1 issued before group g's FMAs).
 // kPfAt: when the prefetch is issued — 0 at the slice start, k (1..3) once the
 // warp reaches column k*l/4 of the current slice (a later trigger keeps fewer
@@ -327,6 +333,11 @@ template <typename T, int V, int R, int kWarps, int kMinBlocks, int G, int kRows
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   static_assert(G % Chunk<T>::N == 0, "a column group holds whole 16-byte value chunks");
+  // symbol rows staged per round trip, sized by the instance's register
+  // budget (16 / 12 / 8 loads in flight for >= 96 / >= 80 / fewer registers)
+  constexpr int kMaxRegs = 65536 / (kWarps * 32 * kMinBlocks);
+  constexpr int kLoads = kMaxRegs >= 96 ? 16 : kMaxRegs >= 80 ? 12 : 8;
+  constexpr int kStageB = kRows - 1 < kLoads / R ? kRows - 1 : kLoads / R;
   constexpr int H = 32 * R;
   struct Meta { uint64_t c0, q0; int l, S; };
   __shared__ __align__(16) uint32_t window[kWarps][kRows * H];
@@ -380,7 +391,7 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
       const int b = lane < nb ? int(__ldg(ba + jb + lane)) : 0;
       if (jb == 0) {  // first block starts at symbol 0: stage without waiting for the scan
         __syncwarp();
-        stage_symbols<V, R, kL1>(win, wb, S, 0, min(S, kRows - 1), lane);
+        stage_symbols<V, R, kStageB>(win, wb, S, 0, min(S, kRows - 1), lane);
       }
       int incl = b;  // inclusive scan of the widths over the block
 #pragma unroll
@@ -393,7 +404,7 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
       const int nrows = tot > 0 ? ((obase + tot - 1) >> 5) - qa + 1 : 0;
       if (jb > 0) {
         __syncwarp();
-        stage_symbols<V, R, kL1>(win, wb, S, qa, nrows, lane);
+        stage_symbols<V, R, kStageB>(win, wb, S, qa, nrows, lane);
       }
       {
         const int rel = b ? obase + incl - b - 32 * qa : 0;  // column jb+lane inside the window
