@@ -232,8 +232,8 @@ bro_status_t choose_ell_instance(bro_matrix_s* A, int sms) {
   const bool tiny_ok = A->ell_max_l <= kEllTinyCols;
   const bool small_ok = A->ell_max_S < kEllRowsSmall;
   const bool mid_ok = A->ell_max_S < kEllRowsMid;
-  const bool small_family = want == ELL_SMALL;
-  const bool mid_family = want == ELL_MID || (want >= ELL_X6 && want <= ELL_X10);  // X6..X10: mid-window A/B
+  const bool small_family = want == ELL_SMALL || want == ELL_X6;                 // X6: small-window A/B
+  const bool mid_family = want == ELL_MID || (want >= ELL_X7 && want <= ELL_X10);  // X7..X10: mid-window A/B
   if (want == ELL_AUTO) {
     if (tiny_ok) A->ell_inst = ELL_TINY;
     else if (A->h == 32 && A->s < int64_t(sms) * 32) A->ell_inst = ELL_FEW;

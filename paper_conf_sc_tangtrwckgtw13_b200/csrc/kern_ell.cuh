@@ -35,12 +35,14 @@ KernelRef ell_pick(int inst) {
         else return {(const void*)&bro_ell_od<T, V, 1, 16, 2, 8, kEllRowsSmall, M>, 512};
       case ELL_MID: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M>, 256};
       case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsGen, M>, 256};
-      // A/B candidates (mid window)
-      case ELL_X6: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M, 1>, 256};
-      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 1, 8, 3, 4, kEllRowsMid, M, 1, false, 0, true>, 256};
-      case ELL_X8: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M, 1, false, 2>, 256};
-      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 1, 8, 2, 8, kEllRowsMid, M, 1, false, 0, true>, 256};
-      case ELL_X10: return {(const void*)&bro_ell_od<T, V, 1, 8, 5, 4, kEllRowsMid, M>, 256};
+      // A/B candidates: staging batch (kSB) / mid window occupancy
+      case ELL_X6:
+        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 1, 8, 3, 4, kEllRowsSmall, M, 1, false, 0, true, 4>, 256};
+        else return {(const void*)&bro_ell_od<T, V, 1, 16, 2, 8, kEllRowsSmall, M, 0, false, 0, false, 4>, 512};
+      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M, 0, false, 0, false, 4>, 256};
+      case ELL_X8: return {(const void*)&bro_ell_od<T, V, 1, 8, 5, 4, kEllRowsMid, M, 0, false, 0, false, 4>, 256};
+      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 1, 8, 5, 4, kEllRowsMid, M, 0, false, 0, false, 8>, 256};
+      case ELL_X10: return {(const void*)&bro_ell_od<T, V, 1, 8, 6, 4, kEllRowsMid, M, 0, false, 0, false, 4>, 256};
     }
   } else {
     switch (inst) {
@@ -54,12 +56,14 @@ KernelRef ell_pick(int inst) {
         else return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsSmall, M, 1>, 256};
       case ELL_MID: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M>, 256};
       case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 2, 4, 4, 4, kEllRowsGen, M>, 128};
-      // A/B candidates (mid window)
-      case ELL_X6: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M, 1>, 256};
-      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsMid, M, 1>, 256};
-      case ELL_X8: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 8, kEllRowsMid, M>, 256};
-      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsMid, M, 1, false, 2>, 256};
-      case ELL_X10: return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 2 * Chunk<T>::N, kEllRowsMid, M>, 256};
+      // A/B candidates: staging batch (kSB) / mid window occupancy
+      case ELL_X6:
+        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsSmall, M, 1, false, 0, false, 4>, 256};
+        else return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsSmall, M, 1, false, 0, false, 4>, 256};
+      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M, 0, false, 0, false, 4>, 256};
+      case ELL_X8: return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsMid, M, 0, false, 0, false, 2>, 256};
+      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M, 0, false, 0, false, 8>, 256};
+      case ELL_X10: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 8, kEllRowsMid, M, 1, false, 0, false, 4>, 256};
     }
   }
   return {};

@@ -62,6 +62,19 @@ __device__ __forceinline__ uint32_t ld_stream_u32(const uint32_t* p) {
   asm("ld.global.nc.L1::no_allocate.L2::256B.u32 %0, [%1];" : "=r"(r) : "l"(p));
   return r;
 }
+// never speculated: a guarded load stays a predicated load (symbol staging,
+// whose guards cut off the words of the NEXT slice)
+__device__ __forceinline__ uint32_t ld_stream_u32_g(const uint32_t* p) {
+  uint32_t r;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::256B.u32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ uint4 ld_stream_u4_g(const void* p) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::256B.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
 __device__ __forceinline__ int32_t ld_stream_s32(const int32_t* p) {
   int32_t r;
   asm("ld.global.nc.L1::no_allocate.L2::256B.s32 %0, [%1];" : "=r"(r) : "l"(p));
@@ -253,8 +266,11 @@ __device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __r
       for (int u = 0; u < kB; ++u) {
         const int q = qa + r0 + u;
 #pragma unroll
-        for (int k = 0; k < R; ++k)
-          w[u][k] = (r0 + u < nrows && q < S) ? ld_stream_u32(wb + H * q + 32 * k + lane) : 0u;
+        for (int k = 0; k < R; ++k) w[u][k] = 0u;
+        if (r0 + u < nrows && q < S) {
+#pragma unroll
+          for (int k = 0; k < R; ++k) w[u][k] = ld_stream_u32_g(wb + H * q + 32 * k + lane);
+        }
       }
 #pragma unroll
       for (int u = 0; u < kB; ++u) {
@@ -278,13 +294,15 @@ __device__ __forceinline__ void stage_symbols(uint32_t* win, const uint32_t* __r
 #pragma unroll
         for (int k = 0; k < R; ++k) {
           const int row = 32 * k + lane;
+#pragma unroll
+          for (int e = 0; e < 4; ++e) w4[cc][k][e] = 0u;
           if (c <= c_hi && c < F) {
-            const uint4 v = ld_stream_u4(wb + H * 4 * c + 4 * row);
+            const uint4 v = ld_stream_u4_g(wb + H * 4 * c + 4 * row);
             w4[cc][k][0] = v.x; w4[cc][k][1] = v.y; w4[cc][k][2] = v.z; w4[cc][k][3] = v.w;
-          } else {
+          } else if (c <= c_hi && c == F) {
 #pragma unroll
             for (int e = 0; e < 4; ++e)
-              w4[cc][k][e] = (c <= c_hi && c == F && e < Vp) ? ld_stream_u32(wb + H * 4 * F + Vp * row + e) : 0u;
+              if (e < Vp) w4[cc][k][e] = ld_stream_u32_g(wb + H * 4 * F + Vp * row + e);
           }
         }
       }
@@ -329,7 +347,7 @@ __device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
 // warp reaches column k*l/4 of the current slice (a later trigger keeps fewer
 // prefetched bytes waiting in L2 per warp, so more warps can prefetch).
 template <typename T, int V, int R, int kWarps, int kMinBlocks, int G, int kRows, int kMode, int kPf = 0,
-          bool kL1 = false, int kPfAt = 0, bool kPipe = false>
+          bool kL1 = false, int kPfAt = 0, bool kPipe = false, int kSB = 0>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   static_assert(G % Chunk<T>::N == 0, "a column group holds whole 16-byte value chunks");
@@ -337,7 +355,7 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   // budget (16 / 12 / 8 loads in flight for >= 96 / >= 80 / fewer registers)
   constexpr int kMaxRegs = 65536 / (kWarps * 32 * kMinBlocks);
   constexpr int kLoads = kMaxRegs >= 96 ? 16 : kMaxRegs >= 80 ? 12 : 8;
-  constexpr int kStageB = kRows - 1 < kLoads / R ? kRows - 1 : kLoads / R;
+  constexpr int kStageB = kSB ? kSB : (kRows - 1 < kLoads / R ? kRows - 1 : kLoads / R);
   constexpr int H = 32 * R;
   struct Meta { uint64_t c0, q0; int l, S; };
   __shared__ __align__(16) uint32_t window[kWarps][kRows * H];

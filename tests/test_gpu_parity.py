@@ -139,7 +139,7 @@ def _fits(A, h, inst):
         return inst == 5
     l, S, _ = bro_ell.slice_shapes(A.row_ptr, A.col, A.m, h, 32)
     small, mid = S.max(initial=0) < 10, S.max(initial=0) < 18
-    return {1: l.max(initial=0) <= 4, 2: True, 3: small, 4: mid, 5: True, 6: mid, 7: mid,
+    return {1: l.max(initial=0) <= 4, 2: True, 3: small, 4: mid, 5: True, 6: small, 7: mid,
             8: mid, 9: mid, 10: mid}[inst]
 
 
