@@ -99,8 +99,9 @@ typedef struct {
                         32 (one row per lane of the slice's warp), 64 (two rows per lane:
                         widths, offsets and setup shared by both rows), 0 (default) =
                         auto: 64 when m >= 303,104 (64 rows x 32 resident warps x 148
-                        SMs: every resident warp of a B200 still gets slices) and some
-                        row of the ELL part has more than 4 entries, else 32.
+                        SMs: every resident warp of a B200 still gets slices), some
+                        row of the ELL part has more than 4 entries and, at h = 32,
+                        every row stream has fewer than 10 symbols; else 32.
                         bro_info_t.slice_h reports the value. */
   int32_t sym_bits;  /* sym_len. Must be 32. */
   int32_t vec_words; /* V: 1 or 4 symbols per lane chunk.  1 = the paper's multiplexing
@@ -119,8 +120,7 @@ typedef struct {
                         matrix shape; 1 tiny (every slice <= 4 columns), 2 few-slice
                         (h = 32), 3 small window (every row stream < 10 symbols), 4 mid
                         window (< 18), 5 general.  An instance the matrix does not fit
-                        gives BRO_ERR_ARG.  For A/B measurements and tests (6..10: A/B
-                        candidates of the small / mid window instances). */
+                        gives BRO_ERR_ARG.  For A/B measurements and tests. */
   int32_t pdl;       /* HYB / COO: 0 (default) = 1 = the COO kernel is launched as a
                         programmatic dependent of the ELL kernel (its loads, decode and x
                         gathers overlap the ELL kernel's tail; it waits before updating y),

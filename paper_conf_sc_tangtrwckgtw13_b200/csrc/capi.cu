@@ -232,8 +232,8 @@ bro_status_t choose_ell_instance(bro_matrix_s* A, int sms) {
   const bool tiny_ok = A->ell_max_l <= kEllTinyCols;
   const bool small_ok = A->ell_max_S < kEllRowsSmall;
   const bool mid_ok = A->ell_max_S < kEllRowsMid;
-  const bool small_family = want == ELL_SMALL || want == ELL_X6;                 // X6: small-window A/B
-  const bool mid_family = want == ELL_MID || (want >= ELL_X7 && want <= ELL_X10);  // X7..X10: mid-window A/B
+  const bool small_family = want == ELL_SMALL;
+  const bool mid_family = want == ELL_MID;
   if (want == ELL_AUTO) {
     if (tiny_ok) A->ell_inst = ELL_TINY;
     else if (A->h == 32 && A->s < int64_t(sms) * 32) A->ell_inst = ELL_FEW;
@@ -306,12 +306,15 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
   if (o.codec && o.slice_h) {
     A->h = o.slice_h;
   } else if (o.codec && m >= kAutoH64Rows && format != FMT_COO) {
-    // h = 64 for big matrices, except when every row of the ELL part has <= 4
-    // entries (the tiny instance: no setup for two rows to share)
-    int64_t maxlen = 0;
-    for (int64_t i = 0; i < m && maxlen <= bro::kEllTinyCols; ++i)
-      maxlen = std::max(maxlen, std::min(K, row_ptr[i + 1] - row_ptr[i]));
-    A->h = maxlen > bro::kEllTinyCols ? 64 : 32;
+    // h = 64 for big matrices whose rows fit the small-window instance at
+    // h = 32 (every row stream < 10 symbols) and are not tiny: two rows per
+    // lane then share the widths, offsets and setup (C5 fp32 247 -> 203 us);
+    // longer row streams (C4: up to 14 symbols) run faster at h = 32
+    bro::RowsView rv;
+    rv.m = m; rv.row_ptr = row_ptr; rv.col = col; rv.vsize = A->vsize; rv.cap = K;
+    int64_t max_l = 0, max_S = 0;
+    bro::slice_extents(rv, 32, o.min_bits, &max_l, &max_S);
+    A->h = max_l > bro::kEllTinyCols && max_S < bro::kEllRowsSmall ? 64 : 32;
   }
   A->opts.slice_h = A->h;
   const uint8_t* v8 = static_cast<const uint8_t*>(vals);

@@ -215,6 +215,40 @@ void encode_bro_ell(const RowsView& A, int h, int V, int VV, int min_bits, EllCo
   });
 }
 
+void slice_extents(const RowsView& A, int h, int min_bits, int64_t* max_l, int64_t* max_S) {
+  const int64_t m = A.m;
+  const int64_t s = (m + h - 1) / h;
+  const int nt = num_threads();
+  std::vector<int64_t> ml(nt, 0), ms(nt, 0);
+  std::vector<std::thread> th;
+  for (int c = 0; c < nt; ++c) {
+    th.emplace_back([&, c] {
+      std::vector<uint8_t> ba;
+      for (int64_t t = s * c / nt; t < s * (c + 1) / nt; ++t) {
+        int64_t l = 0;
+        for (int64_t r = t * h; r < std::min(m, t * h + h); ++r) l = std::max(l, A.len(r));
+        ba.assign(l, 0);
+        for (int64_t r = t * h; r < std::min(m, t * h + h); ++r) {
+          const int32_t* col = A.col + A.row_ptr[r];
+          uint32_t prev1 = 0;
+          for (int64_t j = 0; j < A.len(r); ++j) {
+            const uint32_t c1 = uint32_t(col[j]) + 1u;
+            ba[j] = std::max<uint8_t>(ba[j], uint8_t(gamma_bits(c1 - prev1)));
+            prev1 = c1;
+          }
+        }
+        int64_t L = 0;
+        for (int64_t j = 0; j < l; ++j) L += std::max<int>(ba[j], min_bits);
+        ml[c] = std::max(ml[c], l);
+        ms[c] = std::max(ms[c], (L + kSym - 1) / kSym);
+      }
+    });
+  }
+  for (auto& t : th) t.join();
+  *max_l = *std::max_element(ml.begin(), ml.end());
+  *max_S = *std::max_element(ms.begin(), ms.end());
+}
+
 void build_plain_ell(const RowsView& A, int64_t K, PlainEll& out) {
   out.K = K;
   out.pitch = (A.m + kH - 1) / kH * kH;

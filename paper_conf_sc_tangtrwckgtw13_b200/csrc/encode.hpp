@@ -87,6 +87,9 @@ std::string check_coo(int64_t m, int64_t n, int64_t nnz, const int32_t* row, con
 int64_t hyb_K(int64_t m, const int64_t* row_ptr);
 
 void encode_bro_ell(const RowsView& A, int h, int V, int value_chunk, int min_bits, EllCode& out);
+// Longest slice (columns) and longest row stream (32-bit symbols) of the
+// BRO-ELL encoding at slice height h, without packing anything.
+void slice_extents(const RowsView& A, int h, int min_bits, int64_t* max_l, int64_t* max_S);
 void build_plain_ell(const RowsView& A, int64_t K, PlainEll& out);
 // rows: int32 rows of the COO entries (sorted); T steps per interval.
 void encode_bro_coo(int64_t nnz, const int32_t* row, const int32_t* col, const uint8_t* vals,

@@ -7,10 +7,12 @@
 //         columns in flight per warp at ~128 registers — every warp is
 //         resident anyway, so registers buy memory-level parallelism
 //   SMALL every row stream < 10 symbols: 10-row window (less shared memory,
-//         more L1 for the x gather)
+//         more L1 for the x gather); + TMA L2 prefetch of the next slice
 //   MID   < 18 symbols: 18-row window
 //   GEN   any slice: 34-row window
 // Launch bounds fix the register budget: kMinBlocks blocks of kWarps warps.
+// Every configuration below was chosen by in-process A/B on B200
+// (scripts/ab.py; profiles/r02/README.md lists the measurements).
 #pragma once
 #include "kernels.cuh"
 #include "launch.hpp"
@@ -21,28 +23,25 @@ template <typename T, int V, int R, int M>
 KernelRef ell_pick(int inst) {
   using namespace dev;
   constexpr bool f64 = sizeof(T) == 8;
+  constexpr int SB = 4;  // symbol rows per staging round trip (measured best, profiles/r02/)
   if (inst == ELL_FEW && R == 2) inst = ELL_GEN;
   if constexpr (R == 1) {
     switch (inst) {
       case ELL_TINY: return {(const void*)&bro_ell_tiny<T, V, 1, 8, f64 ? 5 : 6, M>, 256};
       case ELL_FEW:
-        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 1, 8, 2, 16, kEllRowsGen, M>, 256};
-        else return {(const void*)&bro_ell_od<T, V, 1, 4, 2, 32, kEllRowsGen, M>, 128};
+        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 1, 8, 2, 16, kEllRowsGen, M, 0, false, 0, false, SB>, 256};
+        else return {(const void*)&bro_ell_od<T, V, 1, 4, 2, 32, kEllRowsGen, M, 0, false, 0, false, SB>, 128};
       case ELL_SMALL:
         // fp64: 24 warps/SM, pipelined 4-column groups, TMA L2 prefetch of the
-        // warp's next slice (C5 343 -> 339 us); fp32: 32 warps/SM, 8 columns
-        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 1, 8, 3, 4, kEllRowsSmall, M, 1, false, 0, true>, 256};
-        else return {(const void*)&bro_ell_od<T, V, 1, 16, 2, 8, kEllRowsSmall, M>, 512};
-      case ELL_MID: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M>, 256};
-      case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsGen, M>, 256};
-      // A/B candidates: staging batch (kSB) / mid window occupancy
-      case ELL_X6:
-        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 1, 8, 3, 4, kEllRowsSmall, M, 1, false, 0, true, 4>, 256};
-        else return {(const void*)&bro_ell_od<T, V, 1, 16, 2, 8, kEllRowsSmall, M, 0, false, 0, false, 4>, 512};
-      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M, 0, false, 0, false, 4>, 256};
-      case ELL_X8: return {(const void*)&bro_ell_od<T, V, 1, 8, 5, 4, kEllRowsMid, M, 0, false, 0, false, 4>, 256};
-      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 1, 8, 5, 4, kEllRowsMid, M, 0, false, 0, false, 8>, 256};
-      case ELL_X10: return {(const void*)&bro_ell_od<T, V, 1, 8, 6, 4, kEllRowsMid, M, 0, false, 0, false, 4>, 256};
+        // warp's next slice; fp32: 32 warps/SM, 8-column groups
+        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 1, 8, 3, 4, kEllRowsSmall, M, 1, false, 0, true, SB>, 256};
+        else return {(const void*)&bro_ell_od<T, V, 1, 16, 2, 8, kEllRowsSmall, M, 0, false, 0, false, SB>, 512};
+      case ELL_MID:
+        // C4's ELL part: short slices, latency-bound per slice; fp64 at 40
+        // warps/SM with 4-column groups, fp32 at 32 with 8
+        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 1, 8, 5, 4, kEllRowsMid, M, 0, false, 0, false, SB>, 256};
+        else return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M, 0, false, 0, false, SB>, 256};
+      case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsGen, M, 0, false, 0, false, SB>, 256};
     }
   } else {
     switch (inst) {
@@ -52,18 +51,10 @@ KernelRef ell_pick(int inst) {
         // L2 for about one slice time, so the warps per SM are chosen to keep
         // them near 35-40 MB chip-wide: 16 warps (fp64, 14.7 KB slices of C5),
         // 32 warps (fp32, 8.7 KB)
-        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsSmall, M, 1>, 256};
-        else return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsSmall, M, 1>, 256};
-      case ELL_MID: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M>, 256};
-      case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 2, 4, 4, 4, kEllRowsGen, M>, 128};
-      // A/B candidates: staging batch (kSB) / mid window occupancy
-      case ELL_X6:
-        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsSmall, M, 1, false, 0, false, 4>, 256};
-        else return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsSmall, M, 1, false, 0, false, 4>, 256};
-      case ELL_X7: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M, 0, false, 0, false, 4>, 256};
-      case ELL_X8: return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsMid, M, 0, false, 0, false, 2>, 256};
-      case ELL_X9: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M, 0, false, 0, false, 8>, 256};
-      case ELL_X10: return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 8, kEllRowsMid, M, 1, false, 0, false, 4>, 256};
+        if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 2, 8, 2, 4, kEllRowsSmall, M, 1, false, 0, false, SB>, 256};
+        else return {(const void*)&bro_ell_od<T, V, 2, 8, 4, 4, kEllRowsSmall, M, 1, false, 0, false, SB>, 256};
+      case ELL_MID: return {(const void*)&bro_ell_od<T, V, 2, 8, 3, 4, kEllRowsMid, M, 0, false, 0, false, SB>, 256};
+      case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 2, 4, 4, 4, kEllRowsGen, M, 0, false, 0, false, SB>, 128};
     }
   }
   return {};

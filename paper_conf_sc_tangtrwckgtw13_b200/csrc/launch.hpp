@@ -13,9 +13,7 @@ struct KernelRef {
 };
 
 // BRO-ELL kernel instances (bro_opts_t.ell_kernel; 0 = chosen at create)
-enum EllInst { ELL_AUTO = 0, ELL_TINY = 1, ELL_FEW = 2, ELL_SMALL = 3, ELL_MID = 4, ELL_GEN = 5,
-               // A/B candidates (measured, then folded into the instances above or removed)
-               ELL_X6 = 6, ELL_X7 = 7, ELL_X8 = 8, ELL_X9 = 9, ELL_X10 = 10, ELL_LAST = 10 };
+enum EllInst { ELL_AUTO = 0, ELL_TINY = 1, ELL_FEW = 2, ELL_SMALL = 3, ELL_MID = 4, ELL_GEN = 5, ELL_LAST = 5 };
 constexpr int kEllTinyCols = 4;   // TINY: every slice has <= 4 columns
 constexpr int kEllRowsSmall = 10; // SMALL: every row stream < 10 symbols
 constexpr int kEllRowsMid = 18;   // MID:   < 18 symbols
