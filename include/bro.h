@@ -125,6 +125,11 @@ typedef struct {
                         programmatic dependent of the ELL kernel (its loads, decode and x
                         gathers overlap the ELL kernel's tail; it waits before updating y),
                         and the fix-up as one of the COO kernel; 2 = plain stream order. */
+  int32_t x_stage;   /* few-slice BRO-ELL instance (h = 32, fewer slices than 148 x 32):
+                        0 (default) = 1 = each block has the TMA engine copy its x
+                        column window (<= 96 KB) into shared memory and gathers from
+                        there, when the window fits and one pass of blocks covers the
+                        matrix (bro_info_t.x_stage_bytes > 0); 2 = gathers from global. */
 } bro_opts_t;
 
 typedef struct {
@@ -136,7 +141,7 @@ typedef struct {
   int32_t slice_h;            /* BRO-ELL slice height (32 or 64) */
   int32_t coo_T;              /* BRO-COO entries per lane of an interval */
   int32_t ell_kernel;         /* BRO-ELL kernel instance resolved at create (see bro_opts_t) */
-  int32_t reserved;
+  int32_t x_stage_bytes;      /* shared memory per block of the x-staged instance (0: not staged) */
   int64_t K;                  /* ELL width bound: HYB K, or max row length for ELL */
   int64_t nnz_ell, nnz_coo;   /* entries in the ELL part and in the COO part */
   int64_t n_slices;           /* BRO-ELL slices s = ceil(m/h) (0 without an ELL part) */
@@ -273,7 +278,9 @@ bro_status_t bro_hyb_K(int64_t m, const int64_t* row_ptr, int64_t* K_out);
  * method 2 = Algorithm 2 with a candidate window (reading R24): line 11's
  * argmin runs over the W non-full partitions nearest to the row's own partition
  * floor(pos/32) in length-sorted order (O(m k W), any m; W >= v equals method 1);
- * W = window, 0 = 64 (ignored by methods 0 and 1).
+ * W = window, 0 = 64 (ignored by methods 0 and 1);
+ * method 3 = method 2 with line 2's length sort replaced by the method-0 signature order
+ * (reading R27): the greedy refines the signature clusters by Eqn (1).
  * Partitions hold 32 rows except the last. */
 bro_status_t bro_reorder_bar(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
                              bro_dtype_t dtype, int32_t method, int32_t window, int64_t* perm_out);

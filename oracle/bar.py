@@ -74,13 +74,15 @@ def window_candidates(pos, sizes, cap, h, W):
     return free[:W]
 
 
-def algorithm2(row_ptr, col, m, h=32, alpha=32, vsize=8, window=None, w=None):
+def algorithm2(row_ptr, col, m, h=32, alpha=32, vsize=8, window=None, w=None, order=None):
     """Algorithm 2, evaluating the full Phi_m of line 9 for every
     candidate partition.  Returns the permutation S_1 ++ S_2 ++ ... .
     window=W restricts line 11 to window_candidates (reading R24); None is
     the paper's algorithm (every non-full partition).  w (warp size, w | h)
     defaults to h: the factor h/w multiplies every partition's term alike and
-    cannot change line 11's argmin (reading R21)."""
+    cannot change line 11's argmin (reading R21).  order: the row sequence D
+    of line 2 (default: the paper's sort by row length); method 3 of
+    bro_reorder_bar passes the signature order (reading R27)."""
     w = h if w is None else w
     row_ptr = np.asarray(row_ptr, dtype=np.int64)
     if m == 0:
@@ -89,7 +91,10 @@ def algorithm2(row_ptr, col, m, h=32, alpha=32, vsize=8, window=None, w=None):
     cap = [h] * (v - 1) + [m - (v - 1) * h]
     S = [[] for _ in range(v)]                                   # line 1
     lens = np.diff(row_ptr)
-    D = sorted(range(m), key=lambda i: (int(lens[i]), i))         # line 2
+    if order is None:
+        D = sorted(range(m), key=lambda i: (int(lens[i]), i))     # line 2
+    else:
+        D = [int(i) for i in order]                               # line 2, reading R27
     seeds = set()
     for t in range(v):                                           # lines 3-6
         S[t].append(D[t * h])

@@ -33,14 +33,15 @@ FORMATS = {0: "ELL", 1: "COO", 2: "HYB"}
 class bro_opts_t(C.Structure):
     _fields_ = [("slice_h", C.c_int32), ("sym_bits", C.c_int32), ("vec_words", C.c_int32),
                 ("coo_T", C.c_int32), ("hyb_K", C.c_int64), ("codec", C.c_int32),
-                ("min_bits", C.c_int32), ("ell_kernel", C.c_int32), ("pdl", C.c_int32)]
+                ("min_bits", C.c_int32), ("ell_kernel", C.c_int32), ("pdl", C.c_int32),
+                ("x_stage", C.c_int32)]
 
 
 class bro_info_t(C.Structure):
     _fields_ = [("m", C.c_int64), ("n", C.c_int64), ("nnz", C.c_int64),
                 ("dtype", C.c_int32), ("codec", C.c_int32), ("format", C.c_int32),
                 ("vec_words", C.c_int32), ("slice_h", C.c_int32), ("coo_T", C.c_int32),
-                ("ell_kernel", C.c_int32), ("reserved", C.c_int32),
+                ("ell_kernel", C.c_int32), ("x_stage_bytes", C.c_int32),
                 ("K", C.c_int64), ("nnz_ell", C.c_int64),
                 ("nnz_coo", C.c_int64), ("n_slices", C.c_int64), ("ell_slots", C.c_int64),
                 ("ell_pitch", C.c_int64), ("n_intervals", C.c_int64),
@@ -246,12 +247,13 @@ class BroMatrix:
     pointers reach the library (the C ABI cannot)."""
 
     def __init__(self, A, fmt="ell", codec=1, device=0, dtype=None, vec_words=0, hyb_K=-1, min_bits=0,
-                 slice_h=0, coo_T=0, ell_kernel=0, pdl=0):
+                 slice_h=0, coo_T=0, ell_kernel=0, pdl=0, x_stage=0):
         vals = A.vals if dtype is None else A.vals.astype(dtype)
         self.dtype = np.dtype(vals.dtype)
         self.m, self.n, self.fmt, self.device = A.m, A.n, fmt, device
         opts = bro_opts_default(codec=codec, vec_words=vec_words, hyb_K=hyb_K, min_bits=min_bits,
-                                slice_h=slice_h, coo_T=coo_T, ell_kernel=ell_kernel, pdl=pdl)
+                                slice_h=slice_h, coo_T=coo_T, ell_kernel=ell_kernel, pdl=pdl,
+                                x_stage=x_stage)
         if fmt == "ell":
             self.h = bro_create_ell(device, A.m, A.n, A.row_ptr, A.col, vals, opts)
         elif fmt == "hyb":

@@ -101,6 +101,13 @@ struct bro_matrix_s {
   Launch ell_k[3];
   Launch coo_k[3];  // 0 spmv, 2 decode
   Launch fix_k, rep_k;
+  // x-window staging of the few-slice instance (row N1): per block {first
+  // column, columns} of its x window, the staged instance, its shared bytes
+  int2* d_xwin = nullptr;
+  std::vector<int2> xwin_host;
+  Launch ell_x;
+  int xwin_bytes = 0;
+  bool xstage = false;
   // end-to-end pipeline of ELL-only handles (bro_spmv_host): column range of
   // every row block (h rows), side streams and events (created on first use)
   std::vector<int32_t> blk_cmin, blk_cmax;
@@ -137,7 +144,8 @@ void free_device(bro_matrix_s* A) {
   DeviceGuard g(A->device);
   void* ps[] = {A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr, A->d_ell_vals, A->d_pell_col,
                 A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr, A->d_coo_row,
-                A->d_coo_col, A->d_coo_vals, A->d_cf, A->d_cl, A->d_last_row, A->d_first_row, A->d_xs, A->d_ys};
+                A->d_coo_col, A->d_coo_vals, A->d_cf, A->d_cl, A->d_last_row, A->d_first_row, A->d_xs, A->d_ys,
+                A->d_xwin};
   for (void* p : ps)
     if (p) cudaFree(p);
   for (cudaEvent_t e : A->e2e_ev) cudaEventDestroy(e);
@@ -157,6 +165,7 @@ bro_status_t check_opts(const bro_opts_t& o) {
   if (o.hyb_K < -1) return fail(BRO_ERR_ARG, "hyb_K must be >= -1");
   if (o.min_bits < 0 || o.min_bits > 31) return fail(BRO_ERR_ARG, "min_bits must be in [0, 31]");
   if (o.pdl < 0 || o.pdl > 2) return fail(BRO_ERR_ARG, "pdl must be 0, 1 or 2");
+  if (o.x_stage < 0 || o.x_stage > 2) return fail(BRO_ERR_ARG, "x_stage must be 0, 1 or 2");
   if (o.ell_kernel < 0 || o.ell_kernel > bro::ELL_LAST)
     return fail(BRO_ERR_ARG, "ell_kernel must be in [0, " + std::to_string(bro::ELL_LAST) + "]");
   return BRO_OK;
@@ -177,6 +186,7 @@ void fill_info(bro_matrix_s* A, double secs) {
   I.m = A->m; I.n = A->n; I.nnz = A->nnz;
   I.dtype = A->dtype; I.codec = A->opts.codec; I.format = A->format; I.vec_words = A->opts.vec_words;
   I.slice_h = A->h; I.coo_T = A->coo_T; I.ell_kernel = A->ell_inst;
+  I.x_stage_bytes = A->xstage ? A->xwin_bytes : 0;
   I.K = A->K; I.nnz_ell = A->nnz_ell; I.nnz_coo = A->nnz_coo;
   I.n_slices = A->s; I.ell_pitch = A->pitch; I.n_intervals = A->nI;
   I.encode_seconds = secs;
@@ -260,6 +270,32 @@ bro_status_t resolve(Launch& L, const bro::KernelRef& k, int sms, const char* wh
   return BRO_OK;
 }
 
+// The x-staged few-slice instance: dynamic shared memory for the largest
+// window, and only if its grid covers every slice in one pass (block b = the
+// b-th group of warps-per-block slices, the group its window was cut for).
+template <typename T>
+bro_status_t resolve_xstage(bro_matrix_s* A, int sms) {
+  const bro::KernelRef k = bro::bro_ell_xstage_ref<T>(A->opts.vec_words);
+  if (!k.fn) return BRO_OK;
+  cudaError_t e = cudaFuncSetAttribute(k.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, A->xwin_bytes);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return BRO_OK;  // no staging on this device
+  }
+  int per_sm = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k.fn, k.threads, A->xwin_bytes);
+  if (e != cudaSuccess || per_sm < 1) {
+    cudaGetLastError();
+    return BRO_OK;
+  }
+  const int64_t blocks = (A->s + k.warps_per_block() - 1) / k.warps_per_block();
+  if (blocks > int64_t(per_sm) * sms) return BRO_OK;  // would need a second pass
+  A->ell_x.k = k;
+  A->ell_x.resident_blocks = int64_t(per_sm) * sms;
+  A->xstage = true;
+  return BRO_OK;
+}
+
 // Resolve every kernel instance of the handle on its device (current).
 template <typename T>
 bro_status_t resolve_kernels(bro_matrix_s* A) {
@@ -274,6 +310,7 @@ bro_status_t resolve_kernels(bro_matrix_s* A) {
       if ((st = choose_ell_instance(A, sms))) return st;
       for (int mode = 0; mode < 3 && !st; ++mode)
         st = resolve(A->ell_k[mode], bro::bro_ell_ref<T>(V, A->h / 32, A->ell_inst, mode), sms, "BRO-ELL");
+      if (!st && A->xwin_bytes > 0 && A->ell_inst == bro::ELL_FEW) st = resolve_xstage<T>(A, sms);
     } else {
       for (int mode = 0; mode < 3 && !st; ++mode) st = resolve(A->ell_k[mode], bro::plain_ell_ref<T>(mode), sms, "ELL");
     }
@@ -366,6 +403,35 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
       A->nI = A->coo.nI;
       A->coo_words = (int64_t)A->coo.words.size();
     }
+    // x windows of the few-slice instance's blocks (row N1): BRO-ELL at h = 32
+    // with fewer slices than the general instance keeps resident (148 SMs x 32)
+    if (A->has_ell && o.codec && o.x_stage != 2 && A->h == 32 && A->ell_max_l > bro::kEllTinyCols &&
+        A->s < kB200Warps && (o.ell_kernel == 0 || o.ell_kernel == bro::ELL_FEW) && !A->host_only) {
+      const int64_t wpb = A->vsize == 8 ? 8 : 4;  // warps per block of the few-slice instance
+      const int64_t E = 16 / A->vsize;            // x elements per 16 bytes
+      const int64_t nb = (A->s + wpb - 1) / wpb;
+      std::vector<int2> win(nb, int2{0, 0});
+      int64_t maxb = 0;
+      for (int64_t b = 0; b < nb; ++b) {
+        int64_t lo = INT64_MAX, hi = -1;
+        for (int64_t r = b * wpb * 32; r < std::min(m, (b + 1) * wpb * 32); ++r) {
+          const int64_t len = std::min(K, row_ptr[r + 1] - row_ptr[r]);
+          if (len <= 0) continue;
+          lo = std::min<int64_t>(lo, col[row_ptr[r]]);
+          hi = std::max<int64_t>(hi, col[row_ptr[r] + len - 1]);
+        }
+        if (hi < 0) continue;
+        lo &= ~(E - 1);  // 16-byte aligned source
+        int64_t cnt = (hi + 1 - lo + E - 1) / E * E;
+        if (lo + cnt > n) cnt = (hi + 1 - lo) / E * E;  // never past x's end: the tail is gathered from global
+        win[b] = int2{int(lo), int(cnt)};
+        maxb = std::max(maxb, cnt * A->vsize);
+      }
+      if (maxb > 0 && maxb <= bro::kXStageMaxBytes) {
+        A->xwin_host = std::move(win);
+        A->xwin_bytes = int(maxb);
+      }
+    }
     // column range of every row block (h rows; ELL-only handles): which part
     // of x a block of rows needs, for the pipelined bro_spmv_host
     if (A->has_ell && !A->has_coo) {
@@ -402,6 +468,7 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
       UP(A->d_symptr, A->ell.symptr);
       if (st == BRO_OK) st = dev_upload(A, &A->d_ell_vals, A->ell.vals.data(), A->ell.vals.size());
     }
+    if (A->xwin_bytes > 0) UP(A->d_xwin, A->xwin_host);
     if (A->has_ell && !o.codec) {
       UP(A->d_pell_col, A->pell.col);
       if (st == BRO_OK) st = dev_upload(A, &A->d_ell_vals, A->pell.vals.data(), A->pell.vals.size());
@@ -472,6 +539,13 @@ cudaError_t launch(const Launch& L, int64_t grid, cudaStream_t st, Args&... args
   return cudaLaunchKernel(L.k.fn, dim3(unsigned(grid)), dim3(unsigned(L.k.threads)), a, 0, st);
 }
 
+template <typename... Args>
+cudaError_t launch_smem(const Launch& L, int64_t grid, size_t smem, cudaStream_t st, Args&... args) {
+  if (grid <= 0) return cudaSuccess;
+  void* a[] = {static_cast<void*>(&args)...};
+  return cudaLaunchKernel(L.k.fn, dim3(unsigned(grid)), dim3(unsigned(L.k.threads)), a, smem, st);
+}
+
 // Launch as a programmatic dependent of the previous kernel on the stream
 // (PDL): it may start while that kernel drains; it waits (griddepcontrol.wait)
 // before touching what that kernel writes.
@@ -521,7 +595,12 @@ cudaError_t launch_ell(const bro_matrix_s* A, int mode, const T* x, const bro::d
   const Launch& L = A->ell_k[mode];
   if (A->opts.codec) {
     bro::dev::EllDev<T> p{r1 - r0, b1 - b0, A->d_words, A->d_bit_alloc, A->d_colptr + b0, A->d_symptr + b0,
-                          static_cast<const T*>(A->d_ell_vals), x};
+                          static_cast<const T*>(A->d_ell_vals), x, A->d_xwin};
+    // whole part, plain SpMV, 16-byte aligned x: the x-window-staged instance
+    if (A->xstage && mode == 0 && b0 == 0 && b1 == A->s && (reinterpret_cast<uintptr_t>(x) & 15) == 0) {
+      const int64_t w = A->ell_x.k.warps_per_block();
+      return launch_smem(A->ell_x, (p.s + w - 1) / w, size_t(A->xwin_bytes), st, p, y, dec);
+    }
     return launch(L, persistent_grid(L, p.s), st, p, y, dec);
   }
   // decode mode covers the padding rows [m, pitch) too (they hold -1)
@@ -706,6 +785,7 @@ void bro_opts_default(bro_opts_t* o) {
   o->min_bits = 0;
   o->ell_kernel = 0;
   o->pdl = 0;
+  o->x_stage = 0;
 }
 
 bro_status_t bro_create_ell(int device, bro_dtype_t dtype, int64_t m, int64_t n, const int64_t* row_ptr,
@@ -901,6 +981,14 @@ bro_status_t bro_reorder_bar(int64_t m, int64_t n, const int64_t* row_ptr, const
       bro::bar_window_order(m, row_ptr, col_idx, dtype == BRO_FP64 ? 8 : 4, window ? window : kBarWindow, perm_out);
       return BRO_OK;
     }
+    if (method == 3) {  // Algorithm 2 windowed, line 2's sequence = the signature order (R27)
+      if (window < 0) return fail(BRO_ERR_ARG, "window must be >= 0");
+      std::vector<int64_t> seed(m);
+      bro::bar_signature_order(m, row_ptr, col_idx, seed.data());
+      bro::bar_window_order(m, row_ptr, col_idx, dtype == BRO_FP64 ? 8 : 4, window ? window : kBarWindow, perm_out,
+                            seed.data());
+      return BRO_OK;
+    }
     if (method == 1) {
       std::string err;
       if (!bro::bar_greedy_order(m, n, row_ptr, col_idx, dtype == BRO_FP64 ? 8 : 4, perm_out, &err))
@@ -910,7 +998,7 @@ bro_status_t bro_reorder_bar(int64_t m, int64_t n, const int64_t* row_ptr, const
   } catch (const std::bad_alloc&) {
     return fail(BRO_ERR_OOM, "host allocation failed");
   }
-  return fail(BRO_ERR_ARG, "method must be 0, 1 or 2");
+  return fail(BRO_ERR_ARG, "method must be 0, 1, 2 or 3");
 }
 
 const char* bro_status_str(bro_status_t s) {

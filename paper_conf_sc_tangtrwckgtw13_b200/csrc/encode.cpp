@@ -494,7 +494,7 @@ namespace bro {
 // most h per column), grown to the partition's longest row.  Full partitions
 // are skipped with two path-compressed "next non-full" forests.
 bool bar_window_order(int64_t m, const int64_t* row_ptr, const int32_t* col, int vsize, int W,
-                      int64_t* perm) {
+                      int64_t* perm, const int64_t* seed_order) {
   const int64_t h = kH;
   if (m == 0) return true;
   if (W < 1) W = 1;
@@ -562,12 +562,16 @@ bool bar_window_order(int64_t m, const int64_t* row_ptr, const int32_t* col, int
     return r - 1;
   };
   auto mark_full = [&](int64_t p) { rpar[p] = p + 1; lpar[p + 1] = p; };
-  // line 2
+  // line 2 (seed_order: the row sequence to use instead, reading R27)
   std::vector<int64_t> D(m);
-  std::iota(D.begin(), D.end(), 0);
-  std::stable_sort(D.begin(), D.end(), [&](int64_t a, int64_t b) {
-    return row_ptr[a + 1] - row_ptr[a] < row_ptr[b + 1] - row_ptr[b];
-  });
+  if (seed_order) {
+    std::copy(seed_order, seed_order + m, D.begin());
+  } else {
+    std::iota(D.begin(), D.end(), 0);
+    std::stable_sort(D.begin(), D.end(), [&](int64_t a, int64_t b) {
+      return row_ptr[a + 1] - row_ptr[a] < row_ptr[b + 1] - row_ptr[b];
+    });
+  }
   // lines 3-6
   for (int64_t t = 0; t < v; ++t) {
     insert(t, D[t * h]);

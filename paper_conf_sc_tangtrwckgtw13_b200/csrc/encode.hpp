@@ -100,7 +100,7 @@ void build_plain_coo(int64_t nnz, const int32_t* row, const int32_t* col, const 
 // BAR reordering
 void bar_signature_order(int64_t m, const int64_t* row_ptr, const int32_t* col, int64_t* perm);
 bool bar_window_order(int64_t m, const int64_t* row_ptr, const int32_t* col, int vsize, int W,
-                      int64_t* perm);
+                      int64_t* perm, const int64_t* seed_order = nullptr);
 bool bar_greedy_order(int64_t m, int64_t n, const int64_t* row_ptr, const int32_t* col, int vsize,
                       int64_t* perm, std::string* err);
 

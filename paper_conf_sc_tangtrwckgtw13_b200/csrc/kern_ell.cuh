@@ -70,6 +70,21 @@ KernelRef ell_pick_mode(int inst, int mode) {
   return {};
 }
 
+// the few-slice instance with its block's x window staged in shared memory
+// (same launch shape as ELL_FEW, spmv mode)
+template <typename T, int V>
+KernelRef ell_xstage_pick() {
+  using namespace dev;
+  constexpr bool f64 = sizeof(T) == 8;
+  if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 1, 8, 2, 16, kEllRowsGen, kSpmv, 0, false, 0, false, 4, true>, 256};
+  else return {(const void*)&bro_ell_od<T, V, 1, 4, 2, 32, kEllRowsGen, kSpmv, 0, false, 0, false, 4, true>, 128};
+}
+
+template <typename T>
+KernelRef bro_ell_xstage_ref_impl(int V) {
+  return V == 1 ? ell_xstage_pick<T, 1>() : ell_xstage_pick<T, 4>();
+}
+
 template <typename T>
 KernelRef bro_ell_ref_impl(int V, int R, int inst, int mode) {
   if (V == 1 && R == 1) return ell_pick_mode<T, 1, 1>(inst, mode);

@@ -181,7 +181,31 @@ struct EllDev {           // a BRO-ELL part (or a range of its slices)
   const uint64_t* symptr;
   const T* vals;
   const T* x;
+  const int2* xwin;       // x-staged instances: per block, {first column, columns} of its x window
 };
+
+// ------------------------------------------------------------------ TMA bulk copy + mbarrier
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n"
+      "WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra WAIT_%=;\n}\n" :: "r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+// bytes (multiple of 16) from global src (16-byte aligned) into shared dst,
+// completion counted on bar (which expects them)
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
 
 template <typename T>
 struct PellDev {          // plain ELLPACK (column-major, -1 padding)
@@ -343,11 +367,16 @@ __device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
 // into L2 the values, symbols and widths of the slice this warp handles kPf
 // slices later, so its own loads of that slice hit L2 instead of HBM.
 // kPipe: software-pipelined column groups (group g+1 issued before group g's FMAs).
+// kX: x-window staging (single-pass grids only: block b handles slices
+// [b*kWarps, (b+1)*kWarps)): at block start one thread has the TMA engine copy
+// the block's x window p.xwin[b] into dynamic shared memory; the gathers then
+// read shared memory (north_star: "the x gather ... with TMA or shared-memory
+// staging where the slice's column window fits").
 // kPfAt: when the prefetch is issued — 0 at the slice start, k (1..3) once the
 // warp reaches column k*l/4 of the current slice (a later trigger keeps fewer
 // prefetched bytes waiting in L2 per warp, so more warps can prefetch).
 template <typename T, int V, int R, int kWarps, int kMinBlocks, int G, int kRows, int kMode, int kPf = 0,
-          bool kL1 = false, int kPfAt = 0, bool kPipe = false, int kSB = 0>
+          bool kL1 = false, int kPfAt = 0, bool kPipe = false, int kSB = 0, bool kX = false>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   static_assert(G % Chunk<T>::N == 0, "a column group holds whole 16-byte value chunks");
@@ -366,6 +395,22 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   if constexpr (kMode == kSpmv) pdl_launch_dependents();  // a HYB handle's COO part may be scheduled
   uint32_t* win = window[w];
   const uint2* cm = colmeta[w];
+  // x window of this block (kX): columns [xlo, xlo + xn) in shared memory
+  extern __shared__ __align__(128) unsigned char dsm[];
+  __shared__ uint64_t xbar;
+  const T* xs = reinterpret_cast<const T*>(dsm);
+  int xlo = 0, xn = 0;
+  if constexpr (kX) {
+    const int2 wl = p.xwin[blockIdx.x];
+    xlo = wl.x;
+    xn = wl.y;
+    if (threadIdx.x == 0) {
+      mbar_init(&xbar, 1);
+      if (xn > 0) bulk_g2s(dsm, p.x + xlo, uint32_t(xn * int(sizeof(T))), &xbar);
+    }
+    __syncthreads();
+  }
+  bool xready = !kX;
   const char* win_lane = reinterpret_cast<const char*>(win + lane * R);
   const int64_t stride = int64_t(gridDim.x) * kWarps;
   int k32 = 0;
@@ -478,11 +523,24 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
             for (int kk = 0; kk < G; ++kk)
               if (g + kk < nb) dec[H * (mt.c0 + jb + g + kk) + 32 * k + lane] = q.ok[k][kk] ? q.cidx[k][kk] : -1;
         } else {
+          if constexpr (kX) {
+            if (!xready) {  // the block's x window has landed in shared memory
+              mbar_wait(&xbar, 0);
+              xready = true;
+            }
+          }
 #pragma unroll
           for (int k = 0; k < R; ++k)
 #pragma unroll
             for (int kk = 0; kk < G; ++kk)
-              if (q.ok[k][kk]) q.xv[k][kk] = ldg_x(p.x + q.cidx[k][kk]);
+              if (q.ok[k][kk]) {
+                if constexpr (kX) {
+                  const int cx = q.cidx[k][kk] - xlo;  // columns past the staged window (its 16-byte tail) from global
+                  q.xv[k][kk] = unsigned(cx) < unsigned(xn) ? xs[cx] : ldg_x(p.x + q.cidx[k][kk]);
+                } else {
+                  q.xv[k][kk] = ldg_x(p.x + q.cidx[k][kk]);
+                }
+              }
         }
       };
       auto consume = [&](const Grp& q) {

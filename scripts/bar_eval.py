@@ -5,7 +5,8 @@ throughput of BRO-HYB under the row orderings of bro_reorder_bar.
 Orderings: the matrix as generated (C2: natural FEM order; C4: scrambled),
 C4's unscrambled family order (the generator's ideal), method 0 (signature
 clustering, DESIGN.md proxy), method 1 (Algorithm 2, exact; m <= 65,536 so C2
-only) and method 2 (Algorithm 2 with a 64-partition candidate window).
+only), method 2 (Algorithm 2 with a 64-partition candidate window) and method
+3 (method 2 over the signature order instead of the length sort, R27).
 
 Reports eta_stream / eta_total (host) and, with --gpu, BRO-HYB and plain HYB
 GFLOP/s (median of timed bro_spmv calls, L2 flushed before each).
@@ -31,7 +32,7 @@ def orderings(cfg):
     yield "as generated", A, 0.0
     if cfg == 4:
         yield "family order (unscrambled)", random_block(seed=4, scramble=False), 0.0
-    for meth in (0, 1, 2):
+    for meth in (0, 1, 2, 3):
         if meth == 1 and A.m > 65536:
             continue
         t = time.perf_counter()
@@ -45,7 +46,7 @@ def gpu_time(A, codec, reps=200):
     M = P.BroMatrix(A, fmt="hyb", codec=codec, device=0)
     x = torch.from_numpy(make_x(A.n, 4)).to(dev)
     y = torch.empty(A.m, dtype=torch.float64, device=dev)
-    flush = torch.empty(64 * 2**20, dtype=torch.int32, device=dev)
+    flush = torch.empty(64 * 2**20, dtype=torch.int32, device=dev)  # 256 MB > 2x L2
     for _ in range(5):
         M.spmv(x, y)
     ts = []

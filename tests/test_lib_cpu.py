@@ -478,3 +478,15 @@ def test_auto_slice_height(lib):
             assert lib.bro_get_info(h)["slice_h"] == want, cfg
         finally:
             lib.bro_destroy(h)
+
+
+@pytest.mark.parametrize("seed,m", [(5, None), (6, 290)])
+def test_bar_method3_matches_oracle(lib, seed, m):
+    """Method 3 (windowed Algorithm 2 over the signature order, R27) ==
+    the oracle's algorithm2(window=8, order=signature_order)."""
+    A = random_block(seed=seed, families=10, fam_rows=32)
+    if m is not None:
+        A = row_block(A, 0, m)
+    perm = lib.bro_reorder_bar(A.m, A.n, A.row_ptr, A.col, method=3, window=8)
+    order = bar.signature_order(A.row_ptr, A.col, A.m)
+    assert np.array_equal(perm, bar.algorithm2(A.row_ptr, A.col, A.m, h=32, window=8, order=order))

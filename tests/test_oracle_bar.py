@@ -107,3 +107,26 @@ def test_algorithm2_output_is_equipartition():
     for W in (None, 2):
         perm = bar.algorithm2(A.row_ptr, A.col, A.m, h=32, window=W)
         assert np.array_equal(np.sort(perm), np.arange(A.m))
+
+
+def test_algorithm2_order_window1_is_the_order():
+    """Reading R27: with a window of one partition every row lands in its own
+    partition pos // h, so the result is the seed order itself (closed form),
+    whatever order is passed for line 2."""
+    from gen import random_block, row_block
+    A = row_block(random_block(seed=3, families=5, fam_rows=32), 0, 150)
+    order = bar.signature_order(A.row_ptr, A.col, A.m)
+    got = bar.algorithm2(A.row_ptr, A.col, A.m, h=32, window=1, order=order)
+    assert np.array_equal(got, order)
+    rev = order[::-1].copy()
+    assert np.array_equal(bar.algorithm2(A.row_ptr, A.col, A.m, h=32, window=1, order=rev), rev)
+
+
+def test_algorithm2_default_order_is_length_sort():
+    """order=None and an explicit stable length sort give the same greedy."""
+    from gen import random_block
+    A = random_block(seed=4, families=3, fam_rows=32)
+    lens = np.diff(A.row_ptr)
+    D = np.array(sorted(range(A.m), key=lambda i: (int(lens[i]), i)))
+    assert np.array_equal(bar.algorithm2(A.row_ptr, A.col, A.m, h=32, window=2),
+                          bar.algorithm2(A.row_ptr, A.col, A.m, h=32, window=2, order=D))
