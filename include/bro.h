@@ -126,10 +126,11 @@ typedef struct {
                         gathers overlap the ELL kernel's tail; it waits before updating y),
                         and the fix-up as one of the COO kernel; 2 = plain stream order. */
   int32_t x_stage;   /* few-slice BRO-ELL instance (h = 32, fewer slices than 148 x 32):
-                        0 (default) = 1 = each block has the TMA engine copy its x
-                        column window (<= 96 KB) into shared memory and gathers from
-                        there, when the window fits and one pass of blocks covers the
-                        matrix (bro_info_t.x_stage_bytes > 0); 2 = gathers from global. */
+                        1 = each block has the TMA engine copy its x column window
+                        (<= 96 KB) into shared memory and gathers from there, when the
+                        window fits and one pass of blocks covers the matrix
+                        (bro_info_t.x_stage_bytes > 0); 0 (default) = gathers through
+                        L1/L2 (measured faster on C2: 19.5 vs 22.6 us fp64). */
 } bro_opts_t;
 
 typedef struct {

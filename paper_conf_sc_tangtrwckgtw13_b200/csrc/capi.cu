@@ -165,7 +165,7 @@ bro_status_t check_opts(const bro_opts_t& o) {
   if (o.hyb_K < -1) return fail(BRO_ERR_ARG, "hyb_K must be >= -1");
   if (o.min_bits < 0 || o.min_bits > 31) return fail(BRO_ERR_ARG, "min_bits must be in [0, 31]");
   if (o.pdl < 0 || o.pdl > 2) return fail(BRO_ERR_ARG, "pdl must be 0, 1 or 2");
-  if (o.x_stage < 0 || o.x_stage > 2) return fail(BRO_ERR_ARG, "x_stage must be 0, 1 or 2");
+  if (o.x_stage < 0 || o.x_stage > 1) return fail(BRO_ERR_ARG, "x_stage must be 0 or 1");
   if (o.ell_kernel < 0 || o.ell_kernel > bro::ELL_LAST)
     return fail(BRO_ERR_ARG, "ell_kernel must be in [0, " + std::to_string(bro::ELL_LAST) + "]");
   return BRO_OK;
@@ -405,7 +405,7 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
     }
     // x windows of the few-slice instance's blocks (row N1): BRO-ELL at h = 32
     // with fewer slices than the general instance keeps resident (148 SMs x 32)
-    if (A->has_ell && o.codec && o.x_stage != 2 && A->h == 32 && A->ell_max_l > bro::kEllTinyCols &&
+    if (A->has_ell && o.codec && o.x_stage == 1 && A->h == 32 && A->ell_max_l > bro::kEllTinyCols &&
         A->s < kB200Warps && (o.ell_kernel == 0 || o.ell_kernel == bro::ELL_FEW) && !A->host_only) {
       const int64_t wpb = A->vsize == 8 ? 8 : 4;  // warps per block of the few-slice instance
       const int64_t E = 16 / A->vsize;            // x elements per 16 bytes

@@ -1,8 +1,6 @@
-OUT=gpurun_out/r02m; mkdir -p $OUT
+OUT=gpurun_out/r02n; mkdir -p $OUT
 python -c "import __graft_entry__ as g; g.build()" > $OUT/build.txt 2>&1 || { tail $OUT/build.txt; exit 1; }
-K="(spmv_random and (tiny or ragged or long or all_empty)) or (instances and float64) or coo_intervals or single_long or inf or empty_matrix or forced or pdl or scatter_matches"
-for tool in memcheck racecheck initcheck; do
-  timeout 1700 compute-sanitizer --tool $tool --error-exitcode 9 --target-processes all \
-    python -m pytest tests/test_gpu_parity.py tests/test_gpu_dist.py -m gpu -q -x -p no:cacheprovider -k "$K" > $OUT/$tool.txt 2>&1
-  echo "$tool rc=$?"; grep -E "ERROR SUMMARY|passed|failed" $OUT/$tool.txt | tail -3
-done
+timeout 900 python -m pytest tests/test_gpu_parity.py -m gpu -q -p no:cacheprovider -x -k "x_window or instances" > $OUT/pytest_q.txt 2>&1; echo "tests rc=$?"; tail -3 $OUT/pytest_q.txt
+for dt in f64 f32; do timeout 600 python scripts/ab.py C2 $dt "x_stage=0" "x_stage=2" > $OUT/ab_C2_$dt.txt 2>&1; cat $OUT/ab_C2_$dt.txt; done
+for dt in f64 f32; do timeout 600 python scripts/ab.py C1 $dt "x_stage=0" "x_stage=2" > $OUT/ab_C1_$dt.txt 2>&1; cat $OUT/ab_C1_$dt.txt; done
+timeout 1500 python scripts/bar_eval.py --gpu --configs 4,2 --out $OUT/bar_eval.json > $OUT/bar_eval.txt 2>&1; cat $OUT/bar_eval.txt | tail -12

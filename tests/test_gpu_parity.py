@@ -439,14 +439,14 @@ def test_x_window_staging(lib, dev, dtype):
         A = A.astype(dtype)
         x = make_x(A.n, 11, dtype)
         Ms, ys = [], []
-        for xs in (0, 2):
+        for xs in (1, 0):
             M, _, y = _run(lib, A, "ell", 1, dtype, dev, x=x, x_stage=xs)
             _check_y(A, x, y, dtype)
             Ms.append(M)
             ys.append(y)
         staged = Ms[0].info["x_stage_bytes"]
         assert Ms[1].info["x_stage_bytes"] == 0
-        if A.name.startswith("C") or A.name == "band20001_300":
+        if dtype == np.float64 and (A.name.startswith("C") or A.name == "band20001_300"):
             assert staged > 0, A.name
         assert np.array_equal(ys[0], ys[1]), A.name
         # misaligned x through the raw C ABI: one element into a padded buffer
