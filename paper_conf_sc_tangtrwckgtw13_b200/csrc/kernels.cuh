@@ -811,13 +811,15 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
     }
     if (ch == 0) {
       lim = int(min(int64_t(I), p.nnz - e0));  // valid entries of the interval
+      // the whole header at once, unconditionally: the words' address must not
+      // wait for the width (width -> symptr -> words would be 3 round trips)
       first = int(p.base_row[i]);              // row of the interval's first entry
       row = first;
       if constexpr (kBro) {
         b = int(p.width[i]);
+        const uint64_t q0 = p.symptr[i];
+        S = int(p.symptr[i + 1] - q0);
         if (b > 0) {  // b = 0: one row for the whole interval, empty stream
-          const uint64_t q0 = p.symptr[i];
-          S = int(p.symptr[i + 1] - q0);
           const uint32_t* wb = p.words + 32 * q0 + lane;  // V = 1: word q of lane l at 32q + l
           if (S <= 2) {
             // short streams (T*b <= 64 bits; C3/C4 intervals have small row
