@@ -108,8 +108,8 @@ typedef struct {
                         (comp_str_i[q*h + tid]); 4 = 16-byte per-lane chunks (128-bit loads);
                         0 (default) = auto: 1 for BRO_FP64, 4 for BRO_FP32. */
   int32_t coo_T;     /* BRO-COO entries per lane of an interval (interval = 32*T entries):
-                        8, 16 or 32; 0 (default) = auto: the largest T for which the COO
-                        part still has >= 4,736 intervals (32 warps x 148 SMs), else 8. */
+                        8, 16 or 32; 0 (default) = 8 (measured fastest on B200 for both
+                        BRO-COO and plain COO: the kernels are latency-bound). */
   int64_t hyb_K;     /* HYB dividing column; -1 = the "less than a third" rule. */
   int32_t codec;     /* 1 = BRO compressed formats; 0 = uncompressed ELL/COO/HYB baseline. */
   int32_t min_bits;  /* 0 = natural widths; k in [1, 31] forces every BRO-ELL width

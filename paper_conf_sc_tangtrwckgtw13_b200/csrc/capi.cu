@@ -171,13 +171,10 @@ bro_status_t check_opts(const bro_opts_t& o) {
   return BRO_OK;
 }
 
-// coo_T = 0: the largest T whose interval count still fills a B200 (32 warps
-// on each of 148 SMs), else the smallest (more, shorter intervals)
-int auto_coo_T(int64_t nnz_coo) {
-  for (int T : {32, 16})
-    if (nnz_coo >= int64_t(32) * T * kB200Warps) return T;
-  return 8;
-}
+// coo_T = 0: T = 8 (256-entry intervals) — measured fastest for BRO-COO and
+// plain COO alike on C3 and C4 (profiles/r02/ab/r02o): both kernels are
+// latency-bound, and shorter intervals give more warps in flight
+int auto_coo_T(int64_t) { return 8; }
 
 void fill_info(bro_matrix_s* A, double secs) {
   bro_info_t& I = A->info;
