@@ -121,10 +121,11 @@ typedef struct {
                         (h = 32), 3 small window (every row stream < 10 symbols), 4 mid
                         window (< 18), 5 general.  An instance the matrix does not fit
                         gives BRO_ERR_ARG.  For A/B measurements and tests. */
-  int32_t pdl;       /* HYB / COO: 0 (default) = 1 = the COO kernel is launched as a
-                        programmatic dependent of the ELL kernel (its loads, decode and x
-                        gathers overlap the ELL kernel's tail; it waits before updating y),
-                        and the fix-up as one of the COO kernel; 2 = plain stream order. */
+  int32_t pdl;       /* HYB: 0 (default) = 1 = the COO kernel is launched as a programmatic
+                        dependent of the ELL kernel (its loads, decode and x gathers
+                        overlap the ELL kernel's tail; it waits before updating y);
+                        2 = plain stream order.  Rows that cross COO intervals are
+                        resolved inside the COO kernel (deterministic look-back). */
   int32_t x_stage;   /* few-slice BRO-ELL instance (h = 32, fewer slices than 148 x 32):
                         1 = each block has the TMA engine copy its x column window
                         (<= 96 KB) into shared memory and gathers from there, when the

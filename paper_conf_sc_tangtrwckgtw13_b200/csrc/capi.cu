@@ -94,13 +94,15 @@ struct bro_matrix_s {
   void* d_cl = nullptr;
   int32_t* d_last_row = nullptr;
   int32_t* d_first_row = nullptr;
+  int32_t* d_flag = nullptr;   // per interval: epoch of the call that published its carries
+  int32_t* d_sync = nullptr;   // {epoch, block ticket} of the COO kernel
   void* d_xs = nullptr;
   void* d_ys = nullptr;
   int64_t device_bytes = 0;
   // kernel instances (index = mode: 0 spmv, 1 scatter, 2 decode)
   Launch ell_k[3];
   Launch coo_k[3];  // 0 spmv, 2 decode
-  Launch fix_k, rep_k;
+  Launch rep_k;
   // x-window staging of the few-slice instance (row N1): per block {first
   // column, columns} of its x window, the staged instance, its shared bytes
   int2* d_xwin = nullptr;
@@ -145,7 +147,7 @@ void free_device(bro_matrix_s* A) {
   void* ps[] = {A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr, A->d_ell_vals, A->d_pell_col,
                 A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr, A->d_coo_row,
                 A->d_coo_col, A->d_coo_vals, A->d_cf, A->d_cl, A->d_last_row, A->d_first_row, A->d_xs, A->d_ys,
-                A->d_xwin};
+                A->d_xwin, A->d_flag, A->d_sync};
   for (void* p : ps)
     if (p) cudaFree(p);
   for (cudaEvent_t e : A->e2e_ev) cudaEventDestroy(e);
@@ -315,7 +317,6 @@ bro_status_t resolve_kernels(bro_matrix_s* A) {
   if (A->has_coo && !st) {
     st = resolve(A->coo_k[0], bro::coo_ref<T>(A->opts.codec == 1, A->coo_T, 0), sms, "COO");
     if (!st) st = resolve(A->coo_k[2], bro::coo_ref<T>(A->opts.codec == 1, A->coo_T, 2), sms, "COO decode");
-    if (!st) st = resolve(A->fix_k, bro::fixup_ref<T>(), sms, "COO fix-up");
   }
   if (!st) st = resolve(A->rep_k, bro::replicate_ref<T>(), sms, "replicate");
   return st;
@@ -481,12 +482,16 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
       } else {
         UP(A->d_coo_row, A->coo.row);
       }
-      // carries of the fix-up: one per work unit (<= max(intervals, warps per block))
-      const size_t nU = size_t(std::max<int64_t>(A->nI, 32));
+      // per-interval carries and their publication flags (decoupled look-back
+      // in the COO kernel); epoch starts at 1, every flag at 0
+      const size_t nU = size_t(A->nI);
       if (st == BRO_OK) st = dev_upload(A, &A->d_cf, nullptr, nU * A->vsize);
       if (st == BRO_OK) st = dev_upload(A, &A->d_cl, nullptr, nU * A->vsize);
       if (st == BRO_OK) st = dev_upload(A, &A->d_last_row, nullptr, nU * 4);
       if (st == BRO_OK) st = dev_upload(A, &A->d_first_row, nullptr, nU * 4);
+      std::vector<int32_t> zeros(nU, 0), sync0{1, 0};
+      UP(A->d_flag, zeros);
+      UP(A->d_sync, sync0);
     }
 #undef UP
     if (st == BRO_OK) st = dtype == BRO_FP64 ? resolve_kernels<double>(A) : resolve_kernels<float>(A);
@@ -610,7 +615,8 @@ template <typename T>
 bro::dev::CooDev<T> coo_dev(const bro_matrix_s* A, const T* x) {
   return bro::dev::CooDev<T>{A->nnz_coo, A->nI, A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr,
                             A->d_coo_row, A->d_coo_col, static_cast<const T*>(A->d_coo_vals), x,
-                            static_cast<T*>(A->d_cf), static_cast<T*>(A->d_cl), A->d_first_row, A->d_last_row};
+                            static_cast<T*>(A->d_cf), static_cast<T*>(A->d_cl), A->d_first_row, A->d_last_row,
+                            A->d_flag, A->d_sync};
 }
 
 int64_t coo_grid(const bro_matrix_s* A, const Launch& L) {
@@ -621,7 +627,7 @@ int64_t coo_grid(const bro_matrix_s* A, const Launch& L) {
 // y = A.x stored into every destination of yo (yo.p[0] = the local y on A's
 // device).  ELL-only handles store all destinations from the ELL kernel's
 // epilogue (fused exchange); handles with a COO part finish y locally and
-// then replicate it (the COO part and the fix-up add into y).
+// then replicate it (the COO part adds into y).
 template <typename T>
 bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& yo, cudaStream_t st) {
   T* y = yo.p[0];
@@ -637,21 +643,11 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
   if (e == cudaSuccess && A->has_coo && A->nI > 0) {
     bro::dev::CooDev<T> p = coo_dev<T>(A, x);
     int32_t* none = nullptr;
-    // the COO kernel overlaps the ELL kernel's tail, the fix-up the COO
-    // kernel's (programmatic dependent launches, bro_opts_t.pdl)
-    const bool pdl = A->opts.pdl != 2;
-    const bool after_ell = A->has_ell && pdl;
+    // the COO kernel overlaps the ELL kernel's tail (programmatic dependent
+    // launch, bro_opts_t.pdl); rows crossing intervals are resolved inside it
+    const bool after_ell = A->has_ell && A->opts.pdl != 2;
     e = after_ell ? launch_pdl(A->coo_k[0], coo_grid(A, A->coo_k[0]), st, p, y, none)
                   : launch(A->coo_k[0], coo_grid(A, A->coo_k[0]), st, p, y, none);
-    if (e == cudaSuccess) {
-      int64_t nU = A->nI;
-      const int32_t* fr = A->d_first_row;
-      const int32_t* lr = A->d_last_row;
-      const T* cf = static_cast<const T*>(A->d_cf);
-      const T* cl = static_cast<const T*>(A->d_cl);
-      e = pdl ? launch_pdl(A->fix_k, (nU + 255) / 256, st, nU, fr, lr, cf, cl, y)
-              : launch(A->fix_k, (nU + 255) / 256, st, nU, fr, lr, cf, cl, y);
-    }
   }
   if (e == cudaSuccess && !fused && A->m > 0 && multi) {
     int64_t m = A->m;

@@ -21,9 +21,10 @@
 //     decodes its deltas from a staged window, one warp scan of the lane
 //     totals gives every lane its start row, the lane reduces its entries
 //     sequentially and ONE warp segmented scan per interval links segments
-//     that cross lanes (the "parallel scan primitive" of P:L343); a
-//     deterministic fix-up kernel adds the partials of rows crossing
-//     intervals (the "extra kernel invocation for data reduction").
+//     that cross lanes (the "parallel scan primitive" of P:L343); rows that
+//     cross intervals are resolved in the same kernel by a deterministic
+//     decoupled look-back (the paper's "extra kernel invocation for data
+//     reduction" becomes a single pass).
 //   * Uncompressed baselines: ell_spmv (thread per row, column-major
 //     ELLPACK) and coo_spmv<kBro=false> (same traversal, explicit rows).
 //   * Every kernel takes a Mode: kSpmv (y = A.x), kScatter (y also stored
@@ -230,7 +231,18 @@ struct CooDev {           // (BRO-)COO part
   T* cl;                  // per interval: partial of its last row
   int32_t* first_row;
   int32_t* last_row;
+  int32_t* flag;          // per interval: epoch of the call that published the four above
+  int32_t* sync;          // [0] epoch of the current call, [1] block ticket
 };
+
+__device__ __forceinline__ void st_release(int32_t* p, int32_t v) {
+  asm volatile("st.release.gpu.global.s32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ int32_t ld_acquire(const int32_t* p) {
+  int32_t v;
+  asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
 
 // Programmatic dependent launch (PDL): a kernel launched with the
 // programmatic-serialization attribute may start while the previous kernel
@@ -765,18 +777,13 @@ __device__ __forceinline__ void cp_async4(uint32_t* dst, const uint32_t* src) {
                "l"(src) : "memory");
 }
 
-template <typename T, bool kBro, int TT, int kWarps, int kMinBlocks, int kMode>
-__global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
-coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
+// One interval of the (BRO-)COO kernel (warp i).
+template <typename T, bool kBro, int TT, int kWarps, int kMode>
+__device__ __forceinline__ void coo_interval(const CooDev<T>& p, T* __restrict__ y, int32_t* __restrict__ dec,
+                                             int64_t i, int32_t epoch, uint32_t* cw, int lane) {
   constexpr int I = 32 * TT;
   constexpr int CH = TT < 16 ? TT : 16;  // entries per lane loaded at once (one chunk)
   constexpr int NC = TT / CH;
-  __shared__ uint32_t cwin[kWarps][kBro ? (TT + 1) * 32 : 1];  // <= T symbol rows + a zero guard row
-  const int lane = threadIdx.x & 31;
-  const int w = threadIdx.x >> 5;
-  const int64_t i = int64_t(blockIdx.x) * kWarps + w;
-  if constexpr (kMode != kDecode) pdl_launch_dependents();  // the fix-up may be scheduled
-  if (i >= p.nI) return;
   const int64_t e0 = i * I;
   const int32_t* cb = p.col + e0;
   const T* vb = p.vals + e0;
@@ -787,7 +794,7 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   bool one = true;
   int b = 0, S = 0, row = 0, first = 0, lim = 0;
   uint32_t w0 = 0, w1 = 0;
-  const uint32_t* wl = cwin[w] + lane;
+  const uint32_t* wl = cw + lane;
 #pragma unroll
   for (int ch = 0; ch < NC; ++ch) {
     // the chunk's col / vals (and plain rows) first: nothing they need
@@ -827,7 +834,7 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
             w0 = ld_stream_u32(wb);
             w1 = S > 1 ? ld_stream_u32(wb + 32) : 0u;
           } else {  // the lane words -> [q][lane] window by cp.async
-            uint32_t* win = cwin[w] + lane;
+            uint32_t* win = cw + lane;
             for (int q = 0; q < S; ++q) cp_async4(win + 32 * q, wb + 32 * q);
             asm volatile("cp.async.commit_group;" ::: "memory");
             win[32 * S] = 0u;
@@ -930,24 +937,94 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   }
   T cin = __shfl_up_sync(0xffffffffu, co, 1);
   if (!link) cin = T(0);
+  // complete segments of rows other than the interval's first go straight to
+  // y (each such row lives in this interval alone, or is its last row and
+  // ends here); the first row's partial is collected for the carry logic
+  T fpart = T(0);
+  bool hasF = false;
   auto emit = [&](int rr, T val) {
-    if (rr == first) p.cf[i] = val;
+    if (rr == first) { fpart = val; hasF = true; }
     else atomicAdd(y + rr, val);
   };
   if (!one) emit(f, A + cin);  // first segment complete inside this lane
   const int fnext = __shfl_down_sync(0xffffffffu, f, 1);
   if (lane < 31 && fnext != L) emit(L, co);  // trailing segment complete at this lane
-  if (lane == 31) {  // the interval's last row: its partial is carried
+  // Rows that cross intervals, resolved in this kernel (decoupled look-back,
+  // deterministic): interval i publishes the partials of its first row F and
+  // last row L with a flag tagged by the call's epoch; the interval holding
+  // the END of a row that began earlier (its owner) looks back, sums the
+  // row's partials in a fixed order and adds them to y once.  Whether a row
+  // continues into interval i+1 is static: base_row[i+1].
+  const int Lw = __shfl_sync(0xffffffffu, L, 31);
+  const T co31 = __shfl_sync(0xffffffffu, co, 31);
+  const unsigned mF = __ballot_sync(0xffffffffu, hasF);
+  T Fp = mF ? __shfl_sync(0xffffffffu, fpart, __ffs(mF) - 1) : co31;  // L == F: the whole interval
+  const int nf = i + 1 < p.nI ? int(p.base_row[i + 1]) : -1;  // first row of interval i+1
+  if (lane == 31) {  // publish
     p.first_row[i] = first;
-    p.last_row[i] = L;
-    if (L == first) {
-      p.cf[i] = co;
-      p.cl[i] = T(0);
-    } else {
-      p.cl[i] = co;
+    p.last_row[i] = Lw;
+    p.cf[i] = Fp;
+    p.cl[i] = Lw != first ? co31 : T(0);
+    st_release(p.flag + i, epoch);
+  }
+  if (Lw != first && Lw != nf && lane == 31) atomicAdd(y + Lw, co31);  // L starts and ends here
+  const bool f_owner = Lw != first || first != nf;  // F ends in this interval
+  if (f_owner) {
+    // look back over intervals i-1, i-2, ...: lane k examines j = jb - k;
+    // j holds F iff its last row is F; j contributes cf[j] if it is all F
+    // (and the walk goes on), cl[j] if F starts in j (the walk stops)
+    T sum = Fp;
+    for (int64_t jb = i - 1;; jb -= 32) {
+      const int64_t j = jb - lane;
+      bool holds = false, stop = true;
+      T c = T(0);
+      if (j >= 0) {
+        while (ld_acquire(p.flag + j) != epoch) __nanosleep(32);
+        const int lj = p.last_row[j];
+        holds = lj == first;
+        if (holds) {
+          const int fj = p.first_row[j];
+          stop = fj != first;
+          c = stop ? p.cl[j] : p.cf[j];
+        }
+      }
+      const unsigned ms = __ballot_sync(0xffffffffu, stop);
+      const int k0 = ms ? __ffs(ms) - 1 : 32;  // first lane that ends the walk
+      if (!(lane < k0 || (lane == k0 && holds))) c = T(0);
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) c += __shfl_xor_sync(0xffffffffu, c, off);  // fixed tree
+      sum += c;
+      if (ms) break;
+    }
+    if (lane == 0) atomicAdd(y + first, sum);
+  }
+}
+template <typename T, bool kBro, int TT, int kWarps, int kMinBlocks, int kMode>
+__global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
+coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
+  __shared__ uint32_t cwin[kWarps][kBro ? (TT + 1) * 32 : 1];  // <= T symbol rows + a zero guard row
+  const int lane = threadIdx.x & 31;
+  const int w = threadIdx.x >> 5;
+  const int64_t i = int64_t(blockIdx.x) * kWarps + w;
+  if constexpr (kMode == kDecode) {
+    if (i >= p.nI) return;
+    coo_interval<T, kBro, TT, kWarps, kMode>(p, y, dec, i, 0, cwin[w], lane);
+  } else {
+    const int32_t epoch = *reinterpret_cast<volatile int32_t*>(p.sync);  // this call's epoch
+    if (i < p.nI) coo_interval<T, kBro, TT, kWarps, kMode>(p, y, dec, i, epoch, cwin[w], lane);
+    // the last block to finish advances the epoch for the next call
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      if (atomicAdd(p.sync + 1, 1) == int(gridDim.x) - 1) {
+        p.sync[1] = 0;
+        __threadfence();
+        atomicExch(p.sync, epoch + 1);
+      }
     }
   }
 }
+
 
 // Exchange of a finished y for formats whose last kernel is not an ELL
 // kernel (COO / HYB: the COO part and the fix-up add into y after the ELL
@@ -967,64 +1044,6 @@ __global__ void replicate_y(int64_t m, const YOut<T> o) {
         if (k < o.n) o.p[k][i] = v;
     }
   }
-}
-
-// Deterministic application of the intervals' carries (one thread per
-// interval, fixed summation order = interval order).  first[u] / last[u] =
-// rows of the interval's first and last entries; cf = partial of the first
-// row (the whole interval if first == last), cl = partial of the last row.
-// acc += cf[j] for the intervals j = i+1, i+2, ... that continue row R
-// (first[j] == R), stopping after the first of them that ends on another
-// row.  Intervals are read 8 at a time (one round trip for rows spanning up
-// to 9 intervals); the additions stay in interval order.
-template <typename T>
-__device__ __forceinline__ T chain_sum(int64_t i, int64_t nU, int R, T acc, const int32_t* __restrict__ first,
-                                       const int32_t* __restrict__ last_row, const T* __restrict__ cf) {
-  constexpr int B = 8;
-  for (int64_t j0 = i + 1; j0 < nU; j0 += B) {
-    int fj[B], lj[B];
-    T cj[B];
-#pragma unroll
-    for (int k = 0; k < B; ++k) {
-      const bool in = j0 + k < nU;
-      fj[k] = in ? first[j0 + k] : -1;
-      lj[k] = in ? last_row[j0 + k] : -1;
-      cj[k] = in ? cf[j0 + k] : T(0);
-    }
-    bool done = false;
-#pragma unroll
-    for (int k = 0; k < B; ++k) {
-      if (!done) {
-        if (fj[k] < 0) {
-          // an empty unit holds no row: skip it
-        } else if (fj[k] != R) {
-          done = true;
-        } else {
-          acc += cj[k];
-          done = lj[k] != R;
-        }
-      }
-    }
-    if (done) break;
-  }
-  return acc;
-}
-
-template <typename T>
-__global__ void coo_fixup(int64_t nU, const int32_t* __restrict__ first, const int32_t* __restrict__ last_row,
-                          const T* __restrict__ cf, const T* __restrict__ cl, T* __restrict__ y) {
-  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
-  pdl_wait();  // the carries come from the COO kernel
-  if (i >= nU) return;
-  const int F = first[i];
-  const int L = last_row[i];
-  if (F < 0) return;  // an empty unit
-  if (L != F)  // unit i is the first one holding row L
-    y[L] += chain_sum<T>(i, nU, L, cl[i], first, last_row, cf);
-  int64_t j = i - 1;  // the previous non-empty unit
-  while (j >= 0 && first[j] < 0) --j;
-  if (j < 0 || last_row[j] != F)  // unit i is the first one holding row F
-    y[F] += L == F ? chain_sum<T>(i, nU, F, cf[i], first, last_row, cf) : cf[i];
 }
 
 }  // namespace dev

@@ -1,7 +1,10 @@
-OUT=gpurun_out/r02o; mkdir -p $OUT
-python -c "import __graft_entry__ as g; g.build()" > $OUT/build.txt 2>&1 || { tail $OUT/build.txt; exit 1; }
-timeout 900 python -m pytest tests/test_gpu_parity.py -m gpu -q -p no:cacheprovider -x -k "coo_intervals or pdl or x_window" > $OUT/pytest_q.txt 2>&1; echo "tests rc=$?"; tail -2 $OUT/pytest_q.txt
-for dt in f64 f32; do for T in 8 16 32; do timeout 600 python scripts/ab.py C4 $dt --format coo "coo_T=$T" --baseline-opts "coo_T=$T" > $OUT/ab_C4_coo_${dt}_T$T.txt 2>&1; tail -1 $OUT/ab_C4_coo_${dt}_T$T.txt | cut -c1-110; done; done
-for dt in f64 f32; do for T in 8 16 32; do timeout 600 python scripts/ab.py C3 $dt --format coo "coo_T=$T" --baseline-opts "coo_T=$T" > $OUT/ab_C3_coo_${dt}_T$T.txt 2>&1; tail -1 $OUT/ab_C3_coo_${dt}_T$T.txt | cut -c1-110; head -1 $OUT/ab_C3_coo_${dt}_T$T.txt | cut -c1-60; done; done
-for dt in f64 f32; do timeout 600 python scripts/ab.py C4 $dt "coo_T=8" "coo_T=16" "coo_T=32" --baseline-opts "coo_T=8" > $OUT/ab_C4_hyb_$dt.txt 2>&1; cat $OUT/ab_C4_hyb_$dt.txt | cut -c1-130; done
-for dt in f64 f32; do timeout 600 python scripts/ab.py C3 $dt "coo_T=8" "coo_T=16" --baseline-opts "coo_T=8" > $OUT/ab_C3_hyb_$dt.txt 2>&1; cat $OUT/ab_C3_hyb_$dt.txt | cut -c1-130; done
+OUT=gpurun_out/r02p; mkdir -p $OUT
+bash scripts/gpu_r02.sh r02p tests smoke bench benchall launches
+for wl in C3 C4; do for dt in f64 f32; do
+  fl=""; [ $wl = C3 ] && fl="--flush-l2"
+  timeout 600 python bench.py --workload $wl --dtype $dt --format coo --steps 500 --no-cpu-baseline --no-e2e $fl > $OUT/bench_${wl}_${dt}_coo.json 2>> $OUT/benchcoo.err; echo "$wl $dt coo rc=$?"
+done; done
+for wl in C3 C4; do
+  timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 30 --csv --log-file $OUT/launches_$wl.csv python scripts/prof_one.py $wl f64 --launches 10 > /dev/null 2>&1; python scripts/launch_summary.py $OUT/launches_$wl.csv
+done
+timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29533 bench.py --gpus 2 --steps 50 --warmup 5 --workload C2 --dist-backend gloo --no-e2e > $OUT/bench_gloo2_C2.json 2> $OUT/bench_gloo2.err; echo "gloo2 rc=$?"; cut -c1-600 $OUT/bench_gloo2_C2.json

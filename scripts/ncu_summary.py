@@ -9,7 +9,7 @@ def run(*a):
     return subprocess.run(["ncu", "-i", rep, *a], capture_output=True, text=True).stdout
 
 raw = list(csv.reader(io.StringIO(run("--page", "raw", "--csv"))))
-hdr, units, vals = raw[0], raw[1], raw[2]
+hdr, units = raw[0], raw[1]
 want = ["Kernel Name", "gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
         "dram__throughput.avg.pct_of_peak_sustained_elapsed", "launch__registers_per_thread",
         "launch__grid_size", "launch__block_size", "sm__warps_active.avg.pct_of_peak_sustained_active",
@@ -17,12 +17,13 @@ want = ["Kernel Name", "gpu__time_duration.sum", "dram__bytes_read.sum", "dram__
         "l1tex__t_sector_hit_rate.pct", "smsp__issue_active.avg.pct_of_peak_sustained_active",
         "lts__t_bytes.sum", "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum",
         "launch__shared_mem_per_block_dynamic"]
-for w in want:
+for vals in raw[2:]:  # one row per captured kernel launch
+  for w in want:
     if w in hdr:
         i = hdr.index(w)
         print(f"{w:60s} {vals[i]} {units[i]}")
-stalls = []
-for i, h in enumerate(hdr):
+  stalls = []
+  for i, h in enumerate(hdr):
     if h.startswith("smsp__average_warp_latency_issue_stalled_") and h.endswith(".ratio"):
         try:
             stalls.append((float(vals[i].replace(",", "")), h[len("smsp__average_warp_latency_issue_stalled_"):]))
@@ -33,15 +34,22 @@ for i, h in enumerate(hdr):
             stalls.append((float(vals[i].replace(",", "")), h[len("smsp__average_warps_issue_stalled_"):]))
         except ValueError:
             pass
-print("stalls (warps per issue):", ", ".join(f"{n}={v:.2f}" for v, n in sorted(stalls, reverse=True)[:10]))
+  print("stalls (warps per issue):", ", ".join(f"{n}={v:.2f}" for v, n in sorted(stalls, reverse=True)[:10]))
+  print()
 src = list(csv.reader(io.StringIO(run("--page", "source", "--csv", "--print-source", "sass"))))
 if len(src) > 2:
     h = src[1]
     ix = {k: j for j, k in enumerate(h)}
     rows = src[2:]
     key = "Warp Stall Sampling (All Samples)"
-    tot = sum(int(r[ix[key]] or 0) for r in rows)
+    def n(r):
+        try:
+            return int(r[ix[key]] or 0)
+        except ValueError:
+            return 0
+    rows = [r for r in rows if len(r) > ix[key]]
+    tot = sum(n(r) for r in rows)
     print(f"SASS instructions: {len(rows)}, stall samples: {tot}")
-    for r in sorted(rows, key=lambda r: -int(r[ix[key]] or 0))[:topn]:
-        print(f"  {r[ix['Address']][-5:]} {r[ix['Source']][:60]:60s} {int(r[ix[key]] or 0):6d} "
+    for r in sorted(rows, key=lambda r: -n(r))[:topn]:
+        print(f"  {r[ix['Address']][-5:]} {r[ix['Source']][:60]:60s} {n(r):6d} "
               f"exec={r[ix['Instructions Executed']]}")
