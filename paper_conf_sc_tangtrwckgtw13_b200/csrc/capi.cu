@@ -95,7 +95,7 @@ struct bro_matrix_s {
   int32_t* d_last_row = nullptr;
   int32_t* d_first_row = nullptr;
   int32_t* d_flag = nullptr;   // per interval: epoch of the call that published its carries
-  int32_t* d_sync = nullptr;   // {epoch, block ticket} of the COO kernel
+  int32_t* d_sync = nullptr;   // {epoch, finish ticket, start ticket} of the COO kernel
   void* d_xs = nullptr;
   void* d_ys = nullptr;
   int64_t device_bytes = 0;
@@ -489,7 +489,7 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
       if (st == BRO_OK) st = dev_upload(A, &A->d_cl, nullptr, nU * A->vsize);
       if (st == BRO_OK) st = dev_upload(A, &A->d_last_row, nullptr, nU * 4);
       if (st == BRO_OK) st = dev_upload(A, &A->d_first_row, nullptr, nU * 4);
-      std::vector<int32_t> zeros(nU, 0), sync0{1, 0};
+      std::vector<int32_t> zeros(nU, 0), sync0{1, 0, 0};
       UP(A->d_flag, zeros);
       UP(A->d_sync, sync0);
     }

@@ -232,7 +232,7 @@ struct CooDev {           // (BRO-)COO part
   int32_t* first_row;
   int32_t* last_row;
   int32_t* flag;          // per interval: epoch of the call that published the four above
-  int32_t* sync;          // [0] epoch of the current call, [1] block ticket
+  int32_t* sync;          // [0] epoch of the current call, [1] finish ticket, [2] start ticket
 };
 
 __device__ __forceinline__ void st_release(int32_t* p, int32_t v) {
@@ -1005,26 +1005,33 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   __shared__ uint32_t cwin[kWarps][kBro ? (TT + 1) * 32 : 1];  // <= T symbol rows + a zero guard row
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
-  const int64_t i = int64_t(blockIdx.x) * kWarps + w;
   if constexpr (kMode == kDecode) {
+    const int64_t i = int64_t(blockIdx.x) * kWarps + w;
     if (i >= p.nI) return;
     coo_interval<T, kBro, TT, kWarps, kMode>(p, y, dec, i, 0, cwin[w], lane);
   } else {
+    // the block's intervals come from a start ticket, not blockIdx: every
+    // interval an owner looks back at belongs to a block that has started
+    // (no dependence on the hardware's block dispatch order)
+    __shared__ int64_t tile;
+    if (threadIdx.x == 0) tile = atomicAdd(p.sync + 2, 1);
+    __syncthreads();
+    const int64_t i = tile * kWarps + w;
     const int32_t epoch = *reinterpret_cast<volatile int32_t*>(p.sync);  // this call's epoch
     if (i < p.nI) coo_interval<T, kBro, TT, kWarps, kMode>(p, y, dec, i, epoch, cwin[w], lane);
-    // the last block to finish advances the epoch for the next call
+    // the last block to finish resets the tickets and advances the epoch
     __syncthreads();
     if (threadIdx.x == 0) {
       __threadfence();
       if (atomicAdd(p.sync + 1, 1) == int(gridDim.x) - 1) {
         p.sync[1] = 0;
+        p.sync[2] = 0;
         __threadfence();
         atomicExch(p.sync, epoch + 1);
       }
     }
   }
 }
-
 
 // Exchange of a finished y for formats whose last kernel is not an ELL
 // kernel (COO / HYB: the COO part and the fix-up add into y after the ELL
