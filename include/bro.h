@@ -48,7 +48,8 @@
  *   BRO-COO, intervals of 32*T entries (T = 8, 16 or 32): lane l of interval
  *     i owns the T consecutive entries e = i*32*T + T*l + t (DESIGN.md
  *     reading R13); deltas follow entry order, delta(e) = row(e) - row(e-1),
- *     delta of the first entry 0, base_row[i] = row of the first entry, one
+ *     delta of the first entry 0, base_row[i] = row of the first entry,
+ *     end_row[i] = row of the last entry (reading R28), one
  *     width width[i] per interval; lane l's T fields, MSB first,
  *     padded to S_i = ceil(T*width/32) symbols at
  *     coo_words[32*coo_symptr[i] + 32*q + l] (the paper's V = 1 multiplexing,
@@ -178,7 +179,8 @@ typedef enum {
   BRO_PART_COO_VALS = 10,     /* value[nI*32*T]  same arrangement, 0 past nnz */
   BRO_PART_COO_ROW = 11,      /* int32[nI*32*T]  plain COO rows (codec 0), last row past nnz */
   BRO_PART_PELL_COL = 12,     /* int32[K*pitch]  plain ELL, column-major, -1 = padding (codec 0) */
-  BRO_PART_PELL_VALS = 13     /* value[K*pitch]  plain ELL values (codec 0) */
+  BRO_PART_PELL_VALS = 13,    /* value[K*pitch]  plain ELL values (codec 0) */
+  BRO_PART_COO_END_ROW = 14   /* uint32[nI]      row of each interval's last entry (BRO and plain COO) */
 } bro_part_t;
 
 /* Fill *opts with the defaults: h 0 (auto), sym 32, V 0 (auto), T 0 (auto),

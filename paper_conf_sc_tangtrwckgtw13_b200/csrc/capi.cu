@@ -85,16 +85,14 @@ struct bro_matrix_s {
   int32_t* d_pell_col = nullptr;
   uint32_t* d_coo_words = nullptr;
   uint32_t* d_coo_base = nullptr;
+  uint32_t* d_coo_end = nullptr;
   uint8_t* d_coo_width = nullptr;
   uint64_t* d_coo_symptr = nullptr;
   int32_t* d_coo_row = nullptr;
   int32_t* d_coo_col = nullptr;
   void* d_coo_vals = nullptr;
-  void* d_cf = nullptr;
-  void* d_cl = nullptr;
-  int32_t* d_last_row = nullptr;
-  int32_t* d_first_row = nullptr;
-  int32_t* d_flag = nullptr;   // per interval: epoch of the call that published its carries
+  void* d_cy = nullptr;        // per interval: partial of its last row when that row continues
+  int32_t* d_flag = nullptr;   // per interval: epoch of the call that published its carry
   int32_t* d_sync = nullptr;   // {epoch, finish ticket, start ticket} of the COO kernel
   void* d_xs = nullptr;
   void* d_ys = nullptr;
@@ -146,8 +144,8 @@ void free_device(bro_matrix_s* A) {
   DeviceGuard g(A->device);
   void* ps[] = {A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr, A->d_ell_vals, A->d_pell_col,
                 A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr, A->d_coo_row,
-                A->d_coo_col, A->d_coo_vals, A->d_cf, A->d_cl, A->d_last_row, A->d_first_row, A->d_xs, A->d_ys,
-                A->d_xwin, A->d_flag, A->d_sync};
+                A->d_coo_col, A->d_coo_vals, A->d_cy, A->d_xs, A->d_ys, A->d_xwin, A->d_flag, A->d_sync,
+                A->d_coo_end};
   for (void* p : ps)
     if (p) cudaFree(p);
   for (cudaEvent_t e : A->e2e_ev) cudaEventDestroy(e);
@@ -208,11 +206,11 @@ void fill_info(bro_matrix_s* A, double secs) {
     if (A->opts.codec) {
       I.coo_stream_bytes = 4 * A->coo_words;
       stream += I.coo_stream_bytes;
-      meta += A->nI * (4 + 1) + 8 * (A->nI + 1);  // base_row, width, symptr
+      meta += A->nI * (4 + 4 + 1) + 8 * (A->nI + 1);  // base_row, end_row, width, symptr
       raw_index += 4 * slots;                     // col
     } else {
       raw_index += 8 * slots;                     // row + col
-      meta += 4 * A->nI;                          // interval first rows
+      meta += 8 * A->nI;                          // interval first and last rows
     }
     values += slots * vs;
   }
@@ -473,6 +471,7 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
     }
     if (A->has_coo) {
       UP(A->d_coo_base, A->coo.base_row);
+      UP(A->d_coo_end, A->coo.end_row);
       UP(A->d_coo_col, A->coo.col);
       if (st == BRO_OK) st = dev_upload(A, &A->d_coo_vals, A->coo.vals.data(), A->coo.vals.size());
       if (o.codec) {
@@ -482,13 +481,10 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
       } else {
         UP(A->d_coo_row, A->coo.row);
       }
-      // per-interval carries and their publication flags (decoupled look-back
-      // in the COO kernel); epoch starts at 1, every flag at 0
+      // per-interval carries and their publication flags (look-back in the
+      // COO kernel); epoch starts at 1, every flag at 0
       const size_t nU = size_t(A->nI);
-      if (st == BRO_OK) st = dev_upload(A, &A->d_cf, nullptr, nU * A->vsize);
-      if (st == BRO_OK) st = dev_upload(A, &A->d_cl, nullptr, nU * A->vsize);
-      if (st == BRO_OK) st = dev_upload(A, &A->d_last_row, nullptr, nU * 4);
-      if (st == BRO_OK) st = dev_upload(A, &A->d_first_row, nullptr, nU * 4);
+      if (st == BRO_OK) st = dev_upload(A, &A->d_cy, nullptr, nU * A->vsize);
       std::vector<int32_t> zeros(nU, 0), sync0{1, 0, 0};
       UP(A->d_flag, zeros);
       UP(A->d_sync, sync0);
@@ -615,8 +611,7 @@ template <typename T>
 bro::dev::CooDev<T> coo_dev(const bro_matrix_s* A, const T* x) {
   return bro::dev::CooDev<T>{A->nnz_coo, A->nI, A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr,
                             A->d_coo_row, A->d_coo_col, static_cast<const T*>(A->d_coo_vals), x,
-                            static_cast<T*>(A->d_cf), static_cast<T*>(A->d_cl), A->d_first_row, A->d_last_row,
-                            A->d_flag, A->d_sync};
+                            A->d_coo_end, static_cast<T*>(A->d_cy), A->d_flag, A->d_sync};
 }
 
 int64_t coo_grid(const bro_matrix_s* A, const Launch& L) {
@@ -683,6 +678,7 @@ PartView part_view(bro_matrix_s* A, int32_t part) {
     case BRO_PART_ELL_VALS: if (bro_ell) set(A->ell.vals.data(), A->d_ell_vals, vs * size_t(A->ell_slots)); break;
     case BRO_PART_COO_WORDS: if (bro_coo) set(A->coo.words.data(), A->d_coo_words, 4 * size_t(A->coo_words)); break;
     case BRO_PART_COO_BASE_ROW: if (bro_coo) set(A->coo.base_row.data(), A->d_coo_base, 4 * size_t(A->nI)); break;
+    case BRO_PART_COO_END_ROW: if (coo) set(A->coo.end_row.data(), A->d_coo_end, 4 * size_t(A->nI)); break;
     case BRO_PART_COO_WIDTH: if (bro_coo) set(A->coo.width.data(), A->d_coo_width, size_t(A->nI)); break;
     case BRO_PART_COO_SYMPTR: if (bro_coo) set(A->coo.symptr.data(), A->d_coo_symptr, 8 * size_t(A->nI + 1)); break;
     case BRO_PART_COO_COL: if (coo) set(A->coo.col.data(), A->d_coo_col, 4 * slots); break;

@@ -227,11 +227,9 @@ struct CooDev {           // (BRO-)COO part
   const int32_t* col;
   const T* vals;
   const T* x;
-  T* cf;                  // per interval: partial of its first row
-  T* cl;                  // per interval: partial of its last row
-  int32_t* first_row;
-  int32_t* last_row;
-  int32_t* flag;          // per interval: epoch of the call that published the four above
+  const uint32_t* end_row; // per interval: row of its last entry (static, reading R28)
+  T* cy;                  // per interval: partial of its last row, when that row continues
+  int32_t* flag;          // per interval: epoch of the call that published cy
   int32_t* sync;          // [0] epoch of the current call, [1] finish ticket, [2] start ticket
 };
 
@@ -949,56 +947,56 @@ __device__ __forceinline__ void coo_interval(const CooDev<T>& p, T* __restrict__
   if (!one) emit(f, A + cin);  // first segment complete inside this lane
   const int fnext = __shfl_down_sync(0xffffffffu, f, 1);
   if (lane < 31 && fnext != L) emit(L, co);  // trailing segment complete at this lane
-  // Rows that cross intervals, resolved in this kernel (decoupled look-back,
-  // deterministic): interval i publishes the partials of its first row F and
-  // last row L with a flag tagged by the call's epoch; the interval holding
-  // the END of a row that began earlier (its owner) looks back, sums the
-  // row's partials in a fixed order and adds them to y once.  Whether a row
-  // continues into interval i+1 is static: base_row[i+1].
-  const int Lw = __shfl_sync(0xffffffffu, L, 31);
+  // Rows that cross intervals, resolved in this kernel (look-back,
+  // deterministic).  Which rows cross is static: interval j's first row is
+  // base_row[j] and its last row end_row[j] (reading R28).  A row R that
+  // spans intervals a..b is added to y once, by its owner b (the interval
+  // where it ends), as its partial in b plus the partials the intervals a..b-1
+  // published (cy[j], the partial of j's last row) in a fixed order; every
+  // other row of the interval is complete here and gets one direct add.
+  const int Lw = __shfl_sync(0xffffffffu, L, 31);  // == end_row[i]
   const T co31 = __shfl_sync(0xffffffffu, co, 31);
   const unsigned mF = __ballot_sync(0xffffffffu, hasF);
-  T Fp = mF ? __shfl_sync(0xffffffffu, fpart, __ffs(mF) - 1) : co31;  // L == F: the whole interval
-  const int nf = i + 1 < p.nI ? int(p.base_row[i + 1]) : -1;  // first row of interval i+1
-  if (lane == 31) {  // publish
-    p.first_row[i] = first;
-    p.last_row[i] = Lw;
-    p.cf[i] = Fp;
-    p.cl[i] = Lw != first ? co31 : T(0);
-    st_release(p.flag + i, epoch);
+  const T Fp = mF ? __shfl_sync(0xffffffffu, fpart, __ffs(mF) - 1) : co31;  // L == F: the whole interval
+  const bool last_continues = i + 1 < p.nI && int(p.base_row[i + 1]) == Lw;
+  const bool first_continued = i > 0 && int(p.end_row[i - 1]) == first;
+  if (last_continues) {  // publish the partial of the last row for its owner
+    if (lane == 31) {
+      p.cy[i] = Lw == first ? Fp : co31;
+      st_release(p.flag + i, epoch);
+    }
+  } else if (Lw != first && lane == 31) {
+    atomicAdd(y + Lw, co31);  // the last row starts and ends here
   }
-  if (Lw != first && Lw != nf && lane == 31) atomicAdd(y + Lw, co31);  // L starts and ends here
-  const bool f_owner = Lw != first || first != nf;  // F ends in this interval
-  if (f_owner) {
-    // look back over intervals i-1, i-2, ...: lane k examines j = jb - k;
-    // j holds F iff its last row is F; j contributes cf[j] if it is all F
-    // (and the walk goes on), cl[j] if F starts in j (the walk stops)
+  if (Lw != first || !last_continues) {  // this interval owns its first row F
     T sum = Fp;
-    for (int64_t jb = i - 1;; jb -= 32) {
-      const int64_t j = jb - lane;
-      bool holds = false, stop = true;
-      T c = T(0);
-      if (j >= 0) {
-        while (ld_acquire(p.flag + j) != epoch) __nanosleep(32);
-        const int lj = p.last_row[j];
-        holds = lj == first;
-        if (holds) {
-          const int fj = p.first_row[j];
-          stop = fj != first;
-          c = stop ? p.cl[j] : p.cf[j];
+    if (first_continued) {
+      // intervals i-1, i-2, ... hold F (end_row == F); all of those whose
+      // first row is F too continue the walk, the one where F starts ends it.
+      // Lane k examines j = jb - k; the flags waited for are exactly those of
+      // intervals holding F.
+      for (int64_t jb = i - 1;; jb -= 32) {
+        const int64_t j = jb - lane;
+        const bool whole = j >= 0 && int(p.base_row[j]) == first;  // j is all F
+        const unsigned mw = __ballot_sync(0xffffffffu, whole);
+        const int k0 = ~mw ? __ffs(~mw) - 1 : 32;  // first lane not all F
+        // lanes < k0 are all-F intervals; lane k0 holds F iff its last row is F
+        const bool needed = lane < k0 || (lane == k0 && j >= 0 && int(p.end_row[j]) == first);
+        T c = T(0);
+        if (needed) {
+          while (ld_acquire(p.flag + j) != epoch) __nanosleep(20);
+          c = p.cy[j];
         }
-      }
-      const unsigned ms = __ballot_sync(0xffffffffu, stop);
-      const int k0 = ms ? __ffs(ms) - 1 : 32;  // first lane that ends the walk
-      if (!(lane < k0 || (lane == k0 && holds))) c = T(0);
 #pragma unroll
-      for (int off = 16; off > 0; off >>= 1) c += __shfl_xor_sync(0xffffffffu, c, off);  // fixed tree
-      sum += c;
-      if (ms) break;
+        for (int off = 16; off > 0; off >>= 1) c += __shfl_xor_sync(0xffffffffu, c, off);  // fixed tree
+        sum += c;
+        if (k0 < 32) break;
+      }
     }
     if (lane == 0) atomicAdd(y + first, sum);
   }
 }
+
 template <typename T, bool kBro, int TT, int kWarps, int kMinBlocks, int kMode>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
