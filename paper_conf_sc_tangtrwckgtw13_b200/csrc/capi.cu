@@ -92,8 +92,7 @@ struct bro_matrix_s {
   int32_t* d_coo_col = nullptr;
   void* d_coo_vals = nullptr;
   void* d_cy = nullptr;        // per interval: partial of its last row when that row continues
-  int32_t* d_flag = nullptr;   // per interval: epoch of the call that published its carry
-  int32_t* d_sync = nullptr;   // {epoch, finish ticket, start ticket} of the COO kernel
+  int32_t* d_flag = nullptr;   // per interval: 1 once its carry is published (cleared every call)
   void* d_xs = nullptr;
   void* d_ys = nullptr;
   int64_t device_bytes = 0;
@@ -144,8 +143,7 @@ void free_device(bro_matrix_s* A) {
   DeviceGuard g(A->device);
   void* ps[] = {A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr, A->d_ell_vals, A->d_pell_col,
                 A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr, A->d_coo_row,
-                A->d_coo_col, A->d_coo_vals, A->d_cy, A->d_xs, A->d_ys, A->d_xwin, A->d_flag, A->d_sync,
-                A->d_coo_end};
+                A->d_coo_col, A->d_coo_vals, A->d_cy, A->d_xs, A->d_ys, A->d_xwin, A->d_flag, A->d_coo_end};
   for (void* p : ps)
     if (p) cudaFree(p);
   for (cudaEvent_t e : A->e2e_ev) cudaEventDestroy(e);
@@ -481,13 +479,10 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
       } else {
         UP(A->d_coo_row, A->coo.row);
       }
-      // per-interval carries and their publication flags (look-back in the
-      // COO kernel); epoch starts at 1, every flag at 0
+      // per-interval carries and their publication flags (look-back in the COO kernel)
       const size_t nU = size_t(A->nI);
       if (st == BRO_OK) st = dev_upload(A, &A->d_cy, nullptr, nU * A->vsize);
-      std::vector<int32_t> zeros(nU, 0), sync0{1, 0, 0};
-      UP(A->d_flag, zeros);
-      UP(A->d_sync, sync0);
+      if (st == BRO_OK) st = dev_upload(A, &A->d_flag, nullptr, nU * 4);
     }
 #undef UP
     if (st == BRO_OK) st = dtype == BRO_FP64 ? resolve_kernels<double>(A) : resolve_kernels<float>(A);
@@ -583,6 +578,9 @@ bro::dev::YOut<T> make_yout(T* y) {
 template <typename T>
 cudaError_t launch_ell(const bro_matrix_s* A, int mode, const T* x, const bro::dev::YOut<T>& yo, int32_t* dec,
                        int64_t b0, int64_t b1, cudaStream_t st) {
+  // a HYB handle's ELL kernel clears the COO part's publication flags
+  int32_t* zero = mode != 2 && A->has_coo ? A->d_flag : nullptr;
+  int64_t nzero = zero ? A->nI : 0;
   const int64_t H = A->h;
   const int64_t r0 = H * b0, r1 = std::min(A->m, H * b1);
   if (r1 <= r0) return cudaSuccess;
@@ -593,7 +591,7 @@ cudaError_t launch_ell(const bro_matrix_s* A, int mode, const T* x, const bro::d
   const Launch& L = A->ell_k[mode];
   if (A->opts.codec) {
     bro::dev::EllDev<T> p{r1 - r0, b1 - b0, A->d_words, A->d_bit_alloc, A->d_colptr + b0, A->d_symptr + b0,
-                          static_cast<const T*>(A->d_ell_vals), x, A->d_xwin};
+                          static_cast<const T*>(A->d_ell_vals), x, A->d_xwin, zero, nzero};
     // whole part, plain SpMV, 16-byte aligned x: the x-window-staged instance
     if (A->xstage && mode == 0 && b0 == 0 && b1 == A->s && (reinterpret_cast<uintptr_t>(x) & 15) == 0) {
       const int64_t w = A->ell_x.k.warps_per_block();
@@ -603,7 +601,8 @@ cudaError_t launch_ell(const bro_matrix_s* A, int mode, const T* x, const bro::d
   }
   // decode mode covers the padding rows [m, pitch) too (they hold -1)
   const int64_t rows = mode == 2 && b0 == 0 ? A->pitch : r1 - r0;
-  bro::dev::PellDev<T> p{rows, A->K, A->pitch, A->d_pell_col + r0, static_cast<const T*>(A->d_ell_vals) + r0, x};
+  bro::dev::PellDev<T> p{rows, A->K, A->pitch, A->d_pell_col + r0, static_cast<const T*>(A->d_ell_vals) + r0, x,
+                         zero, nzero};
   return launch(L, (p.m + L.k.threads - 1) / L.k.threads, st, p, y, dec);
 }
 
@@ -611,7 +610,7 @@ template <typename T>
 bro::dev::CooDev<T> coo_dev(const bro_matrix_s* A, const T* x) {
   return bro::dev::CooDev<T>{A->nnz_coo, A->nI, A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr,
                             A->d_coo_row, A->d_coo_col, static_cast<const T*>(A->d_coo_vals), x,
-                            A->d_coo_end, static_cast<T*>(A->d_cy), A->d_flag, A->d_sync};
+                            A->d_coo_end, static_cast<T*>(A->d_cy), A->d_flag};
 }
 
 int64_t coo_grid(const bro_matrix_s* A, const Launch& L) {
@@ -634,6 +633,7 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
     e = launch_ell<T>(A, fused && multi ? 1 : 0, x, fused ? yo : make_yout(y), nullptr, 0, nb, st);
   } else if (A->m > 0) {
     e = cudaMemsetAsync(y, 0, size_t(A->m) * sizeof(T), st);
+    if (e == cudaSuccess && A->has_coo && A->nI > 0) e = cudaMemsetAsync(A->d_flag, 0, size_t(A->nI) * 4, st);
   }
   if (e == cudaSuccess && A->has_coo && A->nI > 0) {
     bro::dev::CooDev<T> p = coo_dev<T>(A, x);

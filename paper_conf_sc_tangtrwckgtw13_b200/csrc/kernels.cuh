@@ -183,7 +183,16 @@ struct EllDev {           // a BRO-ELL part (or a range of its slices)
   const T* vals;
   const T* x;
   const int2* xwin;       // x-staged instances: per block, {first column, columns} of its x window
+  int32_t* zero;          // HYB: the COO part's publication flags, cleared by this kernel
+  int64_t nzero;
 };
+
+// Clear n ints with every thread of the grid (the COO flags of a HYB handle,
+// cleared by the kernel that runs before the COO kernel).
+__device__ __forceinline__ void grid_clear(int32_t* p, int64_t n) {
+  const int64_t stride = int64_t(gridDim.x) * blockDim.x;
+  for (int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; k < n; k += stride) p[k] = 0;
+}
 
 // ------------------------------------------------------------------ TMA bulk copy + mbarrier
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -214,6 +223,8 @@ struct PellDev {          // plain ELLPACK (column-major, -1 padding)
   const int32_t* col;
   const T* vals;
   const T* x;
+  int32_t* zero;          // HYB: the COO part's publication flags, cleared by this kernel
+  int64_t nzero;
 };
 
 template <typename T>
@@ -229,8 +240,7 @@ struct CooDev {           // (BRO-)COO part
   const T* x;
   const uint32_t* end_row; // per interval: row of its last entry (static, reading R28)
   T* cy;                  // per interval: partial of its last row, when that row continues
-  int32_t* flag;          // per interval: epoch of the call that published cy
-  int32_t* sync;          // [0] epoch of the current call, [1] finish ticket, [2] start ticket
+  int32_t* flag;          // per interval: 1 once cy is published (cleared before every call)
 };
 
 __device__ __forceinline__ void st_release(int32_t* p, int32_t v) {
@@ -403,6 +413,7 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
   if constexpr (kMode == kSpmv) pdl_launch_dependents();  // a HYB handle's COO part may be scheduled
+  if constexpr (kMode != kDecode) grid_clear(p.zero, p.nzero);
   uint32_t* win = window[w];
   const uint2* cm = colmeta[w];
   // x window of this block (kX): columns [xlo, xlo + xn) in shared memory
@@ -610,6 +621,7 @@ bro_ell_tiny(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
   if constexpr (kMode == kSpmv) pdl_launch_dependents();  // a HYB handle's COO part may be scheduled
+  if constexpr (kMode != kDecode) grid_clear(p.zero, p.nzero);
   const int64_t stride = int64_t(gridDim.x) * kWarps;
   int k32 = 0;
   for (int64_t t = int64_t(blockIdx.x) * kWarps + w; t < p.s; t += stride, k32 = (k32 + 1) & 31) {
@@ -693,6 +705,7 @@ ell_spmv(const PellDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   constexpr int G = 8;
   const int64_t row = int64_t(blockIdx.x) * kThreads + threadIdx.x;
   if constexpr (kMode == kSpmv) pdl_launch_dependents();  // a HYB handle's COO part may be scheduled
+  if constexpr (kMode != kDecode) grid_clear(p.zero, p.nzero);
   if (row >= p.m) return;
   if constexpr (kMode == kDecode) {
     for (int64_t j = 0; j < p.K; ++j) dec[j * p.pitch + row] = ld_stream_s32(p.col + j * p.pitch + row);
@@ -778,7 +791,7 @@ __device__ __forceinline__ void cp_async4(uint32_t* dst, const uint32_t* src) {
 // One interval of the (BRO-)COO kernel (warp i).
 template <typename T, bool kBro, int TT, int kWarps, int kMode>
 __device__ __forceinline__ void coo_interval(const CooDev<T>& p, T* __restrict__ y, int32_t* __restrict__ dec,
-                                             int64_t i, int32_t epoch, uint32_t* cw, int lane) {
+                                             int64_t i, uint32_t* cw, int lane) {
   constexpr int I = 32 * TT;
   constexpr int CH = TT < 16 ? TT : 16;  // entries per lane loaded at once (one chunk)
   constexpr int NC = TT / CH;
@@ -954,6 +967,9 @@ __device__ __forceinline__ void coo_interval(const CooDev<T>& p, T* __restrict__
   // where it ends), as its partial in b plus the partials the intervals a..b-1
   // published (cy[j], the partial of j's last row) in a fixed order; every
   // other row of the interval is complete here and gets one direct add.
+  // Owners wait only on lower intervals (blockIdx order, as in a single-pass
+  // scan); the flags are cleared before every call (HYB: by the ELL kernel,
+  // which runs first; COO-only: by the memset that zeroes y).
   const int Lw = __shfl_sync(0xffffffffu, L, 31);  // == end_row[i]
   const T co31 = __shfl_sync(0xffffffffu, co, 31);
   const unsigned mF = __ballot_sync(0xffffffffu, hasF);
@@ -963,7 +979,7 @@ __device__ __forceinline__ void coo_interval(const CooDev<T>& p, T* __restrict__
   if (last_continues) {  // publish the partial of the last row for its owner
     if (lane == 31) {
       p.cy[i] = Lw == first ? Fp : co31;
-      st_release(p.flag + i, epoch);
+      st_release(p.flag + i, 1);
     }
   } else if (Lw != first && lane == 31) {
     atomicAdd(y + Lw, co31);  // the last row starts and ends here
@@ -984,7 +1000,7 @@ __device__ __forceinline__ void coo_interval(const CooDev<T>& p, T* __restrict__
         const bool needed = lane < k0 || (lane == k0 && j >= 0 && int(p.end_row[j]) == first);
         T c = T(0);
         if (needed) {
-          while (ld_acquire(p.flag + j) != epoch) __nanosleep(20);
+          while (ld_acquire(p.flag + j) != 1) __nanosleep(20);
           c = p.cy[j];
         }
 #pragma unroll
@@ -1003,32 +1019,10 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   __shared__ uint32_t cwin[kWarps][kBro ? (TT + 1) * 32 : 1];  // <= T symbol rows + a zero guard row
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
-  if constexpr (kMode == kDecode) {
-    const int64_t i = int64_t(blockIdx.x) * kWarps + w;
-    if (i >= p.nI) return;
-    coo_interval<T, kBro, TT, kWarps, kMode>(p, y, dec, i, 0, cwin[w], lane);
-  } else {
-    // the block's intervals come from a start ticket, not blockIdx: every
-    // interval an owner looks back at belongs to a block that has started
-    // (no dependence on the hardware's block dispatch order)
-    __shared__ int64_t tile;
-    if (threadIdx.x == 0) tile = atomicAdd(p.sync + 2, 1);
-    __syncthreads();
-    const int64_t i = tile * kWarps + w;
-    const int32_t epoch = *reinterpret_cast<volatile int32_t*>(p.sync);  // this call's epoch
-    if (i < p.nI) coo_interval<T, kBro, TT, kWarps, kMode>(p, y, dec, i, epoch, cwin[w], lane);
-    // the last block to finish resets the tickets and advances the epoch
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      __threadfence();
-      if (atomicAdd(p.sync + 1, 1) == int(gridDim.x) - 1) {
-        p.sync[1] = 0;
-        p.sync[2] = 0;
-        __threadfence();
-        atomicExch(p.sync, epoch + 1);
-      }
-    }
-  }
+  const int64_t i = int64_t(blockIdx.x) * kWarps + w;
+  if constexpr (kMode != kDecode) pdl_launch_dependents();
+  if (i >= p.nI) return;
+  coo_interval<T, kBro, TT, kWarps, kMode>(p, y, dec, i, cwin[w], lane);
 }
 
 // Exchange of a finished y for formats whose last kernel is not an ELL
