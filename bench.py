@@ -391,14 +391,13 @@ def main():
         base = RowBlockSpmv(A, rank, world, dev, fmt=fmt, codec=0, dtype=dtype, bounds=bounds,
                             coo_T=args.coo_T)
     info, binfo = blk.mat.info, base.mat.info
-    # our kernels per step: ELL kernel, COO kernel (rows crossing intervals
-    # resolved inside it); the overlap exchange runs one SpMV per row part
-    # (interior / head / tail); a HYB/COO handle scattering to peers adds its
-    # replicate kernel
-    per_spmv = (0 if fmt == "coo" else 1) + (1 if info["nnz_coo"] else 0)
+    # our kernels per step: ELL kernel, COO kernel + fix-up; the overlap
+    # exchange runs one SpMV per row part (interior / head / tail); a
+    # HYB/COO handle scattering to peers adds its replicate kernel
+    per_spmv = (0 if fmt == "coo" else 1) + (2 if info["nnz_coo"] else 0)
     launches = per_spmv
     if world > 1 and blk.exchange == "overlap":
-        launches = sum((0 if fmt == "coo" else 1) + (1 if p.info["nnz_coo"] else 0) for _, _, p in blk.parts)
+        launches = sum((0 if fmt == "coo" else 1) + (2 if p.info["nnz_coo"] else 0) for _, _, p in blk.parts)
     elif world > 1 and blk.exchange == "p2p" and info["nnz_coo"]:
         launches = per_spmv + 1
     flush_buf = torch.empty(2 * L2_BYTES // 4, dtype=torch.int32, device=dev) if args.flush_l2 else None
@@ -550,8 +549,8 @@ def main():
                      "kernel": (f"bro_ell_{'tiny' if info['ell_kernel'] == 1 else 'od'}"
                                 f"<{'double' if dtype == np.float64 else 'float'},V={info['vec_words']},"
                                 f"R={info['slice_h'] // 32}>")
-                     if fmt == "ell" else ("coo_spmv" if fmt == "coo" else
-                                           "bro_ell + coo_spmv"),
+                     if fmt == "ell" else ("coo_spmv + coo_fixup" if fmt == "coo" else
+                                           "bro_ell + coo_spmv + coo_fixup"),
                      "algorithmic_bytes_per_launch": alg_bytes, "kernel_ms": kern_ms,
                      "frac_of_8TBps_spec": achieved / 8000.0,
                      "read_stream_GBps": rc, "read_stream_how": "torch.sum over 2 GiB fp32 (a library "

@@ -48,8 +48,7 @@
  *   BRO-COO, intervals of 32*T entries (T = 8, 16 or 32): lane l of interval
  *     i owns the T consecutive entries e = i*32*T + T*l + t (DESIGN.md
  *     reading R13); deltas follow entry order, delta(e) = row(e) - row(e-1),
- *     delta of the first entry 0, base_row[i] = row of the first entry,
- *     end_row[i] = row of the last entry (reading R28), one
+ *     delta of the first entry 0, base_row[i] = row of the first entry, one
  *     width width[i] per interval; lane l's T fields, MSB first,
  *     padded to S_i = ceil(T*width/32) symbols at
  *     coo_words[32*coo_symptr[i] + 32*q + l] (the paper's V = 1 multiplexing,
@@ -122,11 +121,10 @@ typedef struct {
                         (h = 32), 3 small window (every row stream < 10 symbols), 4 mid
                         window (< 18), 5 general.  An instance the matrix does not fit
                         gives BRO_ERR_ARG.  For A/B measurements and tests. */
-  int32_t pdl;       /* HYB: 0 (default) = 1 = the COO kernel is launched as a programmatic
-                        dependent of the ELL kernel (its loads, decode and x gathers
-                        overlap the ELL kernel's tail; it waits before updating y);
-                        2 = plain stream order.  Rows that cross COO intervals are
-                        resolved inside the COO kernel (deterministic look-back). */
+  int32_t pdl;       /* HYB / COO: 0 (default) = 1 = the COO kernel is launched as a
+                        programmatic dependent of the ELL kernel (its loads, decode and x
+                        gathers overlap the ELL kernel's tail; it waits before updating y),
+                        and the fix-up as one of the COO kernel; 2 = plain stream order. */
   int32_t x_stage;   /* few-slice BRO-ELL instance (h = 32, fewer slices than 148 x 32):
                         1 = each block has the TMA engine copy its x column window
                         (<= 96 KB) into shared memory and gathers from there, when the
@@ -179,8 +177,7 @@ typedef enum {
   BRO_PART_COO_VALS = 10,     /* value[nI*32*T]  same arrangement, 0 past nnz */
   BRO_PART_COO_ROW = 11,      /* int32[nI*32*T]  plain COO rows (codec 0), last row past nnz */
   BRO_PART_PELL_COL = 12,     /* int32[K*pitch]  plain ELL, column-major, -1 = padding (codec 0) */
-  BRO_PART_PELL_VALS = 13,    /* value[K*pitch]  plain ELL values (codec 0) */
-  BRO_PART_COO_END_ROW = 14   /* uint32[nI]      row of each interval's last entry (BRO and plain COO) */
+  BRO_PART_PELL_VALS = 13     /* value[K*pitch]  plain ELL values (codec 0) */
 } bro_part_t;
 
 /* Fill *opts with the defaults: h 0 (auto), sym 32, V 0 (auto), T 0 (auto),

@@ -28,9 +28,6 @@ SURVEY §8(f) NEXT-4):
   * b_i = Gamma(max delta) (0 allowed: one row per interval); lane l's
     stream is its T fields of b_i bits, MSB first, padded to
     S_i = ceil(T*b_i/32) symbols and multiplexed with BRO-ELL's place();
-  * end_row[i] = the row of the interval's last entry (reading R28: metadata
-    that lets the kernel tell, without decoding a neighbour, whether a row
-    crosses into the next interval);
   * col and vals are stored in the same lane-contiguous arrangement,
     multiplexed for 16-byte chunk loads exactly like BRO-ELL's values
     (P:L116's multiplexing applied to the raw arrays, reading R26): entry
@@ -55,7 +52,6 @@ class BroCoo:
     T: int
     V: int
     base_row: np.ndarray    # uint32[nI]
-    end_row: np.ndarray     # uint32[nI]  row of the interval's last entry (carry metadata, reading R28)
     width: np.ndarray       # uint8[nI]   (bit_alloc of P:L140, one per interval)
     symptr: np.ndarray      # uint64[nI+1] per-lane words before interval i
     words: np.ndarray       # uint32[32*symptr[nI]]
@@ -135,7 +131,6 @@ def encode(rows, cols, vals, T=32, V=4, sym_len=32) -> BroCoo:
     I = 32 * T
     nI = -(-N // I)
     base_row = np.zeros(nI, dtype=np.uint32)
-    end_row = np.zeros(nI, dtype=np.uint32)
     width = np.zeros(nI, dtype=np.uint8)
     symptr = np.zeros(nI + 1, dtype=np.uint64)
     streams = []
@@ -154,7 +149,6 @@ def encode(rows, cols, vals, T=32, V=4, sym_len=32) -> BroCoo:
             mask = (1 << sym_len) - 1
             lane_syms.append([(stream >> (sym_len * (S - 1 - q))) & mask for q in range(S)])
         base_row[i] = base
-        end_row[i] = int(rows[min((i + 1) * I, N) - 1])
         width[i] = b
         symptr[i + 1] = symptr[i] + S
         streams.append((S, lane_syms))
@@ -166,7 +160,7 @@ def encode(rows, cols, vals, T=32, V=4, sym_len=32) -> BroCoo:
                 words[wb + place(lane, q, S, V, 32)] = lane_syms[lane][q]
     col = arrange(np.asarray(cols, dtype=np.int32), T, 4, 0)
     v = arrange(vals, T, value_chunk(vals.dtype.itemsize), 0)
-    return BroCoo(N, T, V, base_row, end_row, width, symptr, words, col, v)
+    return BroCoo(N, T, V, base_row, width, symptr, words, col, v)
 
 
 def plain_rows(rows, T=32):

@@ -25,7 +25,7 @@ STATUS = {0: "BRO_OK", 1: "BRO_ERR_ARG", 2: "BRO_ERR_INDEX", 3: "BRO_ERR_SHAPE",
 PARTS = {
     "ell_words": 0, "ell_bit_alloc": 1, "ell_colptr": 2, "ell_symptr": 3, "ell_vals": 4,
     "coo_words": 5, "coo_base_row": 6, "coo_width": 7, "coo_symptr": 8, "coo_col": 9,
-    "coo_vals": 10, "coo_row": 11, "pell_col": 12, "pell_vals": 13, "coo_end_row": 14,
+    "coo_vals": 10, "coo_row": 11, "pell_col": 12, "pell_vals": 13,
 }
 FORMATS = {0: "ELL", 1: "COO", 2: "HYB"}
 
@@ -190,7 +190,7 @@ def bro_get_info(h: int) -> dict:
 
 
 _PART_DTYPES = {0: np.uint32, 1: np.uint8, 2: np.uint64, 3: np.uint64, 5: np.uint32, 6: np.uint32,
-                7: np.uint8, 8: np.uint64, 9: np.int32, 11: np.int32, 12: np.int32, 14: np.uint32}
+                7: np.uint8, 8: np.uint64, 9: np.int32, 11: np.int32, 12: np.int32}
 
 
 def bro_export_encoded(h: int, part, value_dtype=None) -> np.ndarray:

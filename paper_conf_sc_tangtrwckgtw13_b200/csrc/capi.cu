@@ -85,21 +85,22 @@ struct bro_matrix_s {
   int32_t* d_pell_col = nullptr;
   uint32_t* d_coo_words = nullptr;
   uint32_t* d_coo_base = nullptr;
-  uint32_t* d_coo_end = nullptr;
   uint8_t* d_coo_width = nullptr;
   uint64_t* d_coo_symptr = nullptr;
   int32_t* d_coo_row = nullptr;
   int32_t* d_coo_col = nullptr;
   void* d_coo_vals = nullptr;
-  void* d_cy = nullptr;        // per interval: partial of its last row when that row continues
-  int32_t* d_flag = nullptr;   // per interval: 1 once its carry is published (cleared every call)
+  void* d_cf = nullptr;
+  void* d_cl = nullptr;
+  int32_t* d_last_row = nullptr;
+  int32_t* d_first_row = nullptr;
   void* d_xs = nullptr;
   void* d_ys = nullptr;
   int64_t device_bytes = 0;
   // kernel instances (index = mode: 0 spmv, 1 scatter, 2 decode)
   Launch ell_k[3];
   Launch coo_k[3];  // 0 spmv, 2 decode
-  Launch rep_k;
+  Launch fix_k, rep_k;
   // x-window staging of the few-slice instance (row N1): per block {first
   // column, columns} of its x window, the staged instance, its shared bytes
   int2* d_xwin = nullptr;
@@ -143,7 +144,8 @@ void free_device(bro_matrix_s* A) {
   DeviceGuard g(A->device);
   void* ps[] = {A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr, A->d_ell_vals, A->d_pell_col,
                 A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr, A->d_coo_row,
-                A->d_coo_col, A->d_coo_vals, A->d_cy, A->d_xs, A->d_ys, A->d_xwin, A->d_flag, A->d_coo_end};
+                A->d_coo_col, A->d_coo_vals, A->d_cf, A->d_cl, A->d_last_row, A->d_first_row, A->d_xs, A->d_ys,
+                A->d_xwin};
   for (void* p : ps)
     if (p) cudaFree(p);
   for (cudaEvent_t e : A->e2e_ev) cudaEventDestroy(e);
@@ -204,11 +206,11 @@ void fill_info(bro_matrix_s* A, double secs) {
     if (A->opts.codec) {
       I.coo_stream_bytes = 4 * A->coo_words;
       stream += I.coo_stream_bytes;
-      meta += A->nI * (4 + 4 + 1) + 8 * (A->nI + 1);  // base_row, end_row, width, symptr
+      meta += A->nI * (4 + 1) + 8 * (A->nI + 1);  // base_row, width, symptr
       raw_index += 4 * slots;                     // col
     } else {
       raw_index += 8 * slots;                     // row + col
-      meta += 8 * A->nI;                          // interval first and last rows
+      meta += 4 * A->nI;                          // interval first rows
     }
     values += slots * vs;
   }
@@ -313,6 +315,7 @@ bro_status_t resolve_kernels(bro_matrix_s* A) {
   if (A->has_coo && !st) {
     st = resolve(A->coo_k[0], bro::coo_ref<T>(A->opts.codec == 1, A->coo_T, 0), sms, "COO");
     if (!st) st = resolve(A->coo_k[2], bro::coo_ref<T>(A->opts.codec == 1, A->coo_T, 2), sms, "COO decode");
+    if (!st) st = resolve(A->fix_k, bro::fixup_ref<T>(), sms, "COO fix-up");
   }
   if (!st) st = resolve(A->rep_k, bro::replicate_ref<T>(), sms, "replicate");
   return st;
@@ -469,7 +472,6 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
     }
     if (A->has_coo) {
       UP(A->d_coo_base, A->coo.base_row);
-      UP(A->d_coo_end, A->coo.end_row);
       UP(A->d_coo_col, A->coo.col);
       if (st == BRO_OK) st = dev_upload(A, &A->d_coo_vals, A->coo.vals.data(), A->coo.vals.size());
       if (o.codec) {
@@ -479,10 +481,12 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
       } else {
         UP(A->d_coo_row, A->coo.row);
       }
-      // per-interval carries and their publication flags (look-back in the COO kernel)
-      const size_t nU = size_t(A->nI);
-      if (st == BRO_OK) st = dev_upload(A, &A->d_cy, nullptr, nU * A->vsize);
-      if (st == BRO_OK) st = dev_upload(A, &A->d_flag, nullptr, nU * 4);
+      // carries of the fix-up: one per work unit (<= max(intervals, warps per block))
+      const size_t nU = size_t(std::max<int64_t>(A->nI, 32));
+      if (st == BRO_OK) st = dev_upload(A, &A->d_cf, nullptr, nU * A->vsize);
+      if (st == BRO_OK) st = dev_upload(A, &A->d_cl, nullptr, nU * A->vsize);
+      if (st == BRO_OK) st = dev_upload(A, &A->d_last_row, nullptr, nU * 4);
+      if (st == BRO_OK) st = dev_upload(A, &A->d_first_row, nullptr, nU * 4);
     }
 #undef UP
     if (st == BRO_OK) st = dtype == BRO_FP64 ? resolve_kernels<double>(A) : resolve_kernels<float>(A);
@@ -578,9 +582,6 @@ bro::dev::YOut<T> make_yout(T* y) {
 template <typename T>
 cudaError_t launch_ell(const bro_matrix_s* A, int mode, const T* x, const bro::dev::YOut<T>& yo, int32_t* dec,
                        int64_t b0, int64_t b1, cudaStream_t st) {
-  // a HYB handle's ELL kernel clears the COO part's publication flags
-  int32_t* zero = mode != 2 && A->has_coo ? A->d_flag : nullptr;
-  int64_t nzero = zero ? A->nI : 0;
   const int64_t H = A->h;
   const int64_t r0 = H * b0, r1 = std::min(A->m, H * b1);
   if (r1 <= r0) return cudaSuccess;
@@ -591,7 +592,7 @@ cudaError_t launch_ell(const bro_matrix_s* A, int mode, const T* x, const bro::d
   const Launch& L = A->ell_k[mode];
   if (A->opts.codec) {
     bro::dev::EllDev<T> p{r1 - r0, b1 - b0, A->d_words, A->d_bit_alloc, A->d_colptr + b0, A->d_symptr + b0,
-                          static_cast<const T*>(A->d_ell_vals), x, A->d_xwin, zero, nzero};
+                          static_cast<const T*>(A->d_ell_vals), x, A->d_xwin};
     // whole part, plain SpMV, 16-byte aligned x: the x-window-staged instance
     if (A->xstage && mode == 0 && b0 == 0 && b1 == A->s && (reinterpret_cast<uintptr_t>(x) & 15) == 0) {
       const int64_t w = A->ell_x.k.warps_per_block();
@@ -601,8 +602,7 @@ cudaError_t launch_ell(const bro_matrix_s* A, int mode, const T* x, const bro::d
   }
   // decode mode covers the padding rows [m, pitch) too (they hold -1)
   const int64_t rows = mode == 2 && b0 == 0 ? A->pitch : r1 - r0;
-  bro::dev::PellDev<T> p{rows, A->K, A->pitch, A->d_pell_col + r0, static_cast<const T*>(A->d_ell_vals) + r0, x,
-                         zero, nzero};
+  bro::dev::PellDev<T> p{rows, A->K, A->pitch, A->d_pell_col + r0, static_cast<const T*>(A->d_ell_vals) + r0, x};
   return launch(L, (p.m + L.k.threads - 1) / L.k.threads, st, p, y, dec);
 }
 
@@ -610,7 +610,7 @@ template <typename T>
 bro::dev::CooDev<T> coo_dev(const bro_matrix_s* A, const T* x) {
   return bro::dev::CooDev<T>{A->nnz_coo, A->nI, A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr,
                             A->d_coo_row, A->d_coo_col, static_cast<const T*>(A->d_coo_vals), x,
-                            A->d_coo_end, static_cast<T*>(A->d_cy), A->d_flag};
+                            static_cast<T*>(A->d_cf), static_cast<T*>(A->d_cl), A->d_first_row, A->d_last_row};
 }
 
 int64_t coo_grid(const bro_matrix_s* A, const Launch& L) {
@@ -621,7 +621,7 @@ int64_t coo_grid(const bro_matrix_s* A, const Launch& L) {
 // y = A.x stored into every destination of yo (yo.p[0] = the local y on A's
 // device).  ELL-only handles store all destinations from the ELL kernel's
 // epilogue (fused exchange); handles with a COO part finish y locally and
-// then replicate it (the COO part adds into y).
+// then replicate it (the COO part and the fix-up add into y).
 template <typename T>
 bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& yo, cudaStream_t st) {
   T* y = yo.p[0];
@@ -633,16 +633,25 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
     e = launch_ell<T>(A, fused && multi ? 1 : 0, x, fused ? yo : make_yout(y), nullptr, 0, nb, st);
   } else if (A->m > 0) {
     e = cudaMemsetAsync(y, 0, size_t(A->m) * sizeof(T), st);
-    if (e == cudaSuccess && A->has_coo && A->nI > 0) e = cudaMemsetAsync(A->d_flag, 0, size_t(A->nI) * 4, st);
   }
   if (e == cudaSuccess && A->has_coo && A->nI > 0) {
     bro::dev::CooDev<T> p = coo_dev<T>(A, x);
     int32_t* none = nullptr;
-    // the COO kernel overlaps the ELL kernel's tail (programmatic dependent
-    // launch, bro_opts_t.pdl); rows crossing intervals are resolved inside it
-    const bool after_ell = A->has_ell && A->opts.pdl != 2;
+    // the COO kernel overlaps the ELL kernel's tail, the fix-up the COO
+    // kernel's (programmatic dependent launches, bro_opts_t.pdl)
+    const bool pdl = A->opts.pdl != 2;
+    const bool after_ell = A->has_ell && pdl;
     e = after_ell ? launch_pdl(A->coo_k[0], coo_grid(A, A->coo_k[0]), st, p, y, none)
                   : launch(A->coo_k[0], coo_grid(A, A->coo_k[0]), st, p, y, none);
+    if (e == cudaSuccess) {
+      int64_t nU = A->nI;
+      const int32_t* fr = A->d_first_row;
+      const int32_t* lr = A->d_last_row;
+      const T* cf = static_cast<const T*>(A->d_cf);
+      const T* cl = static_cast<const T*>(A->d_cl);
+      e = pdl ? launch_pdl(A->fix_k, (nU + 255) / 256, st, nU, fr, lr, cf, cl, y)
+              : launch(A->fix_k, (nU + 255) / 256, st, nU, fr, lr, cf, cl, y);
+    }
   }
   if (e == cudaSuccess && !fused && A->m > 0 && multi) {
     int64_t m = A->m;
@@ -678,7 +687,6 @@ PartView part_view(bro_matrix_s* A, int32_t part) {
     case BRO_PART_ELL_VALS: if (bro_ell) set(A->ell.vals.data(), A->d_ell_vals, vs * size_t(A->ell_slots)); break;
     case BRO_PART_COO_WORDS: if (bro_coo) set(A->coo.words.data(), A->d_coo_words, 4 * size_t(A->coo_words)); break;
     case BRO_PART_COO_BASE_ROW: if (bro_coo) set(A->coo.base_row.data(), A->d_coo_base, 4 * size_t(A->nI)); break;
-    case BRO_PART_COO_END_ROW: if (coo) set(A->coo.end_row.data(), A->d_coo_end, 4 * size_t(A->nI)); break;
     case BRO_PART_COO_WIDTH: if (bro_coo) set(A->coo.width.data(), A->d_coo_width, size_t(A->nI)); break;
     case BRO_PART_COO_SYMPTR: if (bro_coo) set(A->coo.symptr.data(), A->d_coo_symptr, 8 * size_t(A->nI + 1)); break;
     case BRO_PART_COO_COL: if (coo) set(A->coo.col.data(), A->d_coo_col, 4 * slots); break;

@@ -306,11 +306,9 @@ void encode_bro_coo(int64_t nnz, const int32_t* row, const int32_t* col, const u
   out.nnz = nnz;
   out.nI = nI;
   out.base_row.assign(nI, 0);
-  out.end_row.assign(nI, 0);
   out.width.assign(nI, 0);
   std::vector<uint64_t> nsym(nI, 0);
   auto at = [&](int64_t e) { return (uint32_t)row[std::min(e, nnz - 1)]; };
-  for (int64_t i = 0; i < nI; ++i) out.end_row[i] = at(std::min((i + 1) * I, nnz) - 1);
   parallel_for(nI, [&](int64_t lo, int64_t hi) {
     for (int64_t i = lo; i < hi; ++i) {
       const uint32_t base = at(i * I);
@@ -354,11 +352,7 @@ void build_plain_coo(int64_t nnz, const int32_t* row, const int32_t* col, const 
   out.nnz = nnz;
   out.nI = (nnz + I - 1) / I;
   out.base_row.assign(out.nI, 0);
-  out.end_row.assign(out.nI, 0);
-  for (int64_t i = 0; i < out.nI; ++i) {
-    out.base_row[i] = (uint32_t)row[i * I];
-    out.end_row[i] = (uint32_t)row[std::min((i + 1) * I, nnz) - 1];
-  }
+  for (int64_t i = 0; i < out.nI; ++i) out.base_row[i] = (uint32_t)row[i * I];
   out.row.assign(out.nI * I, 0);
   arrange<int32_t>(nnz, T, 4, row, nnz ? row[nnz - 1] : 0, 4, reinterpret_cast<uint8_t*>(out.row.data()), out.nI);
   arrange_col_vals(nnz, col, vals, vsize, T, out);

@@ -55,7 +55,6 @@ struct CooCode {
   int T = 32;
   int64_t nnz = 0, nI = 0;
   std::vector<uint32_t> base_row; // nI
-  std::vector<uint32_t> end_row;  // nI: row of the interval's last entry (reading R28)
   std::vector<uint8_t> width;     // nI
   std::vector<uint64_t> symptr;   // nI+1
   std::vector<uint32_t> words;    // 32*symptr[nI]

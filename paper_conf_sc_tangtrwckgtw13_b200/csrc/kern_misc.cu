@@ -46,6 +46,8 @@ template <> KernelRef plain_ell_ref<double>(int mode) { return plain_ell_impl<do
 template <> KernelRef plain_ell_ref<float>(int mode) { return plain_ell_impl<float>(mode); }
 template <> KernelRef coo_ref<double>(bool bro, int TT, int mode) { return coo_impl<double>(bro, TT, mode); }
 template <> KernelRef coo_ref<float>(bool bro, int TT, int mode) { return coo_impl<float>(bro, TT, mode); }
+template <> KernelRef fixup_ref<double>() { return {(const void*)&dev::coo_fixup<double>, 256}; }
+template <> KernelRef fixup_ref<float>() { return {(const void*)&dev::coo_fixup<float>, 256}; }
 template <> KernelRef replicate_ref<double>() { return {(const void*)&dev::replicate_y<double>, 256}; }
 template <> KernelRef replicate_ref<float>() { return {(const void*)&dev::replicate_y<float>, 256}; }
 

@@ -21,10 +21,9 @@
 //     decodes its deltas from a staged window, one warp scan of the lane
 //     totals gives every lane its start row, the lane reduces its entries
 //     sequentially and ONE warp segmented scan per interval links segments
-//     that cross lanes (the "parallel scan primitive" of P:L343); rows that
-//     cross intervals are resolved in the same kernel by a deterministic
-//     decoupled look-back (the paper's "extra kernel invocation for data
-//     reduction" becomes a single pass).
+//     that cross lanes (the "parallel scan primitive" of P:L343); a
+//     deterministic fix-up kernel adds the partials of rows crossing
+//     intervals (the "extra kernel invocation for data reduction").
 //   * Uncompressed baselines: ell_spmv (thread per row, column-major
 //     ELLPACK) and coo_spmv<kBro=false> (same traversal, explicit rows).
 //   * Every kernel takes a Mode: kSpmv (y = A.x), kScatter (y also stored
@@ -183,16 +182,7 @@ struct EllDev {           // a BRO-ELL part (or a range of its slices)
   const T* vals;
   const T* x;
   const int2* xwin;       // x-staged instances: per block, {first column, columns} of its x window
-  int32_t* zero;          // HYB: the COO part's publication flags, cleared by this kernel
-  int64_t nzero;
 };
-
-// Clear n ints with every thread of the grid (the COO flags of a HYB handle,
-// cleared by the kernel that runs before the COO kernel).
-__device__ __forceinline__ void grid_clear(int32_t* p, int64_t n) {
-  const int64_t stride = int64_t(gridDim.x) * blockDim.x;
-  for (int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; k < n; k += stride) p[k] = 0;
-}
 
 // ------------------------------------------------------------------ TMA bulk copy + mbarrier
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -223,8 +213,6 @@ struct PellDev {          // plain ELLPACK (column-major, -1 padding)
   const int32_t* col;
   const T* vals;
   const T* x;
-  int32_t* zero;          // HYB: the COO part's publication flags, cleared by this kernel
-  int64_t nzero;
 };
 
 template <typename T>
@@ -238,19 +226,11 @@ struct CooDev {           // (BRO-)COO part
   const int32_t* col;
   const T* vals;
   const T* x;
-  const uint32_t* end_row; // per interval: row of its last entry (static, reading R28)
-  T* cy;                  // per interval: partial of its last row, when that row continues
-  int32_t* flag;          // per interval: 1 once cy is published (cleared before every call)
+  T* cf;                  // per interval: partial of its first row
+  T* cl;                  // per interval: partial of its last row
+  int32_t* first_row;
+  int32_t* last_row;
 };
-
-__device__ __forceinline__ void st_release(int32_t* p, int32_t v) {
-  asm volatile("st.release.gpu.global.s32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
-}
-__device__ __forceinline__ int32_t ld_acquire(const int32_t* p) {
-  int32_t v;
-  asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
 
 // Programmatic dependent launch (PDL): a kernel launched with the
 // programmatic-serialization attribute may start while the previous kernel
@@ -413,7 +393,6 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
   if constexpr (kMode == kSpmv) pdl_launch_dependents();  // a HYB handle's COO part may be scheduled
-  if constexpr (kMode != kDecode) grid_clear(p.zero, p.nzero);
   uint32_t* win = window[w];
   const uint2* cm = colmeta[w];
   // x window of this block (kX): columns [xlo, xlo + xn) in shared memory
@@ -621,7 +600,6 @@ bro_ell_tiny(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   const int lane = threadIdx.x & 31;
   const int w = threadIdx.x >> 5;
   if constexpr (kMode == kSpmv) pdl_launch_dependents();  // a HYB handle's COO part may be scheduled
-  if constexpr (kMode != kDecode) grid_clear(p.zero, p.nzero);
   const int64_t stride = int64_t(gridDim.x) * kWarps;
   int k32 = 0;
   for (int64_t t = int64_t(blockIdx.x) * kWarps + w; t < p.s; t += stride, k32 = (k32 + 1) & 31) {
@@ -705,7 +683,6 @@ ell_spmv(const PellDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   constexpr int G = 8;
   const int64_t row = int64_t(blockIdx.x) * kThreads + threadIdx.x;
   if constexpr (kMode == kSpmv) pdl_launch_dependents();  // a HYB handle's COO part may be scheduled
-  if constexpr (kMode != kDecode) grid_clear(p.zero, p.nzero);
   if (row >= p.m) return;
   if constexpr (kMode == kDecode) {
     for (int64_t j = 0; j < p.K; ++j) dec[j * p.pitch + row] = ld_stream_s32(p.col + j * p.pitch + row);
@@ -788,13 +765,18 @@ __device__ __forceinline__ void cp_async4(uint32_t* dst, const uint32_t* src) {
                "l"(src) : "memory");
 }
 
-// One interval of the (BRO-)COO kernel (warp i).
-template <typename T, bool kBro, int TT, int kWarps, int kMode>
-__device__ __forceinline__ void coo_interval(const CooDev<T>& p, T* __restrict__ y, int32_t* __restrict__ dec,
-                                             int64_t i, uint32_t* cw, int lane) {
+template <typename T, bool kBro, int TT, int kWarps, int kMinBlocks, int kMode>
+__global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
+coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   constexpr int I = 32 * TT;
   constexpr int CH = TT < 16 ? TT : 16;  // entries per lane loaded at once (one chunk)
   constexpr int NC = TT / CH;
+  __shared__ uint32_t cwin[kWarps][kBro ? (TT + 1) * 32 : 1];  // <= T symbol rows + a zero guard row
+  const int lane = threadIdx.x & 31;
+  const int w = threadIdx.x >> 5;
+  const int64_t i = int64_t(blockIdx.x) * kWarps + w;
+  if constexpr (kMode != kDecode) pdl_launch_dependents();  // the fix-up may be scheduled
+  if (i >= p.nI) return;
   const int64_t e0 = i * I;
   const int32_t* cb = p.col + e0;
   const T* vb = p.vals + e0;
@@ -805,7 +787,7 @@ __device__ __forceinline__ void coo_interval(const CooDev<T>& p, T* __restrict__
   bool one = true;
   int b = 0, S = 0, row = 0, first = 0, lim = 0;
   uint32_t w0 = 0, w1 = 0;
-  const uint32_t* wl = cw + lane;
+  const uint32_t* wl = cwin[w] + lane;
 #pragma unroll
   for (int ch = 0; ch < NC; ++ch) {
     // the chunk's col / vals (and plain rows) first: nothing they need
@@ -845,7 +827,7 @@ __device__ __forceinline__ void coo_interval(const CooDev<T>& p, T* __restrict__
             w0 = ld_stream_u32(wb);
             w1 = S > 1 ? ld_stream_u32(wb + 32) : 0u;
           } else {  // the lane words -> [q][lane] window by cp.async
-            uint32_t* win = cw + lane;
+            uint32_t* win = cwin[w] + lane;
             for (int q = 0; q < S; ++q) cp_async4(win + 32 * q, wb + 32 * q);
             asm volatile("cp.async.commit_group;" ::: "memory");
             win[32 * S] = 0u;
@@ -948,81 +930,23 @@ __device__ __forceinline__ void coo_interval(const CooDev<T>& p, T* __restrict__
   }
   T cin = __shfl_up_sync(0xffffffffu, co, 1);
   if (!link) cin = T(0);
-  // complete segments of rows other than the interval's first go straight to
-  // y (each such row lives in this interval alone, or is its last row and
-  // ends here); the first row's partial is collected for the carry logic
-  T fpart = T(0);
-  bool hasF = false;
   auto emit = [&](int rr, T val) {
-    if (rr == first) { fpart = val; hasF = true; }
+    if (rr == first) p.cf[i] = val;
     else atomicAdd(y + rr, val);
   };
   if (!one) emit(f, A + cin);  // first segment complete inside this lane
   const int fnext = __shfl_down_sync(0xffffffffu, f, 1);
   if (lane < 31 && fnext != L) emit(L, co);  // trailing segment complete at this lane
-  // Rows that cross intervals, resolved in this kernel (look-back,
-  // deterministic).  Which rows cross is static: interval j's first row is
-  // base_row[j] and its last row end_row[j] (reading R28).  A row R that
-  // spans intervals a..b is added to y once, by its owner b (the interval
-  // where it ends), as its partial in b plus the partials the intervals a..b-1
-  // published (cy[j], the partial of j's last row) in a fixed order; every
-  // other row of the interval is complete here and gets one direct add.
-  // Owners wait only on lower intervals (blockIdx order, as in a single-pass
-  // scan); the flags are cleared before every call (HYB: by the ELL kernel,
-  // which runs first; COO-only: by the memset that zeroes y).
-  const int Lw = __shfl_sync(0xffffffffu, L, 31);  // == end_row[i]
-  const T co31 = __shfl_sync(0xffffffffu, co, 31);
-  const unsigned mF = __ballot_sync(0xffffffffu, hasF);
-  const T Fp = mF ? __shfl_sync(0xffffffffu, fpart, __ffs(mF) - 1) : co31;  // L == F: the whole interval
-  const bool last_continues = i + 1 < p.nI && int(p.base_row[i + 1]) == Lw;
-  const bool first_continued = i > 0 && int(p.end_row[i - 1]) == first;
-  if (last_continues) {  // publish the partial of the last row for its owner
-    if (lane == 31) {
-      p.cy[i] = Lw == first ? Fp : co31;
-      st_release(p.flag + i, 1);
+  if (lane == 31) {  // the interval's last row: its partial is carried
+    p.first_row[i] = first;
+    p.last_row[i] = L;
+    if (L == first) {
+      p.cf[i] = co;
+      p.cl[i] = T(0);
+    } else {
+      p.cl[i] = co;
     }
-  } else if (Lw != first && lane == 31) {
-    atomicAdd(y + Lw, co31);  // the last row starts and ends here
   }
-  if (Lw != first || !last_continues) {  // this interval owns its first row F
-    T sum = Fp;
-    if (first_continued) {
-      // intervals i-1, i-2, ... hold F (end_row == F); all of those whose
-      // first row is F too continue the walk, the one where F starts ends it.
-      // Lane k examines j = jb - k; the flags waited for are exactly those of
-      // intervals holding F.
-      for (int64_t jb = i - 1;; jb -= 32) {
-        const int64_t j = jb - lane;
-        const bool whole = j >= 0 && int(p.base_row[j]) == first;  // j is all F
-        const unsigned mw = __ballot_sync(0xffffffffu, whole);
-        const int k0 = ~mw ? __ffs(~mw) - 1 : 32;  // first lane not all F
-        // lanes < k0 are all-F intervals; lane k0 holds F iff its last row is F
-        const bool needed = lane < k0 || (lane == k0 && j >= 0 && int(p.end_row[j]) == first);
-        T c = T(0);
-        if (needed) {
-          while (ld_acquire(p.flag + j) != 1) __nanosleep(20);
-          c = p.cy[j];
-        }
-#pragma unroll
-        for (int off = 16; off > 0; off >>= 1) c += __shfl_xor_sync(0xffffffffu, c, off);  // fixed tree
-        sum += c;
-        if (k0 < 32) break;
-      }
-    }
-    if (lane == 0) atomicAdd(y + first, sum);
-  }
-}
-
-template <typename T, bool kBro, int TT, int kWarps, int kMinBlocks, int kMode>
-__global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
-coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
-  __shared__ uint32_t cwin[kWarps][kBro ? (TT + 1) * 32 : 1];  // <= T symbol rows + a zero guard row
-  const int lane = threadIdx.x & 31;
-  const int w = threadIdx.x >> 5;
-  const int64_t i = int64_t(blockIdx.x) * kWarps + w;
-  if constexpr (kMode != kDecode) pdl_launch_dependents();
-  if (i >= p.nI) return;
-  coo_interval<T, kBro, TT, kWarps, kMode>(p, y, dec, i, cwin[w], lane);
 }
 
 // Exchange of a finished y for formats whose last kernel is not an ELL
@@ -1043,6 +967,64 @@ __global__ void replicate_y(int64_t m, const YOut<T> o) {
         if (k < o.n) o.p[k][i] = v;
     }
   }
+}
+
+// Deterministic application of the intervals' carries (one thread per
+// interval, fixed summation order = interval order).  first[u] / last[u] =
+// rows of the interval's first and last entries; cf = partial of the first
+// row (the whole interval if first == last), cl = partial of the last row.
+// acc += cf[j] for the intervals j = i+1, i+2, ... that continue row R
+// (first[j] == R), stopping after the first of them that ends on another
+// row.  Intervals are read 8 at a time (one round trip for rows spanning up
+// to 9 intervals); the additions stay in interval order.
+template <typename T>
+__device__ __forceinline__ T chain_sum(int64_t i, int64_t nU, int R, T acc, const int32_t* __restrict__ first,
+                                       const int32_t* __restrict__ last_row, const T* __restrict__ cf) {
+  constexpr int B = 8;
+  for (int64_t j0 = i + 1; j0 < nU; j0 += B) {
+    int fj[B], lj[B];
+    T cj[B];
+#pragma unroll
+    for (int k = 0; k < B; ++k) {
+      const bool in = j0 + k < nU;
+      fj[k] = in ? first[j0 + k] : -1;
+      lj[k] = in ? last_row[j0 + k] : -1;
+      cj[k] = in ? cf[j0 + k] : T(0);
+    }
+    bool done = false;
+#pragma unroll
+    for (int k = 0; k < B; ++k) {
+      if (!done) {
+        if (fj[k] < 0) {
+          // an empty unit holds no row: skip it
+        } else if (fj[k] != R) {
+          done = true;
+        } else {
+          acc += cj[k];
+          done = lj[k] != R;
+        }
+      }
+    }
+    if (done) break;
+  }
+  return acc;
+}
+
+template <typename T>
+__global__ void coo_fixup(int64_t nU, const int32_t* __restrict__ first, const int32_t* __restrict__ last_row,
+                          const T* __restrict__ cf, const T* __restrict__ cl, T* __restrict__ y) {
+  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  pdl_wait();  // the carries come from the COO kernel
+  if (i >= nU) return;
+  const int F = first[i];
+  const int L = last_row[i];
+  if (F < 0) return;  // an empty unit
+  if (L != F)  // unit i is the first one holding row L
+    y[L] += chain_sum<T>(i, nU, L, cl[i], first, last_row, cf);
+  int64_t j = i - 1;  // the previous non-empty unit
+  while (j >= 0 && first[j] < 0) --j;
+  if (j < 0 || last_row[j] != F)  // unit i is the first one holding row F
+    y[F] += L == F ? chain_sum<T>(i, nU, F, cf[i], first, last_row, cf) : cf[i];
 }
 
 }  // namespace dev

@@ -26,6 +26,7 @@ template <typename T> KernelRef bro_ell_ref(int V, int R, int inst, int mode);
 template <typename T> KernelRef bro_ell_xstage_ref(int V);  // few-slice instance, x window in shared memory
 template <typename T> KernelRef plain_ell_ref(int mode);
 template <typename T> KernelRef coo_ref(bool bro, int TT, int mode);  // mode 0 or 2
+template <typename T> KernelRef fixup_ref();
 template <typename T> KernelRef replicate_ref();
 
 }  // namespace bro

@@ -109,7 +109,6 @@ def _coo_parts_equal(lib, h, C, r, c, v, codec=1):
         assert np.array_equal(lib.bro_export_encoded(h, "coo_symptr"), C.symptr)
     else:
         assert np.array_equal(lib.bro_export_encoded(h, "coo_row"), bro_coo.plain_rows(r, C.T))
-    assert np.array_equal(lib.bro_export_encoded(h, "coo_end_row"), C.end_row)
     assert np.array_equal(lib.bro_export_encoded(h, "coo_col"), C.col)
     assert np.array_equal(lib.bro_export_encoded(h, "coo_vals", v.dtype), C.vals)
 
