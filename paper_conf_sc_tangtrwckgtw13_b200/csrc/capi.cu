@@ -92,8 +92,11 @@ struct bro_matrix_s {
   void* d_coo_vals = nullptr;
   void* d_cf = nullptr;
   void* d_cl = nullptr;
-  int32_t* d_last_row = nullptr;
-  int32_t* d_first_row = nullptr;
+  int32_t* d_coo_end = nullptr;  // per interval: row of its last entry
+  int4* d_spans = nullptr;       // rows spanning intervals: {row, first interval, last interval, uses cl}
+  int64_t n_spans = 0;
+  std::vector<int32_t> coo_end_host;
+  std::vector<int4> spans_host;
   void* d_xs = nullptr;
   void* d_ys = nullptr;
   int64_t device_bytes = 0;
@@ -144,7 +147,7 @@ void free_device(bro_matrix_s* A) {
   DeviceGuard g(A->device);
   void* ps[] = {A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr, A->d_ell_vals, A->d_pell_col,
                 A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr, A->d_coo_row,
-                A->d_coo_col, A->d_coo_vals, A->d_cf, A->d_cl, A->d_last_row, A->d_first_row, A->d_xs, A->d_ys,
+                A->d_coo_col, A->d_coo_vals, A->d_cf, A->d_cl, A->d_coo_end, A->d_spans, A->d_xs, A->d_ys,
                 A->d_xwin};
   for (void* p : ps)
     if (p) cudaFree(p);
@@ -399,6 +402,21 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
         bro::build_plain_coo(A->nnz_coo, cr.data(), cc.data(), cv.data(), A->vsize, A->coo_T, A->coo);
       A->nI = A->coo.nI;
       A->coo_words = (int64_t)A->coo.words.size();
+      // rows that span COO intervals (for the fix-up): interval i's first row
+      // is cr[i*I], its last row cr[min((i+1)*I, N) - 1]
+      const int64_t I = 32 * int64_t(A->coo_T), N = A->nnz_coo;
+      A->coo_end_host.resize(A->nI);
+      for (int64_t i = 0; i < A->nI; ++i) A->coo_end_host[i] = cr[std::min((i + 1) * I, N) - 1];
+      auto base = [&](int64_t i) { return cr[i * I]; };
+      for (int64_t i = 0; i + 1 < A->nI;) {
+        const int32_t R = A->coo_end_host[i];
+        if (base(i + 1) != R) { ++i; continue; }
+        int64_t b = i + 1;
+        while (b + 1 < A->nI && base(b + 1) == R) ++b;
+        A->spans_host.push_back(int4{R, int(i), int(b), base(i) != R ? 1 : 0});
+        i = b;
+      }
+      A->n_spans = int64_t(A->spans_host.size());
     }
     // x windows of the few-slice instance's blocks (row N1): BRO-ELL at h = 32
     // with fewer slices than the general instance keeps resident (148 SMs x 32)
@@ -481,12 +499,13 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
       } else {
         UP(A->d_coo_row, A->coo.row);
       }
-      // carries of the fix-up: one per work unit (<= max(intervals, warps per block))
-      const size_t nU = size_t(std::max<int64_t>(A->nI, 32));
+      // carries of the rows spanning intervals, the intervals' last rows and
+      // the span list of the fix-up
+      const size_t nU = size_t(A->nI);
       if (st == BRO_OK) st = dev_upload(A, &A->d_cf, nullptr, nU * A->vsize);
       if (st == BRO_OK) st = dev_upload(A, &A->d_cl, nullptr, nU * A->vsize);
-      if (st == BRO_OK) st = dev_upload(A, &A->d_last_row, nullptr, nU * 4);
-      if (st == BRO_OK) st = dev_upload(A, &A->d_first_row, nullptr, nU * 4);
+      UP(A->d_coo_end, A->coo_end_host);
+      UP(A->d_spans, A->spans_host);
     }
 #undef UP
     if (st == BRO_OK) st = dtype == BRO_FP64 ? resolve_kernels<double>(A) : resolve_kernels<float>(A);
@@ -501,6 +520,8 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
     A->ell = bro::EllCode();
     A->pell = bro::PlainEll();
     A->coo = bro::CooCode();
+    A->coo_end_host = std::vector<int32_t>();
+    A->spans_host = std::vector<int4>();
   } else {
     if (A->has_ell && o.codec) {
       bro_status_t st = choose_ell_instance(A, 148);
@@ -610,7 +631,7 @@ template <typename T>
 bro::dev::CooDev<T> coo_dev(const bro_matrix_s* A, const T* x) {
   return bro::dev::CooDev<T>{A->nnz_coo, A->nI, A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr,
                             A->d_coo_row, A->d_coo_col, static_cast<const T*>(A->d_coo_vals), x,
-                            static_cast<T*>(A->d_cf), static_cast<T*>(A->d_cl), A->d_first_row, A->d_last_row};
+                            static_cast<T*>(A->d_cf), static_cast<T*>(A->d_cl), A->d_coo_end};
 }
 
 int64_t coo_grid(const bro_matrix_s* A, const Launch& L) {
@@ -643,14 +664,13 @@ bro_status_t launch_spmv(bro_matrix_s* A, const T* x, const bro::dev::YOut<T>& y
     const bool after_ell = A->has_ell && pdl;
     e = after_ell ? launch_pdl(A->coo_k[0], coo_grid(A, A->coo_k[0]), st, p, y, none)
                   : launch(A->coo_k[0], coo_grid(A, A->coo_k[0]), st, p, y, none);
-    if (e == cudaSuccess) {
-      int64_t nU = A->nI;
-      const int32_t* fr = A->d_first_row;
-      const int32_t* lr = A->d_last_row;
+    if (e == cudaSuccess && A->n_spans > 0) {  // rows spanning intervals
+      int64_t nS = A->n_spans;
+      const int4* sp = A->d_spans;
       const T* cf = static_cast<const T*>(A->d_cf);
       const T* cl = static_cast<const T*>(A->d_cl);
-      e = pdl ? launch_pdl(A->fix_k, (nU + 255) / 256, st, nU, fr, lr, cf, cl, y)
-              : launch(A->fix_k, (nU + 255) / 256, st, nU, fr, lr, cf, cl, y);
+      e = pdl ? launch_pdl(A->fix_k, (nS + 255) / 256, st, nS, sp, cf, cl, y)
+              : launch(A->fix_k, (nS + 255) / 256, st, nS, sp, cf, cl, y);
     }
   }
   if (e == cudaSuccess && !fused && A->m > 0 && multi) {

@@ -226,10 +226,9 @@ struct CooDev {           // (BRO-)COO part
   const int32_t* col;
   const T* vals;
   const T* x;
-  T* cf;                  // per interval: partial of its first row
-  T* cl;                  // per interval: partial of its last row
-  int32_t* first_row;
-  int32_t* last_row;
+  T* cf;                  // per interval: partial of its first row (when that row spans intervals)
+  T* cl;                  // per interval: partial of its last row (when that row spans intervals)
+  const int32_t* end_row; // per interval: row of its last entry (computed at create)
 };
 
 // Programmatic dependent launch (PDL): a kernel launched with the
@@ -850,8 +849,13 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
         for (int k = 0; k < CH; ++k) d[k] = int((W << ((CH * ch + k) * b)) >> (64 - b));
         if (ch == 0) {
           int tot = 0;  // sum of this lane's deltas (all T fields)
+          if constexpr (NC == 1) {
 #pragma unroll
-          for (int t = 0; t < TT; ++t) tot += int((W << (t * b)) >> (64 - b));
+            for (int k = 0; k < CH; ++k) tot += d[k];  // the chunk is the whole lane stream
+          } else {
+#pragma unroll
+            for (int t = 0; t < TT; ++t) tot += int((W << (t * b)) >> (64 - b));
+          }
           int incl = tot;
 #pragma unroll
           for (int off = 1; off < 32; off <<= 1) {
@@ -930,21 +934,34 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   }
   T cin = __shfl_up_sync(0xffffffffu, co, 1);
   if (!link) cin = T(0);
+  // Complete segments of rows other than the interval's first row go straight
+  // to y.  The first row F and the last row L go to y directly too unless they
+  // span intervals (known statically: F spans if the previous interval ends
+  // on F, L spans if the next one starts on L); then their partials are
+  // carried for the fix-up, which adds each spanning row once, in interval
+  // order.
+  T fpart = T(0);
+  bool hasF = false;
   auto emit = [&](int rr, T val) {
-    if (rr == first) p.cf[i] = val;
+    if (rr == first) { fpart = val; hasF = true; }
     else atomicAdd(y + rr, val);
   };
   if (!one) emit(f, A + cin);  // first segment complete inside this lane
   const int fnext = __shfl_down_sync(0xffffffffu, f, 1);
   if (lane < 31 && fnext != L) emit(L, co);  // trailing segment complete at this lane
-  if (lane == 31) {  // the interval's last row: its partial is carried
-    p.first_row[i] = first;
-    p.last_row[i] = L;
-    if (L == first) {
-      p.cf[i] = co;
-      p.cl[i] = T(0);
+  const unsigned mF = __ballot_sync(0xffffffffu, hasF);
+  const T Fp = mF ? __shfl_sync(0xffffffffu, fpart, __ffs(mF) - 1) : T(0);
+  if (lane == 31) {
+    const bool f_spans = i > 0 && p.end_row[i - 1] == first;
+    const bool l_spans = i + 1 < p.nI && int(p.base_row[i + 1]) == L;
+    if (L == first) {  // one row for the whole interval: its partial is co
+      if (f_spans || l_spans) p.cf[i] = co;
+      else atomicAdd(y + first, co);
     } else {
-      p.cl[i] = co;
+      if (f_spans) p.cf[i] = Fp;
+      else atomicAdd(y + first, Fp);
+      if (l_spans) p.cl[i] = co;
+      else atomicAdd(y + L, co);
     }
   }
 }
@@ -969,62 +986,30 @@ __global__ void replicate_y(int64_t m, const YOut<T> o) {
   }
 }
 
-// Deterministic application of the intervals' carries (one thread per
-// interval, fixed summation order = interval order).  first[u] / last[u] =
-// rows of the interval's first and last entries; cf = partial of the first
-// row (the whole interval if first == last), cl = partial of the last row.
-// acc += cf[j] for the intervals j = i+1, i+2, ... that continue row R
-// (first[j] == R), stopping after the first of them that ends on another
-// row.  Intervals are read 8 at a time (one round trip for rows spanning up
-// to 9 intervals); the additions stay in interval order.
+// Deterministic application of the carries of rows that span intervals: one
+// thread per such row (precomputed at create: row R, first interval a, last
+// interval b, whether R is a's last row or a starts with R), the partials
+// summed in interval order: (a's cl or cf) + cf[a+1] + ... + cf[b], added to
+// y[R] once.  The static span list is read before griddepcontrol.wait, so
+// only the carries are read after the COO kernel completes.
 template <typename T>
-__device__ __forceinline__ T chain_sum(int64_t i, int64_t nU, int R, T acc, const int32_t* __restrict__ first,
-                                       const int32_t* __restrict__ last_row, const T* __restrict__ cf) {
-  constexpr int B = 8;
-  for (int64_t j0 = i + 1; j0 < nU; j0 += B) {
-    int fj[B], lj[B];
-    T cj[B];
-#pragma unroll
-    for (int k = 0; k < B; ++k) {
-      const bool in = j0 + k < nU;
-      fj[k] = in ? first[j0 + k] : -1;
-      lj[k] = in ? last_row[j0 + k] : -1;
-      cj[k] = in ? cf[j0 + k] : T(0);
-    }
-    bool done = false;
-#pragma unroll
-    for (int k = 0; k < B; ++k) {
-      if (!done) {
-        if (fj[k] < 0) {
-          // an empty unit holds no row: skip it
-        } else if (fj[k] != R) {
-          done = true;
-        } else {
-          acc += cj[k];
-          done = lj[k] != R;
-        }
-      }
-    }
-    if (done) break;
-  }
-  return acc;
-}
-
-template <typename T>
-__global__ void coo_fixup(int64_t nU, const int32_t* __restrict__ first, const int32_t* __restrict__ last_row,
-                          const T* __restrict__ cf, const T* __restrict__ cl, T* __restrict__ y) {
-  const int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+__global__ void coo_fixup(int64_t nS, const int4* __restrict__ spans, const T* __restrict__ cf,
+                          const T* __restrict__ cl, T* __restrict__ y) {
+  const int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  int4 sp = make_int4(0, 0, -1, 0);
+  if (k < nS) sp = spans[k];  // {row, a, b, a_uses_cl}
   pdl_wait();  // the carries come from the COO kernel
-  if (i >= nU) return;
-  const int F = first[i];
-  const int L = last_row[i];
-  if (F < 0) return;  // an empty unit
-  if (L != F)  // unit i is the first one holding row L
-    y[L] += chain_sum<T>(i, nU, L, cl[i], first, last_row, cf);
-  int64_t j = i - 1;  // the previous non-empty unit
-  while (j >= 0 && first[j] < 0) --j;
-  if (j < 0 || last_row[j] != F)  // unit i is the first one holding row F
-    y[F] += L == F ? chain_sum<T>(i, nU, F, cf[i], first, last_row, cf) : cf[i];
+  if (k >= nS) return;
+  T sum = sp.w ? cl[sp.y] : cf[sp.y];
+  constexpr int B = 8;
+  for (int j0 = sp.y + 1; j0 <= sp.z; j0 += B) {
+    T c[B];
+#pragma unroll
+    for (int u = 0; u < B; ++u) c[u] = j0 + u <= sp.z ? cf[j0 + u] : T(0);
+#pragma unroll
+    for (int u = 0; u < B; ++u) sum += c[u];
+  }
+  y[sp.x] += sum;
 }
 
 }  // namespace dev
