@@ -784,7 +784,7 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   int f = 0, cr = 0;
   T A = T(0), cur = T(0);
   bool one = true;
-  int b = 0, S = 0, row = 0, first = 0, lim = 0;
+  int b = 0, S = 0, row = 0, first = 0, lim = 0, prev_end = -1, next_first = -1;
   uint32_t w0 = 0, w1 = 0;
   const uint32_t* wl = cwin[w] + lane;
 #pragma unroll
@@ -814,6 +814,10 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
       // wait for the width (width -> symptr -> words would be 3 round trips)
       first = int(p.base_row[i]);              // row of the interval's first entry
       row = first;
+      // boundary rows for the epilogue: does the first row continue from
+      // interval i-1, does the next interval start on this one's last row
+      prev_end = i > 0 ? p.end_row[i - 1] : -1;
+      next_first = i + 1 < p.nI ? int(p.base_row[i + 1]) : -1;
       if constexpr (kBro) {
         b = int(p.width[i]);
         const uint64_t q0 = p.symptr[i];
@@ -952,8 +956,8 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   const unsigned mF = __ballot_sync(0xffffffffu, hasF);
   const T Fp = mF ? __shfl_sync(0xffffffffu, fpart, __ffs(mF) - 1) : T(0);
   if (lane == 31) {
-    const bool f_spans = i > 0 && p.end_row[i - 1] == first;
-    const bool l_spans = i + 1 < p.nI && int(p.base_row[i + 1]) == L;
+    const bool f_spans = prev_end == first;
+    const bool l_spans = next_first == L;
     if (L == first) {  // one row for the whole interval: its partial is co
       if (f_spans || l_spans) p.cf[i] = co;
       else atomicAdd(y + first, co);

@@ -1,4 +1,4 @@
-OUT=gpurun_out/r02s; mkdir -p $OUT
+OUT=gpurun_out/r02t; mkdir -p $OUT
 python -c "import __graft_entry__ as g; g.build()" > $OUT/build.txt 2>&1 || { tail $OUT/build.txt; exit 1; }
 timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_gpu_dist.py -m gpu -q -p no:cacheprovider -x -k "coo_intervals or pdl or spmv_random or single or config4 or configs_full or scatter or deterministic or side_stream" > $OUT/pytest_q.txt 2>&1; echo "tests rc=$?"; tail -3 $OUT/pytest_q.txt
 timeout 600 python scripts/ab.py C4 f64 "coo_T=8" --baseline-opts "coo_T=8" > $OUT/ab_C4_f64.txt 2>&1; cat $OUT/ab_C4_f64.txt | cut -c1-120
