@@ -536,7 +536,7 @@ def main():
             "format": bro_name, "m": A.m, "n": A.n, "nnz": A.nnz,
             "vec_words": info["vec_words"], "slice_h": info["slice_h"], "coo_T": info["coo_T"],
             "ell_kernel": {0: None, 1: "tiny", 2: "few-slice", 3: "small-window", 4: "mid-window",
-                           5: "general"}[info["ell_kernel"]] if info["nnz_ell"] or fmt != "coo" else None,
+                           5: "general", 6: "split-4", 7: "split-2"}[info["ell_kernel"]] if info["nnz_ell"] or fmt != "coo" else None,
             "l2": ("flushed (2x L2 write) before every step" if args.flush_l2 else
                    ("inputs larger than L2" if alg_bytes > L2_BYTES else "L2-resident (warm)")),
             "parallelism": f"row-block x{world}" + (f" + {exch_info['exchange']} exchange of y per step (x_(k+1) = A.x_k)"

@@ -119,8 +119,13 @@ typedef struct {
   int32_t ell_kernel;/* BRO-ELL kernel instance: 0 (default) = chosen at create from the
                         matrix shape; 1 tiny (every slice <= 4 columns), 2 few-slice
                         (h = 32), 3 small window (every row stream < 10 symbols), 4 mid
-                        window (< 18), 5 general.  An instance the matrix does not fit
-                        gives BRO_ERR_ARG.  For A/B measurements and tests. */
+                        window (< 18), 5 general, 6 / 7 split slices (h = 32: 4 / 2 warps
+                        share each slice, each owning a range of its columns and
+                        decoding the columns before it without gathering; the block adds
+                        the partial sums in part order — the "multiple threads per row"
+                        of P:L416; at h = 64 they run the general instance).  An
+                        instance the matrix does not fit gives BRO_ERR_ARG.  For A/B
+                        measurements and tests. */
   int32_t pdl;       /* HYB / COO: 0 (default) = 1 = the COO kernel is launched as a
                         programmatic dependent of the ELL kernel (its loads, decode and x
                         gathers overlap the ELL kernel's tail; it waits before updating y),

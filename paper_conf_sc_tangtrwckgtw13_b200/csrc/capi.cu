@@ -619,7 +619,9 @@ cudaError_t launch_ell(const bro_matrix_s* A, int mode, const T* x, const bro::d
       const int64_t w = A->ell_x.k.warps_per_block();
       return launch_smem(A->ell_x, (p.s + w - 1) / w, size_t(A->xwin_bytes), st, p, y, dec);
     }
-    return launch(L, persistent_grid(L, p.s), st, p, y, dec);
+    // split instances: several warps per slice
+    const int64_t parts = A->h == 32 ? (A->ell_inst == bro::ELL_SPLIT ? 4 : A->ell_inst == bro::ELL_SPLIT2 ? 2 : 1) : 1;
+    return launch(L, persistent_grid(L, p.s * parts), st, p, y, dec);
   }
   // decode mode covers the padding rows [m, pitch) too (they hold -1)
   const int64_t rows = mode == 2 && b0 == 0 ? A->pitch : r1 - r0;

@@ -24,7 +24,7 @@ KernelRef ell_pick(int inst) {
   using namespace dev;
   constexpr bool f64 = sizeof(T) == 8;
   constexpr int SB = 4;  // symbol rows per staging round trip (measured best, profiles/r02/)
-  if (inst == ELL_FEW && R == 2) inst = ELL_GEN;
+  if ((inst == ELL_FEW || inst == ELL_SPLIT || inst == ELL_SPLIT2) && R == 2) inst = ELL_GEN;
   if constexpr (R == 1) {
     switch (inst) {
       case ELL_TINY: return {(const void*)&bro_ell_tiny<T, V, 1, 8, f64 ? 5 : 6, M>, 256};
@@ -42,6 +42,11 @@ KernelRef ell_pick(int inst) {
         if constexpr (f64) return {(const void*)&bro_ell_od<T, V, 1, 8, 5, 4, kEllRowsMid, M, 0, false, 0, false, SB>, 256};
         else return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsMid, M, 0, false, 0, false, SB>, 256};
       case ELL_GEN: return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsGen, M, 0, false, 0, false, SB>, 256};
+      // few long slices: 4 (SPLIT) or 2 (SPLIT2) warps per slice, 8-column groups, 32 warps/SM
+      case ELL_SPLIT:
+        return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsGen, M, 0, false, 0, false, SB, false, 4>, 256};
+      case ELL_SPLIT2:
+        return {(const void*)&bro_ell_od<T, V, 1, 8, 4, 8, kEllRowsGen, M, 0, false, 0, false, SB, false, 2>, 256};
     }
   } else {
     switch (inst) {

@@ -374,11 +374,20 @@ __device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
 // kPfAt: when the prefetch is issued — 0 at the slice start, k (1..3) once the
 // warp reaches column k*l/4 of the current slice (a later trigger keeps fewer
 // prefetched bytes waiting in L2 per warp, so more warps can prefetch).
+// kP > 1 (multiple warps per slice, the "multiple threads per row" of P:L416):
+// the kP adjacent warps of a block share one slice, warp `part` owning the
+// column range [part*cs, part*cs + cs) (cs = ceil(l / kP) rounded up to G).
+// A warp decodes the columns before its range without gathering (the column
+// index of a row is the prefix sum of its deltas), then the block adds the kP
+// partial sums of each row in part order (deterministic) and stores y.  For
+// matrices with few, long slices (C2): kP times more warps stream values.
 template <typename T, int V, int R, int kWarps, int kMinBlocks, int G, int kRows, int kMode, int kPf = 0,
-          bool kL1 = false, int kPfAt = 0, bool kPipe = false, int kSB = 0, bool kX = false>
+          bool kL1 = false, int kPfAt = 0, bool kPipe = false, int kSB = 0, bool kX = false, int kP = 1>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   static_assert(G % Chunk<T>::N == 0, "a column group holds whole 16-byte value chunks");
+  static_assert(kWarps % kP == 0 && (kP == 1 || (!kPipe && !kX && kPf == 0)), "split slices: plain groups only");
+  constexpr int kSl = kWarps / kP;  // slices per block per pass
   // symbol rows staged per round trip, sized by the instance's register
   // budget (16 / 12 / 8 loads in flight for >= 96 / >= 80 / fewer registers)
   constexpr int kMaxRegs = 65536 / (kWarps * 32 * kMinBlocks);
@@ -411,9 +420,17 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   }
   bool xready = !kX;
   const char* win_lane = reinterpret_cast<const char*>(win + lane * R);
-  const int64_t stride = int64_t(gridDim.x) * kWarps;
+  const int part = kP > 1 ? w % kP : 0;
+  __shared__ T psum[kP > 1 ? kWarps : 1][kP > 1 ? H : 1];  // split slices: partial sums per part
+  const int64_t stride = int64_t(gridDim.x) * kSl;
   int k32 = 0;
-  for (int64_t t = int64_t(blockIdx.x) * kWarps + w; t < p.s; t += stride, k32 = (k32 + 1) & 31) {
+  // block-uniform trip count (the split epilogue synchronises the block)
+  for (int64_t t0 = int64_t(blockIdx.x) * kSl; t0 < p.s; t0 += stride, k32 = (k32 + 1) & 31) {
+    const int64_t t = t0 + w / kP;
+    T sum[R];
+#pragma unroll
+    for (int k = 0; k < R; ++k) sum[k] = T(0);
+    if (t < p.s) {
     __syncwarp();
     if (k32 == 0) {  // one round trip fetches the metadata of the next 32 slices
       const int64_t tl = t + lane * stride;
@@ -443,12 +460,18 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
     const T* vs = p.vals + H * mt.c0;
     const uint8_t* ba = p.bit_alloc + mt.c0;
     const int lfull = (l / Chunk<T>::N) * Chunk<T>::N;
-    T sum[R];
     int col[R];
 #pragma unroll
-    for (int k = 0; k < R; ++k) { sum[k] = T(0); col[k] = -1; }
+    for (int k = 0; k < R; ++k) col[k] = -1;
+    // this warp's column range [j0, j1) of the slice (the whole slice if kP = 1)
+    int j0 = 0, j1 = l;
+    if constexpr (kP > 1) {
+      const int cs = ((l + kP - 1) / kP + G - 1) / G * G;
+      j0 = min(l, part * cs);
+      j1 = min(l, j0 + cs);
+    }
     int obase = 0;  // bit offset of the current block inside every row stream
-    for (int jb = 0; jb < l; jb += 32) {
+    for (int jb = 0; jb < j1; jb += 32) {
       const int nb = min(32, l - jb);
       const int b = lane < nb ? int(__ldg(ba + jb + lane)) : 0;
       if (jb == 0) {  // first block starts at symbol 0: stage without waiting for the scan
@@ -553,6 +576,20 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
       };
       if constexpr (!kPipe) {
         for (int g = 0; g < nb; g += G) {
+          if constexpr (kP > 1) {
+            if (jb + g >= j1) break;
+            if (jb + g < j0) {  // before this warp's range: advance the column indices only
+#pragma unroll
+              for (int kk = 0; kk < G; ++kk) {
+                const uint2 mm = cm[g + kk];
+                const uint32_t* wp = reinterpret_cast<const uint32_t*>(win_lane + mm.x);
+#pragma unroll
+                for (int k = 0; k < R; ++k)
+                  col[k] += int(shr_clamp(__funnelshift_l(wp[32 * R + k], wp[k], mm.y), mm.y >> 8));
+              }
+              continue;
+            }
+          }
           Grp q;
           issue(q, g);
           consume(q);
@@ -572,11 +609,29 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
       }
       obase += tot;
     }
+    }  // t < p.s
     if constexpr (kMode != kDecode) {
+      if constexpr (kP > 1) {  // partials of the slice's kP warps, added in part order
 #pragma unroll
-      for (int k = 0; k < R; ++k) {
-        const int64_t row = H * t + 32 * k + lane;
-        if (row < p.m) store_y<kMode>(y, row, sum[k]);
+        for (int k = 0; k < R; ++k) psum[w][32 * k + lane] = sum[k];
+        __syncthreads();
+        if (part == 0 && t < p.s) {
+#pragma unroll
+          for (int k = 0; k < R; ++k) {
+            T s = psum[w][32 * k + lane];
+#pragma unroll
+            for (int q = 1; q < kP; ++q) s += psum[w + q][32 * k + lane];
+            const int64_t row = H * t + 32 * k + lane;
+            if (row < p.m) store_y<kMode>(y, row, s);
+          }
+        }
+        __syncthreads();
+      } else if (t < p.s) {
+#pragma unroll
+        for (int k = 0; k < R; ++k) {
+          const int64_t row = H * t + 32 * k + lane;
+          if (row < p.m) store_y<kMode>(y, row, sum[k]);
+        }
       }
     }
   }

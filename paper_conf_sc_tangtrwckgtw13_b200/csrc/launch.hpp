@@ -13,7 +13,8 @@ struct KernelRef {
 };
 
 // BRO-ELL kernel instances (bro_opts_t.ell_kernel; 0 = chosen at create)
-enum EllInst { ELL_AUTO = 0, ELL_TINY = 1, ELL_FEW = 2, ELL_SMALL = 3, ELL_MID = 4, ELL_GEN = 5, ELL_LAST = 5 };
+enum EllInst { ELL_AUTO = 0, ELL_TINY = 1, ELL_FEW = 2, ELL_SMALL = 3, ELL_MID = 4, ELL_GEN = 5, ELL_SPLIT = 6,
+               ELL_SPLIT2 = 7, ELL_LAST = 7 };
 // the x-window-staged variant of the few-slice instance (bro_ell_xstage_ref)
 constexpr int kXStageMaxBytes = 96 * 1024;  // largest x window staged per block
 constexpr int kEllTinyCols = 4;   // TINY: every slice has <= 4 columns
