@@ -26,6 +26,12 @@ What it computes (citations are PAPER.md line numbers, "P:Lnnn"):
   metrics.py  space savings eta = 1 - C/O and compression ratio
               kappa = 1/(1-eta) (P:L246).
   bar.py      BRO-aware reordering: Eqn (1)-(3) and Algorithm 2.
+  value_index.py  value indexing of the BRO-ELL values: the "value data
+              compression" the conclusion names as future work, by
+              the value-index method of the work it cites ([16]):
+              distinct bit patterns + 1- or 2-byte codes in the slot layout
+              (reading R28; pinned by matrix A by hand, the stencil
+              closed form and a bitwise round trip).
 
 Every pin (tests/test_oracle_*.py, tests/golden/) ties these functions to
 something other than themselves: the paper's worked example, closed forms,
