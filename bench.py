@@ -57,7 +57,10 @@ def parse_args():
     ap.add_argument("--vec-words", type=int, default=0, help="0 = auto (fp64: 1, fp32: 4)")
     ap.add_argument("--slice-h", type=int, default=0, help="BRO-ELL slice height: 0 = auto, 32, 64")
     ap.add_argument("--coo-T", type=int, default=0, help="BRO-COO entries per lane: 0 = auto, 8, 16, 32")
-    ap.add_argument("--ell-kernel", type=int, default=0, help="BRO-ELL instance: 0 = auto, 1..5 (A/B only)")
+    ap.add_argument("--ell-kernel", type=int, default=0, help="BRO-ELL instance: 0 = auto, 1..7 (A/B only)")
+    ap.add_argument("--value-codec", type=int, default=0, choices=[0, 1],
+                    help="1 = value indexing of the BRO-ELL values (P:L416 future work, DESIGN reading R28); "
+                         "0 = the paper's BRO formats (default, the headline)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--flush-l2", action="store_true", help="write a 2xL2 buffer between steps")
@@ -269,7 +272,8 @@ def run_reference(args):
 
 def layout_opts(args):
     """BroMatrix layout options of the BRO handle (0 = the library's auto choice)."""
-    return {"slice_h": args.slice_h, "coo_T": args.coo_T, "ell_kernel": args.ell_kernel}
+    return {"slice_h": args.slice_h, "coo_T": args.coo_T, "ell_kernel": args.ell_kernel,
+            "value_codec": args.value_codec}
 
 
 def build_row_block(A, rank, world, dev, fmt, dtype, bounds, args, x_host, stream):
@@ -518,6 +522,8 @@ def main():
     if not args.no_cpu_baseline and world == 1:
         cpu = cpu_oracle_baseline(A, x_host)
     bro_name = {"ell": "BRO-ELL", "hyb": "BRO-HYB", "coo": "BRO-COO"}[fmt]
+    if info["value_code_bytes"]:
+        bro_name += " + value index"
     out = {
         "metric": METRIC,
         "value": value,
@@ -542,6 +548,8 @@ def main():
             "parallelism": f"row-block x{world}" + (f" + {exch_info['exchange']} exchange of y per step (x_(k+1) = A.x_k)"
                                                     if world > 1 else ""),
             "eta_stream": info["eta_stream"], "eta_total": info["eta_total"],
+            "value_codec": ({"codes": f"{info['value_code_bytes']}-byte", "distinct_values": info["value_dict_size"]}
+                            if info["value_code_bytes"] else None),
         },
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,

@@ -136,6 +136,18 @@ typedef struct {
                         window fits and one pass of blocks covers the matrix
                         (bro_info_t.x_stage_bytes > 0); 0 (default) = gathers through
                         L1/L2 (measured faster on C2: 19.5 vs 22.6 us fp64). */
+  int32_t value_codec;/* BRO-ELL values (codec 1, ELL and HYB handles): 0 (default) = stored
+                        as they are (the paper's BRO formats); 1 = value indexing, the
+                        "value data compression" named as future work by the
+                        value-index method of the work the paper cites for it ([16],
+                        P:L408; reading R28): the ELL part's distinct value
+                        bit patterns (sorted as unsigned integers) in a table and one
+                        1-byte (<= 256 distinct) or 2-byte (<= 65,536) code per slot,
+                        slot (r, j) of slice t at h*colptr[t] + place(r, j, l_t, 4/cb, h).
+                        Lossless bit for bit.  More than 65,536 distinct values gives
+                        BRO_ERR_UNSUPPORTED.  Value-indexed ELL handles have no scatter
+                        epilogue (bro_spmv_scatter with more than one destination gives
+                        BRO_ERR_UNSUPPORTED); the COO part of a HYB handle keeps its values. */
 } bro_opts_t;
 
 typedef struct {
@@ -165,6 +177,9 @@ typedef struct {
   double eta_stream;          /* 1 - C/O, C = compressed streams (+ raw COO col for HYB) */
   double eta_total;           /* 1 - index_bytes/O (metadata included) */
   double encode_seconds;      /* host time spent validating + encoding */
+  int32_t value_code_bytes;   /* value-indexed handles: bytes per code (1 or 2), else 0 */
+  int32_t reserved0;
+  int64_t value_dict_size;    /* value-indexed handles: distinct values |D| in the table, else 0 */
 } bro_info_t;
 
 /* Parts of the encoded representation, for bro_export_encoded. */
@@ -182,7 +197,9 @@ typedef enum {
   BRO_PART_COO_VALS = 10,     /* value[nI*32*T]  same arrangement, 0 past nnz */
   BRO_PART_COO_ROW = 11,      /* int32[nI*32*T]  plain COO rows (codec 0), last row past nnz */
   BRO_PART_PELL_COL = 12,     /* int32[K*pitch]  plain ELL, column-major, -1 = padding (codec 0) */
-  BRO_PART_PELL_VALS = 13     /* value[K*pitch]  plain ELL values (codec 0) */
+  BRO_PART_PELL_VALS = 13,    /* value[K*pitch]  plain ELL values (codec 0) */
+  BRO_PART_ELL_VCODES = 14,   /* uint8/uint16[h*colptr[s]]  value codes (value_codec 1), 4-byte chunks */
+  BRO_PART_ELL_VDICT = 15     /* value[|D|]  distinct values, bit patterns ascending (value_codec 1) */
 } bro_part_t;
 
 /* Fill *opts with the defaults: h 0 (auto), sym 32, V 0 (auto), T 0 (auto),

@@ -15,7 +15,8 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libbro.so")
-SOURCES = ["capi.cu", "kern_ell64.cu", "kern_ell32.cu", "kern_misc.cu", "encode.cpp"]
+SOURCES = ["capi.cu", "kern_ell64.cu", "kern_ell32.cu", "kern_ell64_vi.cu", "kern_ell32_vi.cu", "kern_misc.cu",
+           "encode.cpp"]
 HEADERS = ["kernels.cuh", "kern_ell.cuh", "launch.hpp", "encode.hpp", os.path.join("..", "..", "include", "bro.h")]
 OBJDIR = os.path.join(CSRC, "build")
 

@@ -25,7 +25,7 @@ STATUS = {0: "BRO_OK", 1: "BRO_ERR_ARG", 2: "BRO_ERR_INDEX", 3: "BRO_ERR_SHAPE",
 PARTS = {
     "ell_words": 0, "ell_bit_alloc": 1, "ell_colptr": 2, "ell_symptr": 3, "ell_vals": 4,
     "coo_words": 5, "coo_base_row": 6, "coo_width": 7, "coo_symptr": 8, "coo_col": 9,
-    "coo_vals": 10, "coo_row": 11, "pell_col": 12, "pell_vals": 13,
+    "coo_vals": 10, "coo_row": 11, "pell_col": 12, "pell_vals": 13, "ell_vcodes": 14, "ell_vdict": 15,
 }
 FORMATS = {0: "ELL", 1: "COO", 2: "HYB"}
 
@@ -34,7 +34,7 @@ class bro_opts_t(C.Structure):
     _fields_ = [("slice_h", C.c_int32), ("sym_bits", C.c_int32), ("vec_words", C.c_int32),
                 ("coo_T", C.c_int32), ("hyb_K", C.c_int64), ("codec", C.c_int32),
                 ("min_bits", C.c_int32), ("ell_kernel", C.c_int32), ("pdl", C.c_int32),
-                ("x_stage", C.c_int32)]
+                ("x_stage", C.c_int32), ("value_codec", C.c_int32)]
 
 
 class bro_info_t(C.Structure):
@@ -49,7 +49,8 @@ class bro_info_t(C.Structure):
                 ("meta_bytes", C.c_int64), ("index_bytes", C.c_int64), ("value_bytes", C.c_int64),
                 ("device_bytes", C.c_int64), ("algorithmic_bytes", C.c_int64),
                 ("orig_index_bytes", C.c_int64), ("eta_stream", C.c_double),
-                ("eta_total", C.c_double), ("encode_seconds", C.c_double)]
+                ("eta_total", C.c_double), ("encode_seconds", C.c_double),
+                ("value_code_bytes", C.c_int32), ("reserved0", C.c_int32), ("value_dict_size", C.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -190,7 +191,7 @@ def bro_get_info(h: int) -> dict:
 
 
 _PART_DTYPES = {0: np.uint32, 1: np.uint8, 2: np.uint64, 3: np.uint64, 5: np.uint32, 6: np.uint32,
-                7: np.uint8, 8: np.uint64, 9: np.int32, 11: np.int32, 12: np.int32}
+                7: np.uint8, 8: np.uint64, 9: np.int32, 11: np.int32, 12: np.int32, 14: np.uint8}
 
 
 def bro_export_encoded(h: int, part, value_dtype=None) -> np.ndarray:
@@ -247,13 +248,13 @@ class BroMatrix:
     pointers reach the library (the C ABI cannot)."""
 
     def __init__(self, A, fmt="ell", codec=1, device=0, dtype=None, vec_words=0, hyb_K=-1, min_bits=0,
-                 slice_h=0, coo_T=0, ell_kernel=0, pdl=0, x_stage=0):
+                 slice_h=0, coo_T=0, ell_kernel=0, pdl=0, x_stage=0, value_codec=0):
         vals = A.vals if dtype is None else A.vals.astype(dtype)
         self.dtype = np.dtype(vals.dtype)
         self.m, self.n, self.fmt, self.device = A.m, A.n, fmt, device
         opts = bro_opts_default(codec=codec, vec_words=vec_words, hyb_K=hyb_K, min_bits=min_bits,
                                 slice_h=slice_h, coo_T=coo_T, ell_kernel=ell_kernel, pdl=pdl,
-                                x_stage=x_stage)
+                                x_stage=x_stage, value_codec=value_codec)
         if fmt == "ell":
             self.h = bro_create_ell(device, A.m, A.n, A.row_ptr, A.col, vals, opts)
         elif fmt == "hyb":

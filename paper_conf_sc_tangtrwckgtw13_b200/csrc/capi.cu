@@ -69,6 +69,10 @@ struct bro_matrix_s {
   int h = 32;       // BRO-ELL slice height (rows of a row block of the plain ELL)
   int coo_T = 32;   // COO entries per lane of an interval
   int ell_inst = 0; // BRO-ELL kernel instance (launch.hpp EllInst)
+  // value index of the BRO-ELL part (opts.value_codec = 1, reading R28)
+  bro::ValueIndexCode vi;
+  uint8_t* d_vcodes = nullptr;
+  void* d_vdict = nullptr;
   // host encodings (kept only by host-only handles after create)
   bro::EllCode ell;
   bro::PlainEll pell;
@@ -148,7 +152,7 @@ void free_device(bro_matrix_s* A) {
   void* ps[] = {A->d_words, A->d_bit_alloc, A->d_colptr, A->d_symptr, A->d_ell_vals, A->d_pell_col,
                 A->d_coo_words, A->d_coo_base, A->d_coo_width, A->d_coo_symptr, A->d_coo_row,
                 A->d_coo_col, A->d_coo_vals, A->d_cf, A->d_cl, A->d_coo_end, A->d_spans, A->d_xs, A->d_ys,
-                A->d_xwin};
+                A->d_xwin, A->d_vcodes, A->d_vdict};
   for (void* p : ps)
     if (p) cudaFree(p);
   for (cudaEvent_t e : A->e2e_ev) cudaEventDestroy(e);
@@ -169,6 +173,8 @@ bro_status_t check_opts(const bro_opts_t& o) {
   if (o.min_bits < 0 || o.min_bits > 31) return fail(BRO_ERR_ARG, "min_bits must be in [0, 31]");
   if (o.pdl < 0 || o.pdl > 2) return fail(BRO_ERR_ARG, "pdl must be 0, 1 or 2");
   if (o.x_stage < 0 || o.x_stage > 1) return fail(BRO_ERR_ARG, "x_stage must be 0 or 1");
+  if (o.value_codec < 0 || o.value_codec > 1) return fail(BRO_ERR_ARG, "value_codec must be 0 or 1");
+  if (o.value_codec == 1 && o.codec != 1) return fail(BRO_ERR_ARG, "value_codec 1 needs codec 1 (BRO-ELL values)");
   if (o.ell_kernel < 0 || o.ell_kernel > bro::ELL_LAST)
     return fail(BRO_ERR_ARG, "ell_kernel must be in [0, " + std::to_string(bro::ELL_LAST) + "]");
   return BRO_OK;
@@ -197,7 +203,13 @@ void fill_info(bro_matrix_s* A, double secs) {
       I.ell_stream_bytes = 4 * A->ell_words;
       meta += 16 * (A->s + 1) + (A->s ? int64_t(A->ell_slots / A->h) : 0);  // colptr, symptr, bit_alloc
       stream += I.ell_stream_bytes;
-      values += A->ell_slots * vs;
+      if (A->vi.cb) {  // value index: codes per slot + the table
+        values += A->ell_slots * A->vi.cb + A->vi.nd * vs;
+        I.value_code_bytes = A->vi.cb;
+        I.value_dict_size = A->vi.nd;
+      } else {
+        values += A->ell_slots * vs;
+      }
     } else {
       I.ell_slots = A->K * A->pitch;
       raw_index += 4 * A->K * A->pitch;
@@ -308,9 +320,13 @@ bro_status_t resolve_kernels(bro_matrix_s* A) {
   if (A->has_ell) {
     if (A->opts.codec) {
       if ((st = choose_ell_instance(A, sms))) return st;
-      for (int mode = 0; mode < 3 && !st; ++mode)
-        st = resolve(A->ell_k[mode], bro::bro_ell_ref<T>(V, A->h / 32, A->ell_inst, mode), sms, "BRO-ELL");
-      if (!st && A->xwin_bytes > 0 && A->ell_inst == bro::ELL_FEW) st = resolve_xstage<T>(A, sms);
+      for (int mode = 0; mode < 3 && !st; ++mode) {
+        if (A->vi.cb && mode == 1) continue;  // value-indexed handles: no scatter epilogue
+        const bro::KernelRef k = A->vi.cb && mode == 0 ? bro::bro_ell_vi_ref<T>(V, A->h / 32, A->ell_inst, A->vi.cb)
+                                                        : bro::bro_ell_ref<T>(V, A->h / 32, A->ell_inst, mode);
+        st = resolve(A->ell_k[mode], k, sms, "BRO-ELL");
+      }
+      if (!st && A->xwin_bytes > 0 && A->ell_inst == bro::ELL_FEW && !A->vi.cb) st = resolve_xstage<T>(A, sms);
     } else {
       for (int mode = 0; mode < 3 && !st; ++mode) st = resolve(A->ell_k[mode], bro::plain_ell_ref<T>(mode), sms, "ELL");
     }
@@ -372,6 +388,10 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
         A->ell_max_l = A->ell.max_l;
         for (int64_t t = 0; t < A->s; ++t)
           A->ell_max_S = std::max<int64_t>(A->ell_max_S, int64_t(A->ell.symptr[t + 1] - A->ell.symptr[t]));
+        if (o.value_codec == 1 && !bro::encode_value_index(rv, A->ell, A->vi)) {
+          delete A;
+          return fail(BRO_ERR_UNSUPPORTED, "value_codec 1: the BRO-ELL part holds more than 65,536 distinct values");
+        }
       } else {
         bro::build_plain_ell(rv, K, A->pell);
         A->pitch = A->pell.pitch;
@@ -481,7 +501,12 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
       UP(A->d_bit_alloc, A->ell.bit_alloc);
       UP(A->d_colptr, A->ell.colptr);
       UP(A->d_symptr, A->ell.symptr);
-      if (st == BRO_OK) st = dev_upload(A, &A->d_ell_vals, A->ell.vals.data(), A->ell.vals.size());
+      if (A->vi.cb) {  // the codes and the table replace the values
+        UP(A->d_vcodes, A->vi.codes);
+        if (st == BRO_OK) st = dev_upload(A, &A->d_vdict, A->vi.dict.data(), A->vi.dict.size());
+      } else if (st == BRO_OK) {
+        st = dev_upload(A, &A->d_ell_vals, A->ell.vals.data(), A->ell.vals.size());
+      }
     }
     if (A->xwin_bytes > 0) UP(A->d_xwin, A->xwin_host);
     if (A->has_ell && !o.codec) {
@@ -522,6 +547,8 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
     A->coo = bro::CooCode();
     A->coo_end_host = std::vector<int32_t>();
     A->spans_host = std::vector<int4>();
+    A->vi.codes = std::vector<uint8_t>();
+    A->vi.dict = bro::Bytes();
   } else {
     if (A->has_ell && o.codec) {
       bro_status_t st = choose_ell_instance(A, 148);
@@ -613,7 +640,9 @@ cudaError_t launch_ell(const bro_matrix_s* A, int mode, const T* x, const bro::d
   const Launch& L = A->ell_k[mode];
   if (A->opts.codec) {
     bro::dev::EllDev<T> p{r1 - r0, b1 - b0, A->d_words, A->d_bit_alloc, A->d_colptr + b0, A->d_symptr + b0,
-                          static_cast<const T*>(A->d_ell_vals), x, A->d_xwin};
+                          static_cast<const T*>(A->d_ell_vals), x, A->d_xwin, A->d_vcodes,
+                          static_cast<const T*>(A->d_vdict)};
+    if (!L.k.fn) return cudaErrorNotSupported;  // scatter on a value-indexed handle
     // whole part, plain SpMV, 16-byte aligned x: the x-window-staged instance
     if (A->xstage && mode == 0 && b0 == 0 && b1 == A->s && (reinterpret_cast<uintptr_t>(x) & 15) == 0) {
       const int64_t w = A->ell_x.k.warps_per_block();
@@ -706,7 +735,9 @@ PartView part_view(bro_matrix_s* A, int32_t part) {
     case BRO_PART_ELL_BIT_ALLOC: if (bro_ell) set(A->ell.bit_alloc.data(), A->d_bit_alloc, size_t(A->ell_slots) / H); break;
     case BRO_PART_ELL_COLPTR: if (bro_ell) set(A->ell.colptr.data(), A->d_colptr, 8 * size_t(A->s + 1)); break;
     case BRO_PART_ELL_SYMPTR: if (bro_ell) set(A->ell.symptr.data(), A->d_symptr, 8 * size_t(A->s + 1)); break;
-    case BRO_PART_ELL_VALS: if (bro_ell) set(A->ell.vals.data(), A->d_ell_vals, vs * size_t(A->ell_slots)); break;
+    case BRO_PART_ELL_VALS: if (bro_ell && !A->vi.cb) set(A->ell.vals.data(), A->d_ell_vals, vs * size_t(A->ell_slots)); break;
+    case BRO_PART_ELL_VCODES: if (bro_ell && A->vi.cb) set(A->vi.codes.data(), A->d_vcodes, A->vi.codes.size()); break;
+    case BRO_PART_ELL_VDICT: if (bro_ell && A->vi.cb) set(A->vi.dict.data(), A->d_vdict, A->vi.dict.size()); break;
     case BRO_PART_COO_WORDS: if (bro_coo) set(A->coo.words.data(), A->d_coo_words, 4 * size_t(A->coo_words)); break;
     case BRO_PART_COO_BASE_ROW: if (bro_coo) set(A->coo.base_row.data(), A->d_coo_base, 4 * size_t(A->nI)); break;
     case BRO_PART_COO_WIDTH: if (bro_coo) set(A->coo.width.data(), A->d_coo_width, size_t(A->nI)); break;
@@ -805,6 +836,7 @@ void bro_opts_default(bro_opts_t* o) {
   o->ell_kernel = 0;
   o->pdl = 0;
   o->x_stage = 0;
+  o->value_codec = 0;
 }
 
 bro_status_t bro_create_ell(int device, bro_dtype_t dtype, int64_t m, int64_t n, const int64_t* row_ptr,
@@ -875,6 +907,8 @@ bro_status_t bro_spmv_scatter(bro_matrix_t A, const void* x, void* const* y_dsts
     if (y_dsts[i] == x && A->m > 0) return fail(BRO_ERR_ARG, "x and a y destination must not alias");
   }
   if (y_mc && y_mc == x && A->m > 0) return fail(BRO_ERR_ARG, "x and the multicast y must not alias");
+  if (A->vi.cb && !(A->has_coo && A->nI > 0) && (n_dst > 1 || y_mc))
+    return fail(BRO_ERR_UNSUPPORTED, "value-indexed BRO-ELL handles have no scatter epilogue");
   DeviceGuard g(A->device);
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   auto run = [&](auto* tag) {

@@ -215,6 +215,69 @@ void encode_bro_ell(const RowsView& A, int h, int V, int VV, int min_bits, EllCo
   });
 }
 
+template <typename U>
+static bool value_index_impl(const RowsView& A, const EllCode& E, ValueIndexCode& out) {
+  constexpr size_t kMaxD = 65536;
+  const int64_t m = A.m;
+  const int nt = num_threads();
+  // distinct bit patterns per thread (early exit past 65,536), then merged
+  std::vector<std::unordered_set<U>> sets(nt);
+  std::vector<char> over(nt, 0);
+  {
+    std::vector<std::thread> th;
+    for (int c = 0; c < nt; ++c) {
+      th.emplace_back([&, c] {
+        const int64_t lo = m * c / nt, hi = m * (c + 1) / nt;
+        auto& st = sets[c];
+        for (int64_t r = lo; r < hi && !over[c]; ++r) {
+          const U* v = reinterpret_cast<const U*>(A.vals) + A.row_ptr[r];
+          for (int64_t j = 0, len = A.len(r); j < len; ++j) st.insert(v[j]);
+          if (st.size() > kMaxD) over[c] = 1;
+        }
+      });
+    }
+    for (auto& t : th) t.join();
+  }
+  std::unordered_set<U> all;
+  for (int c = 0; c < nt; ++c) {
+    if (over[c]) return false;
+    all.insert(sets[c].begin(), sets[c].end());
+    if (all.size() > kMaxD) return false;
+  }
+  std::vector<U> D(all.begin(), all.end());
+  std::sort(D.begin(), D.end());  // ascending as unsigned integers
+  const int cb = D.size() <= 256 ? 1 : 2;
+  const int64_t VC = 4 / cb;
+  const int64_t h = E.h, s = E.s;
+  out.cb = cb;
+  out.nd = int64_t(D.size());
+  out.dict.resize(D.size() * sizeof(U));
+  if (!D.empty()) std::memcpy(out.dict.data(), D.data(), D.size() * sizeof(U));
+  out.codes.assign(size_t(cb) * h * E.colptr[s], 0);
+  parallel_for(s, [&](int64_t lo, int64_t hi) {
+    for (int64_t t = lo; t < hi; ++t) {
+      const int64_t l = int64_t(E.colptr[t + 1] - E.colptr[t]);
+      uint8_t* base = out.codes.data() + size_t(cb) * h * E.colptr[t];
+      for (int64_t lane = 0; lane < h; ++lane) {
+        const int64_t r = t * h + lane;
+        if (r >= m) break;
+        const U* v = reinterpret_cast<const U*>(A.vals) + A.row_ptr[r];
+        for (int64_t j = 0, len = A.len(r); j < len; ++j) {
+          const uint32_t code = uint32_t(std::lower_bound(D.begin(), D.end(), v[j]) - D.begin());
+          uint8_t* dst = base + size_t(cb) * place(lane, j, l, VC, h);
+          dst[0] = uint8_t(code);
+          if (cb == 2) dst[1] = uint8_t(code >> 8);
+        }
+      }
+    }
+  });
+  return true;
+}
+
+bool encode_value_index(const RowsView& A, const EllCode& E, ValueIndexCode& out) {
+  return A.vsize == 8 ? value_index_impl<uint64_t>(A, E, out) : value_index_impl<uint32_t>(A, E, out);
+}
+
 void slice_extents(const RowsView& A, int h, int min_bits, int64_t* max_l, int64_t* max_S) {
   const int64_t m = A.m;
   const int64_t s = (m + h - 1) / h;

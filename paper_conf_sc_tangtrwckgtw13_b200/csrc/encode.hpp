@@ -63,6 +63,18 @@ struct CooCode {
   Bytes vals;                     // nI*32T
 };
 
+// Value index of a BRO-ELL part (reading R28: the value compression of
+// P:L416 by the value-index method of [16]): the distinct bit
+// patterns of the stored values, sorted as unsigned integers, and one code of
+// cb bytes per slot, slot (r, j) of slice t at h*colptr[t] + place(r, j, l_t,
+// 4/cb, h) (padding 0).
+struct ValueIndexCode {
+  int cb = 0;                     // 1 or 2 bytes per code
+  int64_t nd = 0;                 // |D|
+  Bytes dict;                     // nd values (bit patterns ascending)
+  std::vector<uint8_t> codes;     // cb*h*colptr[s] bytes, little-endian codes
+};
+
 struct PlainEll {                 // ELLPACK, column-major
   int64_t K = 0, pitch = 0;
   std::vector<int32_t> col;       // K*pitch, -1 = padding
@@ -87,6 +99,9 @@ std::string check_coo(int64_t m, int64_t n, int64_t nnz, const int32_t* row, con
 int64_t hyb_K(int64_t m, const int64_t* row_ptr);
 
 void encode_bro_ell(const RowsView& A, int h, int V, int value_chunk, int min_bits, EllCode& out);
+// Value index of the BRO-ELL part E of A; false (out untouched) if the part
+// holds more than 65,536 distinct values.
+bool encode_value_index(const RowsView& A, const EllCode& E, ValueIndexCode& out);
 // Longest slice (columns) and longest row stream (32-bit symbols) of the
 // BRO-ELL encoding at slice height h, without packing anything.
 void slice_extents(const RowsView& A, int h, int min_bits, int64_t* max_l, int64_t* max_S);

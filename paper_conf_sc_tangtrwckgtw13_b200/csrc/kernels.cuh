@@ -182,6 +182,8 @@ struct EllDev {           // a BRO-ELL part (or a range of its slices)
   const T* vals;
   const T* x;
   const int2* xwin;       // x-staged instances: per block, {first column, columns} of its x window
+  const uint8_t* vcodes;  // value-indexed handles (reading R28): codes in the slot layout, 4-byte chunks
+  const T* vdict;         // ... and the table of distinct values they index
 };
 
 // ------------------------------------------------------------------ TMA bulk copy + mbarrier
@@ -269,6 +271,50 @@ __device__ __forceinline__ void load_vals(T* v, const T* vs, int j, int l, int l
       }
     }
   }
+}
+
+// Value indexing (reading R28, the "value data compression" of P:L416 by the
+// value-index method of [16]): the G values of row r are codes of CB bytes in
+// 4-byte chunks of 4/CB codes (slot layout, P:L116 multiplexing), looked up in
+// the table of distinct values (a few KB at most: L1-resident).
+template <int CB>
+__device__ __forceinline__ uint32_t ld_code(const uint8_t* p) {
+  uint32_t r;
+  if constexpr (CB == 1) asm("ld.global.nc.L1::no_allocate.u8 %0, [%1];" : "=r"(r) : "l"(p));
+  else asm("ld.global.nc.L1::no_allocate.u16 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+template <typename T, int G, int H, int CB>
+__device__ __forceinline__ void load_vals_vi(T* v, const uint8_t* cs, const T* __restrict__ dict, int j, int l,
+                                             int r) {
+  constexpr int VC = 4 / CB;
+  static_assert(G % VC == 0, "a column group holds whole 4-byte code chunks");
+  const int lfull = (l / VC) * VC;
+  uint32_t code[G];
+  auto chunk = [&](int u, int jj) {
+    const uint32_t w = ld_stream_u32(reinterpret_cast<const uint32_t*>(cs + CB * (H * jj + r * VC)));
+#pragma unroll
+    for (int q = 0; q < VC; ++q) code[u * VC + q] = CB == 1 ? (w >> (8 * q)) & 0xffu : (w >> (16 * q)) & 0xffffu;
+  };
+  if (j + G <= lfull) {
+#pragma unroll
+    for (int u = 0; u < G / VC; ++u) chunk(u, j + u * VC);
+  } else {
+    const int tw = l - lfull;  // tail codes per row (< VC), contiguous per row
+#pragma unroll
+    for (int u = 0; u < G / VC; ++u) {
+      const int jj = j + u * VC;
+      if (jj + VC <= lfull) {
+        chunk(u, jj);
+      } else {
+#pragma unroll
+        for (int k = 0; k < VC; ++k)
+          code[u * VC + k] = jj + k < l ? ld_code<CB>(cs + CB * (H * lfull + r * tw + (jj + k - lfull))) : 0u;
+      }
+    }
+  }
+#pragma unroll
+  for (int k = 0; k < G; ++k) v[k] = __ldg(dict + code[k]);
 }
 
 // Copy symbol rows [qa, qa + nrows) of this lane's R rows into
@@ -382,7 +428,8 @@ __device__ __forceinline__ void prefetch_l2(const void* p, uint32_t bytes) {
 // partial sums of each row in part order (deterministic) and stores y.  For
 // matrices with few, long slices (C2): kP times more warps stream values.
 template <typename T, int V, int R, int kWarps, int kMinBlocks, int G, int kRows, int kMode, int kPf = 0,
-          bool kL1 = false, int kPfAt = 0, bool kPipe = false, int kSB = 0, bool kX = false, int kP = 1>
+          bool kL1 = false, int kPfAt = 0, bool kPipe = false, int kSB = 0, bool kX = false, int kP = 1,
+          int kVI = 0>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   static_assert(G % Chunk<T>::N == 0, "a column group holds whole 16-byte value chunks");
@@ -446,10 +493,11 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
       if (lane == 0 && k32 + kPf < 32 && t + kPf * stride < p.s) {
         const Meta nx = metas[w][k32 + kPf];
         if (nx.l > 0) {
-          prefetch_l2(p.vals + H * nx.c0, uint32_t(H * nx.l * sizeof(T)));
+          if constexpr (kVI == 0) prefetch_l2(p.vals + H * nx.c0, uint32_t(H * nx.l * sizeof(T)));
           prefetch_l2(p.words + H * nx.q0, uint32_t(H * nx.S * 4));
           const uint64_t b0 = nx.c0 & ~uint64_t(15), b1 = (nx.c0 + uint64_t(nx.l) + 15) & ~uint64_t(15);
           prefetch_l2(p.bit_alloc + b0, uint32_t(b1 - b0));
+          if constexpr (kVI > 0) prefetch_l2(p.vcodes + kVI * H * nx.c0, uint32_t((kVI * H * nx.l + 15) & ~15));
         }
       }
     };
@@ -458,6 +506,7 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
     const int S = mt.S;
     const uint32_t* wb = p.words + H * mt.q0;
     const T* vs = p.vals + H * mt.c0;
+    const uint8_t* vcs = kVI > 0 ? p.vcodes + kVI * H * mt.c0 : nullptr;
     const uint8_t* ba = p.bit_alloc + mt.c0;
     const int lfull = (l / Chunk<T>::N) * Chunk<T>::N;
     int col[R];
@@ -512,7 +561,10 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
         }
         if constexpr (kMode != kDecode) {
 #pragma unroll
-          for (int k = 0; k < R; ++k) load_vals<T, G, H>(q.v[k], vs, jb + g, l, lfull, 32 * k + lane);
+          for (int k = 0; k < R; ++k) {
+            if constexpr (kVI > 0) load_vals_vi<T, G, H, kVI>(q.v[k], vcs, p.vdict, jb + g, l, 32 * k + lane);
+            else load_vals<T, G, H>(q.v[k], vs, jb + g, l, lfull, 32 * k + lane);
+          }
         }
 #pragma unroll
         for (int kk = 0; kk < G; ++kk) {
@@ -645,7 +697,7 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
 // together, then one fetches the x gathers.  Field j starts at the
 // warp-uniform offset o_j = b_0 + ... + b_{j-1}, so q = o_j / 32 selects the
 // word pair uniformly.
-template <typename T, int V, int R, int kWarps, int kMinBlocks, int kMode>
+template <typename T, int V, int R, int kWarps, int kMinBlocks, int kMode, int kVI = 0>
 __global__ void __launch_bounds__(kWarps * 32, kMinBlocks)
 bro_ell_tiny(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   constexpr int H = 32 * R;
@@ -683,7 +735,10 @@ bro_ell_tiny(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
       for (int q = 0; q < 4; ++q) wd[k][q] = q < S ? ld_stream_u32(wb + place(row, q, S, V, H)) : 0u;
       wd[k][4] = 0u;
       if constexpr (kMode != kDecode) {
-        if (l > 0) load_vals<T, 4, H>(v[k], p.vals + H * mt.c0, 0, l, lfull, row);
+        if (l > 0) {
+          if constexpr (kVI > 0) load_vals_vi<T, 4, H, kVI>(v[k], p.vcodes + kVI * H * mt.c0, p.vdict, 0, l, row);
+          else load_vals<T, 4, H>(v[k], p.vals + H * mt.c0, 0, l, lfull, row);
+        }
       }
     }
     int cidx[R][4];

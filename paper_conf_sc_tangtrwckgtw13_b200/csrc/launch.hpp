@@ -25,6 +25,7 @@ constexpr int kEllRowsGen = 34;   // GEN:   any
 // mode: 0 = y = A.x, 1 = scatter (y into every destination), 2 = decode
 template <typename T> KernelRef bro_ell_ref(int V, int R, int inst, int mode);
 template <typename T> KernelRef bro_ell_xstage_ref(int V);  // few-slice instance, x window in shared memory
+template <typename T> KernelRef bro_ell_vi_ref(int V, int R, int inst, int cb);  // value-indexed, spmv mode
 template <typename T> KernelRef plain_ell_ref(int mode);
 template <typename T> KernelRef coo_ref(bool bro, int TT, int mode);  // mode 0 or 2
 template <typename T> KernelRef fixup_ref();

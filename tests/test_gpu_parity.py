@@ -460,3 +460,86 @@ def test_x_window_staging(lib, dev, dtype):
         assert np.array_equal(yd.cpu().numpy(), ys[1])
         for M in Ms:
             M.close()
+
+
+@pytest.mark.parametrize("inst", [1, 2, 3, 4, 5, 6, 7])
+@pytest.mark.parametrize("h", [32, 64])
+@pytest.mark.parametrize("V", [1, 4])
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_value_index_instances(lib, dev, inst, h, V, dtype):
+    """value_codec 1 (reading R28) through every BRO-ELL instance, ELL and HYB
+    handles, 1-byte and 2-byte codes: y on every row within the oracle's bound
+    AND bit-identical to the same instance reading the stored values (the
+    table returns the same bits, the FMAs run in the same order); decode mode
+    bit-exact."""
+    ran = 0
+    for k, (name, mk) in enumerate(INSTANCE_CASES):
+        A = mk()
+        if A.nnz == 0 or A.n > 2**24:
+            continue
+        rng = np.random.default_rng(k)
+        pool = rng.uniform(-1, 1, 3 if k % 2 else 300)
+        A = Csr(A.m, A.n, A.row_ptr, A.col, pool[rng.integers(0, pool.size, A.nnz)], A.name)
+        for fmt in ("ell", "hyb"):
+            if fmt == "hyb":
+                K = hyb.hyb_K(A.row_ptr)
+                ep, ec, ev, _, _, _ = hyb.hyb_split(A.row_ptr, A.col, A.vals, K)
+                E = Csr(A.m, A.n, ep, ec, ev)
+            else:
+                E = A
+            if not _fits(E, h, inst):
+                continue
+            x = make_x(A.n, 9, dtype)
+            M, _, y = _run(lib, A, fmt, 1, dtype, dev, x=x, vec_words=V, slice_h=h, ell_kernel=inst, value_codec=1)
+            assert M.info["value_code_bytes"] == (1 if M.info["value_dict_size"] <= 256 else 2)
+            _check_y(A, x, y, dtype)
+            check_decode(M, A)
+            M.close()
+            Mp, _, yp = _run(lib, A, fmt, 1, dtype, dev, x=x, vec_words=V, slice_h=h, ell_kernel=inst)
+            Mp.close()
+            assert np.array_equal(y.view(np.uint8), yp.view(np.uint8)), f"{name} {fmt}: not bit-identical"
+            ran += 1
+    assert ran > 0
+
+
+def test_value_index_scatter_rejected(lib, dev):
+    """A value-indexed ELL handle has no scatter epilogue: more than one
+    destination is BRO_ERR_UNSUPPORTED (one destination is a plain SpMV)."""
+    A = make_config(1)
+    M = lib.BroMatrix(A, fmt="ell", codec=1, device=0, value_codec=1)
+    x = torch.from_numpy(make_x(A.n, 1)).to(dev)
+    ys = [torch.empty(A.m, dtype=torch.float64, device=dev) for _ in range(2)]
+    with pytest.raises(lib.BroError, match="UNSUPPORTED"):
+        M.spmv_scatter(x, [t.data_ptr() for t in ys])
+    M.spmv_scatter(x, [ys[0].data_ptr()])
+    torch.cuda.synchronize()
+    assert torch.equal(ys[0], M.spmv(x))
+    M.close()
+
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_config5_value_index(lib, dev, dtype):
+    """C5 with value indexing (D = {26, -1}, 1-byte codes) in bench.py's
+    launch configuration: x = 1 gives y_i = 27 - len_i exactly; random x:
+    bit-identical to the stored-values BRO-ELL handle (whose every row
+    test_config5_full_size checks against the oracle) and every row against
+    the oracle on 3 chunks."""
+    A = make_config(5, dtype)
+    M = lib.BroMatrix(A, fmt="ell", codec=1, device=0, dtype=dtype, value_codec=1)
+    assert M.info["value_code_bytes"] == 1 and M.info["value_dict_size"] == 2
+    tdt = torch.float64 if dtype == np.float64 else torch.float32
+    y = M.spmv(torch.ones(A.n, dtype=tdt, device=dev)).cpu().numpy()
+    assert np.array_equal(y, (27.0 - A.row_lengths()).astype(dtype))
+    x = make_x(A.n, 5, dtype)
+    xd = torch.from_numpy(x).to(dev)
+    y = M.spmv(xd).cpu().numpy()
+    M.close()
+    P = lib.BroMatrix(A, fmt="ell", codec=1, device=0, dtype=dtype)
+    yp = P.spmv(xd).cpu().numpy()
+    P.close()
+    assert np.array_equal(y.view(np.uint8), yp.view(np.uint8))
+    for r0 in (0, 3_500_000, A.m - 500_000):
+        B = row_block(A, r0, r0 + 500_000)
+        y_ref, S = spmv.csr_spmv(B.row_ptr, B.col, B.vals, x)
+        ok, _ = spmv.within_tolerance(y[r0:r0 + 500_000], y_ref, S, TOL[dtype])
+        assert ok.all()

@@ -490,3 +490,50 @@ def test_bar_method3_matches_oracle(lib, seed, m):
     perm = lib.bro_reorder_bar(A.m, A.n, A.row_ptr, A.col, method=3, window=8)
     order = bar.signature_order(A.row_ptr, A.col, A.m)
     assert np.array_equal(perm, bar.algorithm2(A.row_ptr, A.col, A.m, h=32, window=8, order=order))
+
+
+@pytest.mark.parametrize("h", [32, 64])
+@pytest.mark.parametrize("nd", [2, 200, 3000])
+@pytest.mark.parametrize("fmt", ["ell", "hyb"])
+def test_value_index_bytes_match_oracle(lib, h, nd, fmt):
+    """value_codec 1 (reading R28): the table and the 1-byte (<= 256 distinct)
+    or 2-byte codes are byte-exact against oracle/value_index.py, for the ELL
+    part only in a HYB handle; sizes reported in bro_info_t."""
+    from oracle import value_index
+    A = random_csr(700, 900, 11 + nd, max_len=30, empty_frac=0.1, long_frac=0.05, long_len=120)
+    rng = np.random.default_rng(nd)
+    pool = rng.uniform(-1, 1, nd)
+    for dt in (np.float64, np.float32):
+        vals = pool.astype(dt)[rng.integers(0, nd, A.nnz)]
+        K = hyb.hyb_K(A.row_ptr) if fmt == "hyb" else None
+        create = lib.bro_create_hyb if fmt == "hyb" else lib.bro_create_ell
+        hd = create(HOST, A.m, A.n, A.row_ptr, A.col, vals, lib.bro_opts_default(slice_h=h, value_codec=1))
+        try:
+            info = lib.bro_get_info(hd)
+            codes = lib.bro_export_encoded(hd, "ell_vcodes")
+            D = lib.bro_export_encoded(hd, "ell_vdict", dt)
+        finally:
+            lib.bro_destroy(hd)
+        E = bro_ell.encode(A.row_ptr, A.col, vals, A.m, A.n, h=h, V=1) if K is None else None
+        if K is not None:
+            ep, ec, ev, _, _, _ = hyb.hyb_split(A.row_ptr, A.col, vals, K)
+            E = bro_ell.encode(ep, ec, ev, A.m, A.n, h=h, V=1)
+        Vx = value_index.encode(A.row_ptr, vals, A.m, h, E.num_col, E.colptr, cap=K)
+        assert info["value_code_bytes"] == Vx.cb and info["value_dict_size"] == Vx.dict_bits.size
+        assert np.array_equal(D.view(Vx.dict_bits.dtype), Vx.dict_bits)
+        assert np.array_equal(codes.view(Vx.codes.dtype), Vx.codes)
+        assert info["value_bytes"] >= Vx.codes.nbytes + Vx.dict_bits.nbytes
+
+
+def test_value_index_errors(lib):
+    """More than 65,536 distinct values: BRO_ERR_UNSUPPORTED; value_codec with
+    the uncompressed baseline or out of range: BRO_ERR_ARG."""
+    A = random_csr(4000, 3000, 5, max_len=40)
+    vals = np.arange(A.nnz, dtype=np.float64)
+    assert A.nnz > 65536
+    with pytest.raises(lib.BroError, match="UNSUPPORTED"):
+        lib.bro_create_ell(HOST, A.m, A.n, A.row_ptr, A.col, vals, lib.bro_opts_default(value_codec=1))
+    with pytest.raises(lib.BroError, match="ARG"):
+        lib.bro_create_ell(HOST, A.m, A.n, A.row_ptr, A.col, A.vals, lib.bro_opts_default(value_codec=1, codec=0))
+    with pytest.raises(lib.BroError, match="ARG"):
+        lib.bro_create_ell(HOST, A.m, A.n, A.row_ptr, A.col, A.vals, lib.bro_opts_default(value_codec=2))
