@@ -513,7 +513,7 @@ def main():
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
         with open(tp) as f:
-            tr = json.load(f).get(f"{args.workload}:{args.dtype}:bro:{world}")
+            tr = json.load(f).get(f"{args.workload}:{args.dtype}:bro{':vi' if args.value_codec else ''}:{world}")
         if tr:
             traffic = tr
     value = 2.0 * A.nnz / (total_ms / args.steps * 1e-3) / 1e9
