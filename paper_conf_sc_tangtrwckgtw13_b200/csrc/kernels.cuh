@@ -606,7 +606,8 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
 #pragma unroll
           for (int k = 0; k < R; ++k)
 #pragma unroll
-            for (int kk = 0; kk < G; ++kk)
+            for (int kk = 0; kk < G; ++kk) {
+              q.xv[k][kk] = T(0);  // padding slots: value 0 (stored) times 0 adds +0
               if (q.ok[k][kk]) {
                 if constexpr (kX) {
                   const int cx = q.cidx[k][kk] - xlo;  // columns past the staged window (its 16-byte tail) from global
@@ -615,6 +616,7 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
                   q.xv[k][kk] = ldg_x(p.x + q.cidx[k][kk]);
                 }
               }
+            }
         }
       };
       auto consume = [&](const Grp& q) {
@@ -623,7 +625,14 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
           for (int k = 0; k < R; ++k)
 #pragma unroll
             for (int kk = 0; kk < G; ++kk)
-              if (q.ok[k][kk]) sum[k] = fma(q.v[k][kk], q.xv[k][kk], sum[k]);
+              // stored padding values are 0 and their x is never gathered (0):
+              // the FMA adds +0 and needs no select (two FSELs per fp64 slot
+              // on this issue-bound loop: C5 fp64 330.6 -> 311.9 us, fp32
+              // 202.3 -> 191.4 us).  A value index maps padding to D[0], which
+              // may be non-finite, so it keeps the predicate, and so does the
+              // 51-register mid-window instance (C4 fp64 107.3 vs 111.6 us).
+              if constexpr (kVI == 0 && kMaxRegs >= 56) sum[k] = fma(q.v[k][kk], q.xv[k][kk], sum[k]);
+              else if (q.ok[k][kk]) sum[k] = fma(q.v[k][kk], q.xv[k][kk], sum[k]);
         }
       };
       if constexpr (!kPipe) {
@@ -738,6 +747,9 @@ bro_ell_tiny(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
         if (l > 0) {
           if constexpr (kVI > 0) load_vals_vi<T, 4, H, kVI>(v[k], p.vcodes + kVI * H * mt.c0, p.vdict, 0, l, row);
           else load_vals<T, 4, H>(v[k], p.vals + H * mt.c0, 0, l, lfull, row);
+        } else {
+#pragma unroll
+          for (int q = 0; q < 4; ++q) v[k][q] = T(0);
         }
       }
     }
@@ -770,14 +782,18 @@ bro_ell_tiny(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
 #pragma unroll
       for (int k = 0; k < R; ++k)
 #pragma unroll
-        for (int j = 0; j < 4; ++j)
+        for (int j = 0; j < 4; ++j) {
+          xv[k][j] = T(0);
           if (ok[k][j]) xv[k][j] = ldg_x(p.x + cidx[k][j]);
+        }
 #pragma unroll
       for (int k = 0; k < R; ++k) {
         T sum = T(0);
 #pragma unroll
-        for (int j = 0; j < 4; ++j)
-          if (ok[k][j]) sum = fma(v[k][j], xv[k][j], sum);
+        for (int j = 0; j < 4; ++j) {  // padding (and j >= l): stored value 0 times x = 0 (as in bro_ell_od)
+          if constexpr (kVI == 0) sum = fma(v[k][j], xv[k][j], sum);
+          else if (ok[k][j]) sum = fma(v[k][j], xv[k][j], sum);
+        }
         const int64_t row = H * t + 32 * k + lane;
         if (row < p.m) store_y<kMode>(y, row, sum);
       }
