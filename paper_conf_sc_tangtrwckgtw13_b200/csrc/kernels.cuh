@@ -112,6 +112,18 @@ template <> struct Chunk<float> {
 template <typename T>
 __device__ __forceinline__ T ldg_x(const T* p) { return __ldg(p); }
 
+// A kernel-parameter pointer the compiler must keep in a register: without
+// this it re-loads the x base from the constant bank (LDC) before every
+// predicated gather of the BRO-ELL loop — one extra instruction per slot.
+// (z is a runtime zero: m >> 62 of a row count; an expression of two
+// parameters is not worth re-materialising, so the sum stays in a register)
+template <typename T>
+__device__ __forceinline__ const T* in_reg(const T* p, int64_t z) {
+  const T* r;
+  asm("add.s64 %0, %1, %2;" : "=l"(r) : "l"(p), "l"(z));
+  return r;
+}
+
 // shl / shr with the PTX clamp (shift >= 32 gives 0)
 __device__ __forceinline__ uint32_t shl_clamp(uint32_t v, uint32_t s) {
   uint32_t r;
@@ -467,6 +479,7 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
   }
   bool xready = !kX;
   const char* win_lane = reinterpret_cast<const char*>(win + lane * R);
+  const T* __restrict__ xg = in_reg(p.x, p.m >> 62);
   const int part = kP > 1 ? w % kP : 0;
   __shared__ T psum[kP > 1 ? kWarps : 1][kP > 1 ? H : 1];  // split slices: partial sums per part
   const int64_t stride = int64_t(gridDim.x) * kSl;
@@ -611,9 +624,9 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
               if (q.ok[k][kk]) {
                 if constexpr (kX) {
                   const int cx = q.cidx[k][kk] - xlo;  // columns past the staged window (its 16-byte tail) from global
-                  q.xv[k][kk] = unsigned(cx) < unsigned(xn) ? xs[cx] : ldg_x(p.x + q.cidx[k][kk]);
+                  q.xv[k][kk] = unsigned(cx) < unsigned(xn) ? xs[cx] : ldg_x(xg + q.cidx[k][kk]);
                 } else {
-                  q.xv[k][kk] = ldg_x(p.x + q.cidx[k][kk]);
+                  q.xv[k][kk] = ldg_x(xg + q.cidx[k][kk]);
                 }
               }
             }
@@ -630,7 +643,7 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
               // on this issue-bound loop: C5 fp64 330.6 -> 311.9 us, fp32
               // 202.3 -> 191.4 us).  A value index maps padding to D[0], which
               // may be non-finite, so it keeps the predicate, and so does the
-              // 51-register mid-window instance (C4 fp64 107.3 vs 111.6 us).
+              // 51-register mid-window instance (C4 fp64 99.1 vs 110.0 us).
               if constexpr (kVI == 0 && kMaxRegs >= 56) sum[k] = fma(q.v[k][kk], q.xv[k][kk], sum[k]);
               else if (q.ok[k][kk]) sum[k] = fma(q.v[k][kk], q.xv[k][kk], sum[k]);
         }
@@ -778,13 +791,14 @@ bro_ell_tiny(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
         for (int j = 0; j < 4; ++j)
           if (j < l) dec[H * (mt.c0 + j) + 32 * k + lane] = ok[k][j] ? cidx[k][j] : -1;
     } else {
+      const T* __restrict__ xg = in_reg(p.x, p.m >> 62);
       T xv[R][4];
 #pragma unroll
       for (int k = 0; k < R; ++k)
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
           xv[k][j] = T(0);
-          if (ok[k][j]) xv[k][j] = ldg_x(p.x + cidx[k][j]);
+          if (ok[k][j]) xv[k][j] = ldg_x(xg + cidx[k][j]);
         }
 #pragma unroll
       for (int k = 0; k < R; ++k) {
