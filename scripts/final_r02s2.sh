@@ -2,12 +2,12 @@
 # Round-2 session-2 evidence run (one gpurun call): full GPU suite, smoke,
 # sanitizers, default bench line, every config/dtype (+ value-index and
 # standalone COO lines), launch lists and ncu --set full captures.
-OUT=gpurun_out/r03z; mkdir -p $OUT
+OUT=${OUT:-gpurun_out/r03z}; mkdir -p $OUT
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,clocks.mem,power.draw,clocks_event_reasons.active --format=csv > $OUT/nvidia-smi.txt 2>&1
 python -c "import __graft_entry__ as g; g.build()" > $OUT/build.txt 2>&1 || { tail -30 $OUT/build.txt; exit 1; }
 timeout 2400 python -m pytest tests -m gpu -q -p no:cacheprovider > $OUT/pytest_gpu.txt 2>&1; echo "pytest rc=$?"; tail -3 $OUT/pytest_gpu.txt
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $OUT/smoke.txt 2>&1; echo "smoke rc=$?"; tail -1 $OUT/smoke.txt
-bash scripts/sanitize.sh $OUT/sanitizer
+[ -n "$SANITIZE" ] && bash scripts/sanitize.sh $OUT/sanitizer  # compute-sanitizer is refused on this pool (profiles/r02/s2/final/sanitizer_refused.txt)
 timeout 900 python bench.py > $OUT/bench.json 2> $OUT/bench.err; echo "bench rc=$?"; cut -c1-300 $OUT/bench.json
 summ() { python - "$1" <<'PY'
 import json,sys
