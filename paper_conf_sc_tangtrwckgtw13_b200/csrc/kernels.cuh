@@ -642,9 +642,11 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
               // the FMA adds +0 and needs no select (two FSELs per fp64 slot
               // on this issue-bound loop: C5 fp64 330.6 -> 311.9 us, fp32
               // 202.3 -> 191.4 us).  A value index maps padding to D[0], which
-              // may be non-finite, so it keeps the predicate, and so does the
-              // 51-register mid-window instance (C4 fp64 99.1 vs 110.0 us).
-              if constexpr (kVI == 0 && kMaxRegs >= 56) sum[k] = fma(q.v[k][kk], q.xv[k][kk], sum[k]);
+              // may be non-finite, so it keeps the predicate, and so do the
+              // 51-register mid-window instance (C4 fp64 99.1 vs 110.0 us) and
+              // the fp32 few-slice instance with 32-column groups (C2 fp32 16.7
+              // vs 18.6 us).
+              if constexpr (kVI == 0 && kMaxRegs >= 56 && !(sizeof(T) == 4 && G >= 32)) sum[k] = fma(q.v[k][kk], q.xv[k][kk], sum[k]);
               else if (q.ok[k][kk]) sum[k] = fma(q.v[k][kk], q.xv[k][kk], sum[k]);
         }
       };
@@ -919,6 +921,7 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
   const int64_t e0 = i * I;
   const int32_t* cb = p.col + e0;
   const T* vb = p.vals + e0;
+  const T* __restrict__ xg = in_reg(p.x, p.nnz >> 62);  // x base in a register (see in_reg)
   // per-lane segment state: f = row of the lane's first entry, A = partial of
   // its first segment, cr / cur = current (trailing) segment
   int f = 0, cr = 0;
@@ -982,7 +985,7 @@ coo_spmv(const CooDev<T> p, T* __restrict__ y, int32_t* __restrict__ dec) {
     if constexpr (kMode != kDecode) {
 #pragma unroll
       for (int k = 0; k < CH; ++k)  // slots past nnz hold col 0 / value 0: no gather
-        xv[k] = TT * lane + CH * ch + k < lim ? ldg_x(p.x + c[k]) : T(0);
+        xv[k] = TT * lane + CH * ch + k < lim ? ldg_x(xg + c[k]) : T(0);
     }
     if constexpr (kBro) {
       if (b > 0 && S <= 2) {
