@@ -54,7 +54,7 @@ def parse_args():
     ap.add_argument("--format", default=None, choices=["ell", "hyb", "coo"],
                     help="override the workload's format (e.g. coo: standalone BRO-COO vs COO, Fig. 7)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--vec-words", type=int, default=0, help="0 = auto (fp64: 1, fp32: 4)")
+    ap.add_argument("--vec-words", type=int, default=0, help="0 = auto (1, the paper's multiplexing)")
     ap.add_argument("--slice-h", type=int, default=0, help="BRO-ELL slice height: 0 = auto, 32, 64")
     ap.add_argument("--coo-T", type=int, default=0, help="BRO-COO entries per lane: 0 = auto, 8, 16, 32")
     ap.add_argument("--ell-kernel", type=int, default=0, help="BRO-ELL instance: 0 = auto, 1..7 (A/B only)")

@@ -106,7 +106,7 @@ typedef struct {
   int32_t sym_bits;  /* sym_len. Must be 32. */
   int32_t vec_words; /* V: 1 or 4 symbols per lane chunk.  1 = the paper's multiplexing
                         (comp_str_i[q*h + tid]); 4 = 16-byte per-lane chunks (128-bit loads);
-                        0 (default) = auto: 1 for BRO_FP64, 4 for BRO_FP32. */
+                        0 (default) = auto: 1 for both dtypes (measured fastest on B200). */
   int32_t coo_T;     /* BRO-COO entries per lane of an interval (interval = 32*T entries):
                         8, 16 or 32; 0 (default) = 8 (measured fastest on B200 for both
                         BRO-COO and plain COO: the kernels are latency-bound). */

@@ -570,9 +570,11 @@ bro_status_t common_checks(bro_dtype_t dtype, const bro_opts_t* opts, bro_opts_t
   if (opts) *o = *opts; else bro_opts_default(o);
   bro_status_t st = check_opts(*o);
   if (st) return st;
-  // vec_words 0 = auto: the layout measured fastest for the dtype on B200
-  // (fp64: V = 1, the paper's multiplexing; fp32: V = 4, 16-byte lane chunks)
-  if (o->vec_words == 0) o->vec_words = dtype == BRO_FP64 ? 1 : 4;
+  // vec_words 0 = auto: V = 1, the paper's multiplexing, measured fastest for
+  // both dtypes once the decode loop was cut down (C5 fp32 185 vs 196 us with
+  // V = 4, C3 fp32 22.8 vs 23.4, C4/C2 level; profiles/r02/s2/vec/)
+  if (o->vec_words == 0) o->vec_words = 1;
+  (void)dtype;
   return BRO_OK;
 }
 
