@@ -145,7 +145,8 @@ typedef struct {
                         1-byte (<= 256 distinct) or 2-byte (<= 65,536) code per slot,
                         slot (r, j) of slice t at h*colptr[t] + place(r, j, l_t, 4/cb, h).
                         Lossless bit for bit.  More than 65,536 distinct values gives
-                        BRO_ERR_UNSUPPORTED.  Value-indexed ELL handles have no scatter
+                        BRO_ERR_UNSUPPORTED; on a COO handle, BRO_ERR_ARG.  Value-indexed
+                        ELL handles have no scatter
                         epilogue (bro_spmv_scatter with more than one destination gives
                         BRO_ERR_UNSUPPORTED); the COO part of a HYB handle keeps its values. */
 } bro_opts_t;

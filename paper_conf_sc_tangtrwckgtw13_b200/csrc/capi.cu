@@ -877,6 +877,7 @@ bro_status_t bro_create_coo(int device, bro_dtype_t dtype, int64_t m, int64_t n,
   bro_opts_t o;
   bro_status_t st = common_checks(dtype, opts, &o, out);
   if (st) return st;
+  if (o.value_codec) return fail(BRO_ERR_ARG, "value_codec indexes BRO-ELL values: ELL and HYB handles only");
   std::string msg = bro::check_coo(m, n, nnz, row_idx, col_idx);
   if (!msg.empty()) return fail(msg.rfind("shape", 0) == 0 ? BRO_ERR_SHAPE : BRO_ERR_INDEX, msg);
   if (nnz > 0 && !vals) return fail(BRO_ERR_ARG, "vals is NULL");
