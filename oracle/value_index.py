@@ -16,7 +16,10 @@ short index per stored value.  Written step by step:
      the values in the BRO-ELL slot layout (R7), grouped per row in 4-byte
      chunks of Vc = 4 / cb codes: slot (r, j) of slice t is code
         vcodes[h * colptr[t] + place(r, j, l_t, Vc, h)]
-     (the multiplexing of P:L116 with 4-byte chunks); padding slots hold 0.
+     (the multiplexing of P:L116 with 4-byte chunks); padding slots hold pz,
+     the code of the first FINITE value of D (a padding slot's x is never
+     gathered, so its product is a finite value times 0 = 0, reading R30);
+     a part with no finite value is not indexed (None).
   4. y_i = sum_j D[code_ij] * x[c_ij] in slot order: the same products as with
      the stored values, bit for bit.
 """
@@ -40,6 +43,7 @@ class ValueIndex:
     dict_vals: np.ndarray   # the same, as values
     cb: int                 # step 2: bytes per code
     codes: np.ndarray       # step 3: uint8 / uint16[h*colptr[s]] in the 4-byte-chunk slot layout
+    pz: int = 0             # step 3: padding code (first finite value of D)
 
 
 def distinct(vals: np.ndarray):
@@ -55,6 +59,12 @@ def distinct(vals: np.ndarray):
     return D, D.view(vals.dtype), cb
 
 
+def padding_code(Dv: np.ndarray):
+    """Step 3's pz: index of the first finite value of D (None if none is)."""
+    fin = np.nonzero(np.isfinite(Dv))[0]
+    return int(fin[0]) if fin.size else (0 if Dv.size == 0 else None)
+
+
 def encode(row_ptr, vals, m, h, num_col, colptr, cap=None) -> ValueIndex | None:
     """Steps 1-3 for the BRO-ELL part whose slices have num_col / colptr (from
     oracle.bro_ell.encode); row i contributes its first min(len_i, cap) values."""
@@ -68,8 +78,11 @@ def encode(row_ptr, vals, m, h, num_col, colptr, cap=None) -> ValueIndex | None:
     if got is None:
         return None
     D, Dv, cb = got
+    pz = padding_code(Dv)
+    if pz is None:
+        return None
     Vc = 4 // cb
-    codes = np.zeros(h * int(colptr[-1]), dtype=np.uint8 if cb == 1 else np.uint16)
+    codes = np.full(h * int(colptr[-1]), pz, dtype=np.uint8 if cb == 1 else np.uint16)
     pos = {int(b): k for k, b in enumerate(D)}
     bits = _bits(vals)
     s = len(num_col)
@@ -83,12 +96,12 @@ def encode(row_ptr, vals, m, h, num_col, colptr, cap=None) -> ValueIndex | None:
             a = int(row_ptr[row])
             for j in range(int(lens[row])):
                 codes[base + place(r, j, l, Vc, h)] = pos[int(bits[a + j])]
-    return ValueIndex(D, Dv, cb, codes)
+    return ValueIndex(D, Dv, cb, codes, pz)
 
 
 def slot_values(V: ValueIndex, h, num_col, colptr, Vv) -> np.ndarray:
     """Step 4's lookup, re-laid out in the value slot layout (chunks of Vv):
-    D[code] of every slot (padding slots: D[0]).  Equal, bit for bit, to the
+    D[code] of every slot (padding slots: D[pz]).  Equal, bit for bit, to the
     BRO-ELL values at every non-padding slot (round-trip pin)."""
     out = np.zeros(h * int(colptr[-1]), dtype=V.dict_vals.dtype)
     Vc = 4 // V.cb

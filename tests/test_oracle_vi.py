@@ -95,3 +95,19 @@ def test_cap_takes_the_ell_part_only():
     assert [float(v) for v in V.dict_vals] == [5.0, 6.0, 7.0]
     assert V.codes.tolist() == [0, 1, 2, 0]
     del E
+
+
+def test_padding_code_is_first_finite_value():
+    """Padding slots hold pz, the code of the first finite value of D (a
+    padding product is then a finite value times 0): D = [+inf, -1.0]
+    (0x7FF0... < 0xBFF0... as unsigned) gives pz = 1; a part whose values are
+    all non-finite is not indexed."""
+    rp = np.array([0, 1, 3])
+    col = np.array([0, 0, 1], dtype=np.int32)
+    vals = np.array([np.inf, -1.0, np.inf])
+    E = bro_ell.encode(rp, col, vals, 2, 2, h=2, sym_len=32, V=1)
+    V = vi.encode(rp, vals, 2, 2, E.num_col, E.colptr)
+    assert [float(v) for v in V.dict_vals] == [np.inf, -1.0] and V.pz == 1
+    # slice l = 2, tail layout: row 0 [inf, pad], row 1 [-1, inf]
+    assert V.codes.tolist() == [0, 1, 1, 0]
+    assert vi.encode(rp, np.array([np.inf, np.nan, -np.inf]), 2, 2, E.num_col, E.colptr) is None
