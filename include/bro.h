@@ -143,8 +143,10 @@ typedef struct {
                         P:L408; reading R28): the ELL part's distinct value
                         bit patterns (sorted as unsigned integers) in a table and one
                         1-byte (<= 256 distinct) or 2-byte (<= 65,536) code per slot,
-                        slot (r, j) of slice t at h*colptr[t] + place(r, j, l_t, 4/cb, h).
-                        Lossless bit for bit.  More than 65,536 distinct values gives
+                        slot (r, j) of slice t at h*colptr[t] + place(r, j, l_t, 4/cb, h);
+                        padding slots hold the code of the first finite value of the
+                        table.  Lossless bit for bit.  More than 65,536 distinct values, or
+                        no finite value at all, gives
                         BRO_ERR_UNSUPPORTED; on a COO handle, BRO_ERR_ARG.  Value-indexed
                         ELL handles have no scatter
                         epilogue (bro_spmv_scatter with more than one destination gives

@@ -388,9 +388,13 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
         A->ell_max_l = A->ell.max_l;
         for (int64_t t = 0; t < A->s; ++t)
           A->ell_max_S = std::max<int64_t>(A->ell_max_S, int64_t(A->ell.symptr[t + 1] - A->ell.symptr[t]));
-        if (o.value_codec == 1 && !bro::encode_value_index(rv, A->ell, A->vi)) {
-          delete A;
-          return fail(BRO_ERR_UNSUPPORTED, "value_codec 1: the BRO-ELL part holds more than 65,536 distinct values");
+        if (o.value_codec == 1) {
+          const int vr = bro::encode_value_index(rv, A->ell, A->vi);
+          if (vr) {
+            delete A;
+            return fail(BRO_ERR_UNSUPPORTED, vr == 1 ? "value_codec 1: the BRO-ELL part holds more than 65,536 distinct values"
+                                                     : "value_codec 1: the BRO-ELL part holds no finite value");
+          }
         }
       } else {
         bro::build_plain_ell(rv, K, A->pell);
@@ -643,7 +647,7 @@ cudaError_t launch_ell(const bro_matrix_s* A, int mode, const T* x, const bro::d
   if (A->opts.codec) {
     bro::dev::EllDev<T> p{r1 - r0, b1 - b0, A->d_words, A->d_bit_alloc, A->d_colptr + b0, A->d_symptr + b0,
                           static_cast<const T*>(A->d_ell_vals), x, A->d_xwin, A->d_vcodes,
-                          static_cast<const T*>(A->d_vdict)};
+                          static_cast<const T*>(A->d_vdict), uint32_t(A->vi.pz)};
     if (!L.k.fn) return cudaErrorNotSupported;  // scatter on a value-indexed handle
     // whole part, plain SpMV, 16-byte aligned x: the x-window-staged instance
     if (A->xstage && mode == 0 && b0 == 0 && b1 == A->s && (reinterpret_cast<uintptr_t>(x) & 15) == 0) {

@@ -216,7 +216,7 @@ void encode_bro_ell(const RowsView& A, int h, int V, int VV, int min_bits, EllCo
 }
 
 template <typename U>
-static bool value_index_impl(const RowsView& A, const EllCode& E, ValueIndexCode& out) {
+static int value_index_impl(const RowsView& A, const EllCode& E, ValueIndexCode& out) {
   constexpr size_t kMaxD = 65536;
   const int64_t m = A.m;
   const int nt = num_threads();
@@ -240,20 +240,31 @@ static bool value_index_impl(const RowsView& A, const EllCode& E, ValueIndexCode
   }
   std::unordered_set<U> all;
   for (int c = 0; c < nt; ++c) {
-    if (over[c]) return false;
+    if (over[c]) return 1;
     all.insert(sets[c].begin(), sets[c].end());
-    if (all.size() > kMaxD) return false;
+    if (all.size() > kMaxD) return 1;
   }
   std::vector<U> D(all.begin(), all.end());
   std::sort(D.begin(), D.end());  // ascending as unsigned integers
+  // padding code: the first finite value (exponent field not all ones)
+  constexpr U kExp = sizeof(U) == 8 ? U(0x7FF0000000000000ull) : U(0x7F800000u);
+  size_t pz = 0;
+  while (pz < D.size() && (D[pz] & kExp) == kExp) ++pz;
+  if (!D.empty() && pz == D.size()) return 2;
+  if (D.empty()) pz = 0;
   const int cb = D.size() <= 256 ? 1 : 2;
   const int64_t VC = 4 / cb;
   const int64_t h = E.h, s = E.s;
   out.cb = cb;
   out.nd = int64_t(D.size());
+  out.pz = uint32_t(pz);
   out.dict.resize(D.size() * sizeof(U));
   if (!D.empty()) std::memcpy(out.dict.data(), D.data(), D.size() * sizeof(U));
   out.codes.assign(size_t(cb) * h * E.colptr[s], 0);
+  for (size_t i = 0; i < out.codes.size(); i += size_t(cb)) {  // every slot starts as padding
+    out.codes[i] = uint8_t(pz);
+    if (cb == 2) out.codes[i + 1] = uint8_t(pz >> 8);
+  }
   parallel_for(s, [&](int64_t lo, int64_t hi) {
     for (int64_t t = lo; t < hi; ++t) {
       const int64_t l = int64_t(E.colptr[t + 1] - E.colptr[t]);
@@ -271,10 +282,10 @@ static bool value_index_impl(const RowsView& A, const EllCode& E, ValueIndexCode
       }
     }
   });
-  return true;
+  return 0;
 }
 
-bool encode_value_index(const RowsView& A, const EllCode& E, ValueIndexCode& out) {
+int encode_value_index(const RowsView& A, const EllCode& E, ValueIndexCode& out) {
   return A.vsize == 8 ? value_index_impl<uint64_t>(A, E, out) : value_index_impl<uint32_t>(A, E, out);
 }
 

@@ -71,6 +71,7 @@ struct CooCode {
 struct ValueIndexCode {
   int cb = 0;                     // 1 or 2 bytes per code
   int64_t nd = 0;                 // |D|
+  uint32_t pz = 0;                // padding code: the first finite value of D (reading R28)
   Bytes dict;                     // nd values (bit patterns ascending)
   std::vector<uint8_t> codes;     // cb*h*colptr[s] bytes, little-endian codes
 };
@@ -99,9 +100,9 @@ std::string check_coo(int64_t m, int64_t n, int64_t nnz, const int32_t* row, con
 int64_t hyb_K(int64_t m, const int64_t* row_ptr);
 
 void encode_bro_ell(const RowsView& A, int h, int V, int value_chunk, int min_bits, EllCode& out);
-// Value index of the BRO-ELL part E of A; false (out untouched) if the part
-// holds more than 65,536 distinct values.
-bool encode_value_index(const RowsView& A, const EllCode& E, ValueIndexCode& out);
+// Value index of the BRO-ELL part E of A: 0 = done, 1 = more than 65,536
+// distinct values, 2 = no finite value (out untouched unless 0).
+int encode_value_index(const RowsView& A, const EllCode& E, ValueIndexCode& out);
 // Longest slice (columns) and longest row stream (32-bit symbols) of the
 // BRO-ELL encoding at slice height h, without packing anything.
 void slice_extents(const RowsView& A, int h, int min_bits, int64_t* max_l, int64_t* max_S);

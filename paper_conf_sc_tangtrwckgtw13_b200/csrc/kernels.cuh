@@ -196,6 +196,7 @@ struct EllDev {           // a BRO-ELL part (or a range of its slices)
   const int2* xwin;       // x-staged instances: per block, {first column, columns} of its x window
   const uint8_t* vcodes;  // value-indexed handles (reading R28): codes in the slot layout, 4-byte chunks
   const T* vdict;         // ... and the table of distinct values they index
+  uint32_t vpad;          // ... and the code of padding slots (a finite value, reading R28)
 };
 
 // ------------------------------------------------------------------ TMA bulk copy + mbarrier
@@ -297,8 +298,8 @@ __device__ __forceinline__ uint32_t ld_code(const uint8_t* p) {
   return r;
 }
 template <typename T, int G, int H, int CB>
-__device__ __forceinline__ void load_vals_vi(T* v, const uint8_t* cs, const T* __restrict__ dict, int j, int l,
-                                             int r) {
+__device__ __forceinline__ void load_vals_vi(T* v, const uint8_t* cs, const T* __restrict__ dict, uint32_t pad,
+                                             int j, int l, int r) {
   constexpr int VC = 4 / CB;
   static_assert(G % VC == 0, "a column group holds whole 4-byte code chunks");
   const int lfull = (l / VC) * VC;
@@ -321,7 +322,7 @@ __device__ __forceinline__ void load_vals_vi(T* v, const uint8_t* cs, const T* _
       } else {
 #pragma unroll
         for (int k = 0; k < VC; ++k)
-          code[u * VC + k] = jj + k < l ? ld_code<CB>(cs + CB * (H * lfull + r * tw + (jj + k - lfull))) : 0u;
+          code[u * VC + k] = jj + k < l ? ld_code<CB>(cs + CB * (H * lfull + r * tw + (jj + k - lfull))) : pad;
       }
     }
   }
@@ -575,7 +576,7 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
         if constexpr (kMode != kDecode) {
 #pragma unroll
           for (int k = 0; k < R; ++k) {
-            if constexpr (kVI > 0) load_vals_vi<T, G, H, kVI>(q.v[k], vcs, p.vdict, jb + g, l, 32 * k + lane);
+            if constexpr (kVI > 0) load_vals_vi<T, G, H, kVI>(q.v[k], vcs, p.vdict, p.vpad, jb + g, l, 32 * k + lane);
             else load_vals<T, G, H>(q.v[k], vs, jb + g, l, lfull, 32 * k + lane);
           }
         }
@@ -641,12 +642,12 @@ bro_ell_od(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
               // stored padding values are 0 and their x is never gathered (0):
               // the FMA adds +0 and needs no select (two FSELs per fp64 slot
               // on this issue-bound loop: C5 fp64 330.6 -> 311.9 us, fp32
-              // 202.3 -> 191.4 us).  A value index maps padding to D[0], which
-              // may be non-finite, so it keeps the predicate, and so do the
-              // 51-register mid-window instance (C4 fp64 99.1 vs 110.0 us) and
-              // the fp32 few-slice instance with 32-column groups (C2 fp32 16.7
-              // vs 18.6 us).
-              if constexpr (kVI == 0 && kMaxRegs >= 56 && !(sizeof(T) == 4 && G >= 32)) sum[k] = fma(q.v[k][kk], q.xv[k][kk], sum[k]);
+              // 202.3 -> 191.4 us; value-indexed C5 fp64 303.7 -> 273.6 us: its
+              // padding code is a finite value, reading R28).  The predicate
+              // stays in the 51-register mid-window instance (C4 fp64 99.1 vs
+              // 110.0 us) and the fp32 few-slice instance with 32-column groups
+              // (C2 fp32 16.7 vs 18.6 us).
+              if constexpr (kMaxRegs >= 56 && !(sizeof(T) == 4 && G >= 32)) sum[k] = fma(q.v[k][kk], q.xv[k][kk], sum[k]);
               else if (q.ok[k][kk]) sum[k] = fma(q.v[k][kk], q.xv[k][kk], sum[k]);
         }
       };
@@ -760,7 +761,7 @@ bro_ell_tiny(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
       wd[k][4] = 0u;
       if constexpr (kMode != kDecode) {
         if (l > 0) {
-          if constexpr (kVI > 0) load_vals_vi<T, 4, H, kVI>(v[k], p.vcodes + kVI * H * mt.c0, p.vdict, 0, l, row);
+          if constexpr (kVI > 0) load_vals_vi<T, 4, H, kVI>(v[k], p.vcodes + kVI * H * mt.c0, p.vdict, p.vpad, 0, l, row);
           else load_vals<T, 4, H>(v[k], p.vals + H * mt.c0, 0, l, lfull, row);
         } else {
 #pragma unroll
@@ -807,8 +808,7 @@ bro_ell_tiny(const EllDev<T> p, const YOut<T> y, int32_t* __restrict__ dec) {
         T sum = T(0);
 #pragma unroll
         for (int j = 0; j < 4; ++j) {  // padding (and j >= l): stored value 0 times x = 0 (as in bro_ell_od)
-          if constexpr (kVI == 0) sum = fma(v[k][j], xv[k][j], sum);
-          else if (ok[k][j]) sum = fma(v[k][j], xv[k][j], sum);
+          sum = fma(v[k][j], xv[k][j], sum);
         }
         const int64_t row = H * t + 32 * k + lane;
         if (row < p.m) store_y<kMode>(y, row, sum);

@@ -341,6 +341,19 @@ def test_configs_full_oracle(lib, dev, cfg, fmt, codec):
         M.close()
 
 
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_config4_bench_input(lib, dev, dtype):
+    """C4 exactly as bench.py builds it (BAR method 3, reading R27, for this
+    dtype) in bench.py's handle configuration: BRO-HYB on every row vs the
+    oracle, every ELL slot and COO row decoded bit-exactly."""
+    import bench
+    A, fmt = bench.load_workload("C4", dtype, lib)
+    M, x, y = _run(lib, A, fmt, 1, dtype, dev, x=make_x(A.n, 4, dtype))
+    _check_y(A, x, y, dtype)
+    check_decode(M, A)
+    M.close()
+
+
 def test_config4_bar_reordered_hyb(lib, dev):
     """C4: random-block, reordered with BAR (signature clustering), BRO-HYB
     fp32 and fp64 vs the oracle on every row, every index decoded."""
@@ -500,6 +513,35 @@ def test_value_index_instances(lib, dev, inst, h, V, dtype):
             assert np.array_equal(y.view(np.uint8), yp.view(np.uint8)), f"{name} {fmt}: not bit-identical"
             ran += 1
     assert ran > 0
+
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_value_index_nonfinite_table(lib, dev, dtype):
+    """A table whose first entry is +inf (D = [+inf, -1.0, -2.0] as unsigned
+    bit patterns 0x7FF0.. < 0xBFF0.. < 0xC000..): padding slots take the first
+    finite code (reading R28), so ragged rows give the same bits as the
+    stored-values handle, non-finite rows included; finite rows within the
+    oracle's bound."""
+    A = random_csr(3000, 2500, 31, max_len=20, empty_frac=0.1)
+    rng = np.random.default_rng(5)
+    vals = np.array([np.inf, -1.0, -2.0], dtype=dtype)[rng.choice(3, A.nnz, p=[0.01, 0.49, 0.5])]
+    A = Csr(A.m, A.n, A.row_ptr, A.col, vals, "inf-table")
+    x = make_x(A.n, 2, dtype)
+    for inst in (0, 1, 5):
+        for h in (32, 64):
+            if inst == 1:
+                continue
+            M, _, y = _run(lib, A, "ell", 1, dtype, dev, x=x, slice_h=h, ell_kernel=inst, value_codec=1)
+            assert M.info["value_dict_size"] == 3
+            M.close()
+            P, _, yp = _run(lib, A, "ell", 1, dtype, dev, x=x, slice_h=h, ell_kernel=inst)
+            P.close()
+            assert np.array_equal(y.view(np.uint8), yp.view(np.uint8))
+    fin = np.array([np.isfinite(vals[A.row_ptr[i]:A.row_ptr[i + 1]]).all() for i in range(A.m)])
+    with np.errstate(invalid="ignore"):  # the inf rows make NaNs in the oracle too
+        y_ref, S = spmv.csr_spmv(A.row_ptr, A.col, A.vals, x)
+    ok, _ = spmv.within_tolerance(y[fin], np.asarray(y_ref)[fin], np.asarray(S)[fin], TOL[dtype])
+    assert ok.all() and not np.isfinite(y[~fin]).any()
 
 
 def test_value_index_scatter_rejected(lib, dev):

@@ -537,6 +537,8 @@ def test_value_index_errors(lib):
         lib.bro_create_ell(HOST, A.m, A.n, A.row_ptr, A.col, A.vals, lib.bro_opts_default(value_codec=1, codec=0))
     with pytest.raises(lib.BroError, match="ARG"):
         lib.bro_create_ell(HOST, A.m, A.n, A.row_ptr, A.col, A.vals, lib.bro_opts_default(value_codec=2))
+    with pytest.raises(lib.BroError, match="UNSUPPORTED"):  # no finite value for the padding code
+        lib.bro_create_ell(HOST, A.m, A.n, A.row_ptr, A.col, np.full(A.nnz, np.inf), lib.bro_opts_default(value_codec=1))
     rows = np.repeat(np.arange(A.m, dtype=np.int32), np.diff(A.row_ptr))
     with pytest.raises(lib.BroError, match="ARG"):  # COO handles have no BRO-ELL values to index
         lib.bro_create_coo(HOST, A.m, A.n, rows, A.col, A.vals, lib.bro_opts_default(value_codec=1))
