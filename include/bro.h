@@ -101,7 +101,7 @@ typedef struct {
                         auto: 64 when m >= 303,104 (64 rows x 32 resident warps x 148
                         SMs: every resident warp of a B200 still gets slices), some
                         row of the ELL part has more than 4 entries and, at h = 32,
-                        every row stream has fewer than 10 symbols; else 32.
+                        every row stream has fewer than 18 symbols; else 32.
                         bro_info_t.slice_h reports the value. */
   int32_t sym_bits;  /* sym_len. Must be 32. */
   int32_t vec_words; /* V: 1 or 4 symbols per lane chunk.  1 = the paper's multiplexing

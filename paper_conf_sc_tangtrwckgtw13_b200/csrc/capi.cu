@@ -359,15 +359,16 @@ bro_status_t build(int device, bro_dtype_t dtype, int64_t m, int64_t n, const in
   if (o.codec && o.slice_h) {
     A->h = o.slice_h;
   } else if (o.codec && m >= kAutoH64Rows && format != FMT_COO) {
-    // h = 64 for big matrices whose rows fit the small-window instance at
-    // h = 32 (every row stream < 10 symbols) and are not tiny: two rows per
-    // lane then share the widths, offsets and setup (C5 fp32 247 -> 203 us);
-    // longer row streams (C4: up to 14 symbols) run faster at h = 32
+    // h = 64 for big matrices whose rows fit the small- or mid-window
+    // instance at h = 32 (every row stream < 18 symbols) and are not tiny:
+    // two rows per lane then share the widths, offsets and setup (C5 fp32
+    // 247 -> 203 us; C4 fp64 99.7 -> 97.3 us since the decode-loop cuts,
+    // profiles/r02/s2/c4/)
     bro::RowsView rv;
     rv.m = m; rv.row_ptr = row_ptr; rv.col = col; rv.vsize = A->vsize; rv.cap = K;
     int64_t max_l = 0, max_S = 0;
     bro::slice_extents(rv, 32, o.min_bits, &max_l, &max_S);
-    A->h = max_l > bro::kEllTinyCols && max_S < bro::kEllRowsSmall ? 64 : 32;
+    A->h = max_l > bro::kEllTinyCols && max_S < bro::kEllRowsMid ? 64 : 32;
   }
   A->opts.slice_h = A->h;
   const uint8_t* v8 = static_cast<const uint8_t*>(vals);

@@ -459,18 +459,18 @@ def test_bar_window_improves_eta_over_scrambled(lib):
 @pytest.mark.slow
 def test_auto_slice_height(lib):
     """slice_h = 0: 64 only for big matrices (>= 303,104 rows) that are not
-    tiny and whose h = 32 row streams fit the small window (< 10 symbols,
-    the oracle's slice shapes): C5 -> 64; C4 (up to 14 symbols) -> 32; C3
+    tiny and whose h = 32 row streams fit the mid window (< 18 symbols,
+    the oracle's slice shapes): C5 -> 64; C4 (up to 14 symbols) -> 64; C3
     (ELL part of <= 2 entries per row) -> 32; C2 (62K rows) -> 32."""
     from gen import permute_rows
-    for cfg, fmt, want in ((5, "ell", 64), (4, "hyb", 32), (3, "hyb", 32), (2, "ell", 32)):
+    for cfg, fmt, want in ((5, "ell", 64), (4, "hyb", 64), (3, "hyb", 32), (2, "ell", 32)):
         A = make_config(cfg)
         if cfg == 4:
             A = permute_rows(A, lib.bro_reorder_bar(A.m, A.n, A.row_ptr, A.col, method=0))
         K = hyb.hyb_K(A.row_ptr) if fmt == "hyb" else int(A.row_lengths().max())
         ep, ec, _, _, _, _ = hyb.hyb_split(A.row_ptr, A.col, A.vals, K)
         l, S, _ = bro_ell.slice_shapes(ep, ec, A.m, 32, 32)
-        expect = 64 if (A.m >= 303104 and l.max() > 4 and S.max() < 10) else 32
+        expect = 64 if (A.m >= 303104 and l.max() > 4 and S.max() < 18) else 32
         assert expect == want, (cfg, l.max(), S.max())
         create = lib.bro_create_hyb if fmt == "hyb" else lib.bro_create_ell
         h = create(HOST, A.m, A.n, A.row_ptr, A.col, A.vals)
