@@ -34,7 +34,7 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 60 --cs
 python scripts/launch_summary.py $OUT/launches_C5.csv | tee $OUT/launches_C5_summary.txt
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 40 --csv --log-file $OUT/launches_C4.csv \
   python scripts/prof_one.py C4 f64 "" --launches 10 > /dev/null 2>&1; python scripts/launch_summary.py $OUT/launches_C4.csv | tee $OUT/launches_C4_summary.txt
-for v in "C5 f64 slice_h=64" "C5 f32 slice_h=64" "C5 f64 value_codec=1" "C4 f64 slice_h=32" ; do
+for v in "C5 f64 slice_h=64" "C5 f32 slice_h=64" "C5 f64 value_codec=1" "C4 f64 slice_h=64" ; do
   set -- $v; tag=${1}_${2}_$(echo $3 | tr '=,' '__')
   timeout 900 ncu --set full --clock-control none --import-source on -s 3 -c 3 -o $OUT/full_$tag python scripts/prof_one.py $1 $2 "$3" > $OUT/ncu_$tag.log 2>&1; echo "ncu $tag rc=$?"
   python scripts/ncu_summary.py $OUT/full_$tag.ncu-rep 12 > $OUT/ncu_$tag.txt 2>&1; grep -E "Kernel Name|gpu__time|dram__bytes" $OUT/ncu_$tag.txt
